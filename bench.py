@@ -1,0 +1,437 @@
+#!/usr/bin/env python
+"""Benchmark of the per-batch view materialisation path (BASELINE.json metric:
+output frames/s per GPU & box at 1/2/4/8 B200; HBM GB/s vs peak).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config k400] [--impl sand|reference]
+    torchrun --nproc-per-node N --master-addr 127.0.0.1 bench.py --gpus N ...
+
+A step = one read_batch (all §8(a) rows) of one batch per rank. Inputs are
+resident in HBM (a replicated synthetic store per GPU, far larger than L2) when
+the timed region starts; the timed region is bracketed by barrier +
+synchronize, timed with CUDA events on the read stream, max over ranks. Rank 0
+prints ONE JSON line. `--impl reference` times the CPU oracle (the reference
+arm for this paper: SAND's own engine is CPU code) on the same config.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+DEFAULT_STEPS = {"tiny": 2000, "k400": 3000, "slowfast": 3000, "twoview": 1000, "ray": 1000}
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+# ------------------------------------------------------------------ clocks (nvidia-smi during the timed region)
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "20"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.05)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                smax.append(float(parts[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        sm.sort()
+        return {"sm_mhz": sm[len(sm) // 2] if sm else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------ peaks
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy read+write)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic(config: str):
+    """DRAM bytes per launch of the dominant kernel from the committed ncu --set full summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        if config in d:
+            return d[config].get("dram_bytes_per_launch")
+    return None
+
+
+# ------------------------------------------------------------------ the oracle (cpu_baseline / reference arm)
+def oracle_frames_per_second(workload, spec, vids, n_frames_target: int | None, seconds: float, family, seed,
+                             warmup: int = 0):
+    """Render output frames of batch (epoch 0, rank 0, it 0) with the oracle, one by one.
+
+    Returns (frames, elapsed_s). Stops after n_frames_target frames, else after `seconds`.
+    """
+    import oracle
+    import synth
+    ospec = _oracle_spec(spec)
+    ods = oracle.make_dataset(vids)
+    metas = oracle.plan_batch(ospec, ods, len(vids), 0, 0, 0)
+    W, H = workload.width, workload.height
+    order = [(b, k, t) for b in range(spec.batch_size) for k, v in enumerate(spec.views) for t in range(v.clip_len)]
+    frames_cache = {}
+
+    def src(video, frame):
+        key = (video, frame)
+        if key not in frames_cache:
+            y, uv = synth.frames(family, seed, video, frame, 1, W, H)
+            frames_cache[key] = (y[0], uv[0])
+        return frames_cache[key]
+
+    # pre-generate the source frames (input generation is not the oracle's work)
+    need = order if n_frames_target is None else [order[i % len(order)] for i in range(n_frames_target + warmup)]
+    for b, k, t in need[: min(len(need), 4 * len(order))]:
+        src(metas[b].video, metas[b].frames[k][t])
+    for i in range(warmup):
+        b, k, t = order[i % len(order)]
+        y, uv = src(metas[b].video, metas[b].frames[k][t])
+        oracle.render_frame(ospec, metas[b], k, y, uv)
+    done = 0
+    t0 = time.perf_counter()
+    i = warmup
+    while True:
+        if n_frames_target is not None and done >= n_frames_target:
+            break
+        if n_frames_target is None and time.perf_counter() - t0 >= seconds:
+            break
+        b, k, t = order[i % len(order)]
+        y, uv = src(metas[b].video, metas[b].frames[k][t])
+        oracle.render_frame(ospec, metas[b], k, y, uv)
+        done += 1
+        i += 1
+    return done, time.perf_counter() - t0
+
+
+def _oracle_spec(spec):
+    import oracle
+    views = [oracle.ViewDesc(clip_len=v.clip_len, stride=v.stride, pool_offset=v.pool_offset,
+                             spatial_group=v.spatial_group, geom=v.geom, scale=v.scale, ratio=v.ratio,
+                             short_side=v.short_side, out_h=v.out_h, out_w=v.out_w, flip_p=v.flip_p,
+                             rot_p=v.rot_p, rot_max_deg=v.rot_max_deg, blur_p=v.blur_p, sigma=v.sigma,
+                             blur_ksize=v.blur_ksize, blur_truncate=v.blur_truncate, mean=v.mean, std=v.std,
+                             out_dtype=v.out_dtype) for v in spec.views]
+    return oracle.make_spec(oracle.SpecDesc(seed=spec.seed, world_size=spec.world_size,
+                                            batch_size=spec.batch_size, samples_per_video=spec.samples_per_video,
+                                            drop_last=spec.drop_last, shared_window=spec.shared_window,
+                                            views=views))
+
+
+def frames_per_step(spec):
+    return spec.batch_size * sum(v.clip_len for v in spec.views)
+
+
+def config_dict(workload, spec, n_store_videos):
+    v0 = spec.views[0]
+    return {"workload": workload.name, "batch_per_rank": spec.batch_size,
+            "views": [{"T": v.clip_len, "stride": v.stride, "out": [v.out_h, v.out_w], "group": v.spatial_group,
+                       "geom": "rrc" if v.geom == 0 else "shortside", "rot_p": v.rot_p, "blur_p": v.blur_p}
+                      for v in spec.views],
+            "source": [workload.width, workload.height], "store_videos_per_gpu": n_store_videos,
+            "frames_per_video": workload.n_frames, "shared_window": bool(spec.shared_window),
+            "out_dtype": {0: "u8", 1: "bf16", 2: "f32"}[v0.out_dtype],
+            "l2": "inputs larger than L2: replicated store of %.1f GB per GPU, fresh clips every step, "
+                  "per-step output > L2 for all but tiny" % (n_store_videos * workload.n_frames *
+                                                              workload.frame_bytes / 1e9)}
+
+
+# ------------------------------------------------------------------ reference arm
+def run_reference(args):
+    rank, world, local = dist_env()
+    if rank != 0:
+        return 0
+    from paper_conf_sosp_yelllhkh25_b200 import configs
+    import synth
+    w = configs.get(args.config)
+    spec = w.spec
+    spec.world_size = 1
+    vids = [(1000 + i, w.n_frames, w.width, w.height) for i in range(w.n_videos)]
+    steps, warm = args.steps, args.warmup
+    done, el = oracle_frames_per_second(w, spec, vids, steps, 0.0, synth.UNIFORM, 1234, warmup=warm)
+    value = done / el
+    line = {"impl": "reference", "metric": "output frames/s", "value": value, "unit": "frames/s",
+            "n_gpus": args.gpus, "steps": steps, "warmup": warm, "ms_per_step": 1000.0 * el / max(done, 1),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8/fp32 (oracle)",
+            "data": "synthetic", "config": config_dict(w, spec, w.n_videos),
+            "cpu_baseline": {"value": value, "unit": "frames/s", "cores": 1, "kind": "oracle",
+                             "sample": f"one output frame per step: {done} frames of batch (epoch 0, rank 0, it 0), "
+                                       f"single-threaded C oracle"},
+            "e2e": {"value": value, "unit": "frames/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ our arm
+def run_sand(args):
+    import torch
+    import torch.distributed as dist
+
+    import synth
+    import paper_conf_sosp_yelllhkh25_b200 as sand
+    from paper_conf_sosp_yelllhkh25_b200 import configs
+
+    rank, world, local = dist_env()
+    if world != args.gpus:
+        log(f"warning: --gpus {args.gpus} but WORLD_SIZE={world}; using WORLD_SIZE")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    w = configs.get(args.config)
+    spec = w.spec
+    spec.world_size = world
+    n_videos = w.n_videos if args.videos is None else args.videos
+    vids = [(1000 + i, w.n_frames, w.width, w.height) for i in range(n_videos)]
+    pitch = (w.width + 63) // 64 * 64
+    frame_stride = (pitch * w.height * 3 // 2 + 255) // 256 * 256
+    cap = n_videos * w.n_frames * frame_stride + (64 << 20)
+    t0 = time.time()
+    store = sand.Store(local, cap)
+    stream = torch.cuda.Stream(local)
+    with torch.cuda.stream(stream):
+        synth.fill_store(store, vids, synth.UNIFORM, 1234, stream.cuda_stream)
+    stream.synchronize()
+    log(f"[rank {rank}] store filled: {n_videos} videos, {cap / 1e9:.1f} GB in {time.time() - t0:.1f}s")
+    view = sand.View(store, spec, [v[0] for v in vids])
+    iters = view.iterations(0, rank)
+    outs_a = view.alloc_outputs()
+    outs_b = view.alloc_outputs()
+    fps = frames_per_step(spec)
+
+    def step_id(s):
+        return s // iters, s % iters
+
+    # plan ahead (pre-materialisation of plans)
+    for e in range(0, (args.warmup + args.steps) // iters + 2):
+        view.prefetch_epoch(e, rank)
+
+    s = 0
+    for _ in range(args.warmup):
+        e, it = step_id(s)
+        view.read_batch(e, rank, it, outs_a if s % 2 == 0 else outs_b, stream.cuda_stream)
+        s += 1
+    stream.synchronize()
+
+    # algorithmic bytes of the timed batches (host-side, outside the timed region)
+    first_timed = s
+    sample = sorted({step_id(first_timed + i) for i in range(0, args.steps, max(1, args.steps // 16))})
+    bb = [view.batch_bytes(e, rank, it) for e, it in sample]
+    alg_read = sum(b.src_bytes for b in bb) / len(bb)
+    alg_write = sum(b.out_bytes for b in bb) / len(bb)
+
+    kstart = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    kend = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    start = torch.cuda.Event(enable_timing=True)
+    end = torch.cuda.Event(enable_timing=True)
+    launches0 = view.stats().kernel_launches
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.2)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    start.record(stream)
+    for i in range(args.steps):
+        e, it = step_id(s)
+        kstart[i].record(stream)
+        view.read_batch(e, rank, it, outs_a if s % 2 == 0 else outs_b, stream.cuda_stream)
+        kend[i].record(stream)
+        s += 1
+    end.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    launches = view.stats().kernel_launches - launches0
+    elapsed_ms = start.elapsed_time(end)
+    kernel_ms = sum(a.elapsed_time(b) for a, b in zip(kstart, kend)) / args.steps
+    t = torch.tensor([elapsed_ms, kernel_ms], dtype=torch.float64, device=f"cuda:{local}")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    elapsed_ms, kernel_ms_max = float(t[0]), float(t[1])
+    ms_per_step = elapsed_ms / args.steps
+    value = fps * args.steps * world / (elapsed_ms / 1000.0)
+
+    # reuse counters: the only collective (NCCL all_gather of a few integers)
+    c = store.counters()
+    mine = torch.tensor([c.fetches, c.uses, c.batches], dtype=torch.int64, device=f"cuda:{local}")
+    if world > 1:
+        gathered = [torch.zeros_like(mine) for _ in range(world)]
+        dist.all_gather(gathered, mine)
+        totals = torch.stack(gathered).sum(0).tolist()
+    else:
+        totals = mine.tolist()
+
+    # ---- e2e through the C-ABI with HOST buffers
+    e2e = None
+    if not args.no_e2e:
+        e2e = run_e2e(args, w, spec, view, store, stream, rank, iters, s, world)
+
+    peak, peak_src = measured_peaks()
+    achieved = (alg_read + alg_write) / (kernel_ms / 1000.0) / 1e9
+    line = {
+        "metric": "output frames/s", "value": value, "unit": "frames/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": {0: "u8", 1: "bf16", 2: "f32"}[spec.views[0].out_dtype],
+        "data": "synthetic (seeded NV12, uniform family)", "config": config_dict(w, spec, n_videos),
+        "batches_per_s": value / fps,
+        "per_gpu_frames_per_s": value / world,
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                     "traffic": ncu_traffic(args.config), "kernel": "sand materialize (k_direct/k_stencil)",
+                     "alg_bytes_per_launch": {"read": alg_read, "write": alg_write},
+                     "kernel_ms_per_step": kernel_ms, "peak_source": peak_src,
+                     "frac_of_8tbs_spec": achieved / 8000.0},
+        "gpu_launches": int(launches),
+        "clocks": clk,
+        "reuse": {"fetches": totals[0], "uses": totals[1], "batches": totals[2]},
+    }
+    if e2e is not None:
+        line["e2e"] = e2e
+    if rank == 0 and not args.no_cpu:
+        line["cpu_baseline"] = cpu_baseline(w, spec, vids, args)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    view.close()
+    store.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def run_e2e(args, w, spec, view, store, stream, rank, iters, s0, world):
+    """Same metric end to end through the public API: every step copies its input frames
+    from pinned host memory into the store (H2D), reads the batch, and copies the batch
+    back to pinned host memory (D2H)."""
+    import torch
+    import synth
+    n = args.e2e_steps
+    steps = [((s0 + i) // iters, (s0 + i) % iters) for i in range(n)]
+    W, H = w.width, w.height
+    fb = W * H * 3 // 2
+    # stage each step's unique source frames in pinned host memory (outside the timed region)
+    staged = []
+    scratch = torch.empty(fb, dtype=torch.uint8, device=f"cuda:{torch.cuda.current_device()}")
+    for e, it in steps:
+        keys = sorted({(m.video, m.frames[k][t]) for m in view.get_meta(e, rank, it)
+                       for k, v in enumerate(spec.views) for t in range(v.clip_len)})
+        host = torch.empty((len(keys), fb), dtype=torch.uint8, pin_memory=True)
+        for i, (vid, f) in enumerate(keys):
+            synth.fill_device(synth.UNIFORM, 1234, vid, f, 1, W, H, scratch.data_ptr(), W,
+                              scratch.data_ptr() + W * H, W, 0, 0)
+            host[i].copy_(scratch)
+        staged.append((keys, host))
+    outs = view.alloc_outputs()
+    host_out = [torch.empty(o.shape, dtype=o.dtype, pin_memory=True) for o in outs]
+    h2d = sum(len(k) * fb for k, _ in staged) / n
+    d2h = sum(o.numel() * o.element_size() for o in outs)
+    torch.cuda.synchronize()
+    start = torch.cuda.Event(enable_timing=True)
+    end = torch.cuda.Event(enable_timing=True)
+    start.record(stream)
+    for (e, it), (keys, host) in zip(steps, staged):
+        base = host.data_ptr()
+        for i, (vid, f) in enumerate(keys):
+            p = base + i * fb
+            store.put_frames(vid, f, 1, p, W, fb, p + W * H, W, fb, False, stream.cuda_stream)
+        view.read_batch(e, rank, it, outs, stream.cuda_stream)
+        with torch.cuda.stream(stream):
+            for ho, o in zip(host_out, outs):
+                ho.copy_(o, non_blocking=True)
+    end.record(stream)
+    torch.cuda.synchronize()
+    ms = start.elapsed_time(end)
+    import torch.distributed as dist
+    t = torch.tensor([ms], dtype=torch.float64, device=f"cuda:{torch.cuda.current_device()}")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t[0])
+    return {"value": frames_per_step(spec) * n * world / (ms / 1000.0), "unit": "frames/s",
+            "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h), "steps": n,
+            "ms_per_step": ms / n}
+
+
+def cpu_baseline(w, spec, vids, args):
+    import synth
+    done, el = oracle_frames_per_second(w, spec, vids, None, args.cpu_seconds, synth.UNIFORM, 1234, warmup=1)
+    return {"value": done / el, "unit": "frames/s", "cores": 1, "kind": "oracle",
+            "sample": f"{done} output frames of batch (epoch 0, rank 0, it 0) rendered one by one by the "
+                      f"single-threaded C oracle in {el:.1f}s (source-frame generation excluded)"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=None)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--config", default="k400", choices=["tiny", "k400", "slowfast", "twoview", "ray"])
+    ap.add_argument("--impl", default="sand", choices=["sand", "reference"])
+    ap.add_argument("--videos", type=int, default=None, help="override the store size (videos per GPU)")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=8)
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    args = ap.parse_args()
+    if args.steps is None:
+        args.steps = DEFAULT_STEPS[args.config] if args.impl == "sand" else 200
+    args.warmup = max(args.warmup, 3)
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_sand(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

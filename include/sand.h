@@ -1,0 +1,230 @@
+/*
+ * sand.h — C-ABI of the B200-native SAND view-materialisation library (libsand.so).
+ *
+ * SAND (SOSP'25, /root/reference/PAPER.md) exposes training batches as *views*:
+ * virtual objects materialised when accessed (§5.1), addressed as
+ * /{task}/{epoch}/{iteration}/view (Table 1) and used through
+ * open / read / getxattr / close (Table 2). This library is that view
+ * abstraction for the per-batch materialisation hot path (BASELINE.json
+ * north_star), with decoded frames resident in an HBM frame store:
+ *
+ *   paper                                  this ABI
+ *   decoded frame objects (Table 1)  sand_store_* (HBM, keyed by (video, frame))
+ *   open(view path)        sand_view_create
+ *   read(fd)        sand_view_read_batch(view, epoch, rank, out)
+ *   getxattr(path, meta)  sand_view_get_meta
+ *   close(fd)        sand_view_destroy
+ *
+ * Conventions
+ *  - Every function returns int: SAND_OK (0) or a negative SAND_E* code; nothing
+ *    throws across the ABI. sand_last_error() gives a thread-local message.
+ *  - Pointers named "device" are CUDA device addresses on the store's device;
+ *    everything else is host memory. Streams are cudaStream_t passed as void*
+ *    (NULL = the legacy default stream). Asynchronous calls are ordered on the
+ *    given stream; the caller keeps sources alive until the stream reaches them.
+ *  - One handle must not be used from two threads at once; distinct handles are
+ *    independent.
+ *  - Output of sand_view_read_batch is a pure function of (store bytes, spec,
+ *    epoch, rank, iteration); per clip it does not depend on world_size or rank
+ *    (RNG counters use global clip ids; R#1).
+ */
+#ifndef SAND_H
+#define SAND_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SAND_MAX_VIEWS 8   /* views (tasks / trials / pathways) per view group */
+#define SAND_MAX_GROUPS 8  /* spatial groups; group ids are 0..7 */
+#define SAND_MAX_T 64      /* frames per clip per view */
+
+enum {
+  SAND_OK = 0,
+  SAND_EINVAL = -1, /* invalid argument / spec (odd NV12 dims, alignment, crop > frame, ...) */
+  SAND_ENOENT = -2, /* a planned (video, frame) is not in the store */
+  SAND_ENOMEM = -3, /* store capacity or allocation failure */
+  SAND_ERANGE = -4, /* iteration >= sand_view_iterations, or video id unknown */
+  SAND_ECUDA = -5,  /* CUDA runtime error (message in sand_last_error) */
+  SAND_EBUSY = -6   /* store still has live views */
+};
+enum { SAND_U8 = 0, SAND_BF16 = 1, SAND_F32 = 2 };             /* output dtypes */
+enum { SAND_GEOM_RRC = 0, SAND_GEOM_SHORTSIDE_CROP = 1 };      /* view geometry */
+
+typedef struct sand_store sand_store; /* opaque; owns the device frame slab */
+typedef struct sand_view sand_view;   /* opaque; a view group over one clip stream */
+typedef void* sand_stream_t;          /* cudaStream_t */
+
+/* ------------------------------------------------------------------ store */
+
+/* Create a frame store on `cuda_device` owning one device slab of capacity_bytes.
+ * *out receives the handle. Errors: EINVAL, ENOMEM, ECUDA. */
+int sand_store_create(int cuda_device, uint64_t capacity_bytes, sand_store** out);
+
+/* Reserve slab space for video `video` with n_frames NV12 frames of width x height
+ * (both even). Each frame is laid out as H rows of the Y plane then H/2 rows of
+ * interleaved UV, row pitch = width rounded up to 64 B, frame stride a multiple of
+ * 256 B. Errors: EINVAL (odd/zero dims, video already added with other dims),
+ * ENOMEM (capacity). Re-adding with identical dims is a no-op. */
+int sand_store_add_video(sand_store* s, uint32_t video, uint32_t n_frames, uint32_t width,
+                         uint32_t height);
+
+/* Copy frames [first_frame, first_frame + n_frames) of a video into the store,
+ * stream-ordered. y/uv point at the first frame's Y and UV planes; consecutive
+ * frames are y_frame_stride / uv_frame_stride bytes apart; rows are y_pitch /
+ * uv_pitch apart. src_on_device != 0: y/uv are device pointers, else host (pinned
+ * host memory makes the copy asynchronous). Putting a frame again overwrites it
+ * and resets its counters. Errors: ERANGE (unknown video / frame range), EINVAL,
+ * ECUDA. */
+int sand_store_put_frames(sand_store* s, uint32_t video, uint32_t first_frame, uint32_t n_frames,
+                          const uint8_t* y, uint64_t y_pitch, uint64_t y_frame_stride,
+                          const uint8_t* uv, uint64_t uv_pitch, uint64_t uv_frame_stride,
+                          int src_on_device, sand_stream_t stream);
+
+/* Device address and layout of one stored frame (for tests / zero-copy producers such
+ * as a decoder writing NV12 in place). Errors: ERANGE. */
+typedef struct {
+  uint64_t y;          /* device address of the Y plane */
+  uint64_t uv;         /* device address of the UV plane */
+  uint32_t pitch;      /* row pitch of both planes, bytes */
+  uint32_t width, height, n_frames;
+  uint64_t frame_stride;
+} sand_frame_layout;
+int sand_store_frame_layout(const sand_store* s, uint32_t video, uint32_t frame,
+                            sand_frame_layout* out);
+
+/* Mark frames as present without copying (after a producer wrote them in place via
+ * sand_store_frame_layout). Errors: ERANGE. */
+int sand_store_mark_present(sand_store* s, uint32_t video, uint32_t first_frame, uint32_t n_frames);
+
+/* Reuse accounting (Fig. 16 / Fig. 19): totals over the store. A
+ * "fetch" is one batch-unique source frame read by a read_batch; a "use" is one
+ * output frame (view, clip, t) produced from it. */
+typedef struct {
+  uint64_t videos, frames_present, bytes_reserved, capacity;
+  uint64_t fetches, uses, batches;
+} sand_counters;
+int sand_store_counters(const sand_store* s, sand_counters* out);
+
+/* Per-frame counters of one video, frames [first, first + n). Errors: ERANGE. */
+int sand_store_frame_counters(const sand_store* s, uint32_t video, uint32_t first, uint32_t n,
+                              uint64_t* fetches, uint64_t* uses);
+
+/* Free the store. EBUSY while views created on it are alive. */
+int sand_store_destroy(sand_store* s);
+
+/* ------------------------------------------------------------------ views */
+
+/* One view: a task, a Ray trial or a SlowFast pathway (P:L180-182 config fields). */
+typedef struct {
+  uint32_t clip_len;        /* T frames per clip (<= SAND_MAX_T)                        */
+  uint32_t stride;          /* temporal stride (P:L180 frame_stride)                    */
+  int32_t pool_offset;      /* -1: random grid offset in the shared pool; >= 0 fixed (R#5) */
+  uint32_t spatial_group;   /* 0..7: views with equal group share spatial draws (R#6);
+                               they must agree on every spatial/augmentation field below */
+  int32_t geom;             /* SAND_GEOM_RRC or SAND_GEOM_SHORTSIDE_CROP                */
+  double scale_min, scale_max, ratio_min, ratio_max;   /* RRC ranges (R#8)               */
+  uint32_t short_side;      /* SHORTSIDE_CROP: short side S before the crop (R#10)      */
+  uint32_t out_h, out_w;    /* output frame size                                        */
+  double flip_p;            /* horizontal flip probability (Fig. 9)          */
+  double rot_p, rot_max_deg;            /* rotation gate and range (R#15)               */
+  double blur_p, sigma_min, sigma_max;  /* blur gate and sigma range (R#16)             */
+  uint32_t blur_ksize;      /* odd; radius cap (k-1)/2                                  */
+  double blur_truncate;     /* radius = min((k-1)/2, floor(truncate*sigma+0.5)); 0 = cap  */
+  double mean[3], std[3];   /* per-channel normalisation (R#17)                         */
+  int32_t out_dtype;        /* SAND_U8 / SAND_BF16 / SAND_F32                           */
+} sand_view_desc;
+
+typedef struct {
+  uint64_t seed;
+  uint32_t world_size, batch_size, samples_per_video;  /* B clips per rank per iteration */
+  int32_t drop_last;        /* DistributedSampler drop_last (R#3)                      */
+  const uint32_t* videos;   /* dataset: store video ids, in dataset order (host)        */
+  uint32_t n_videos;
+  uint32_t n_views;         /* 1..SAND_MAX_VIEWS                                        */
+  int32_t shared_window;    /* P:L295 shared window across RRC groups (R#18)           */
+  sand_view_desc views[SAND_MAX_VIEWS];
+} sand_view_spec;
+
+/* Create a view group on a store (the spec is copied). Validates the spec against
+ * the store's videos. Errors: EINVAL, ERANGE (unknown video), ENOMEM, ECUDA. */
+int sand_view_create(sand_store* s, const sand_view_spec* spec, sand_view** out);
+
+/* Output tensor of view k: contiguous [B][3][T][out_h][out_w] of dtype. */
+typedef struct {
+  uint32_t dims[5];
+  int32_t dtype;
+  uint64_t bytes;
+} sand_tensor_desc;
+int sand_view_output_desc(const sand_view* v, uint32_t k, sand_tensor_desc* out);
+
+/* Iterations per epoch for a rank (DistributedSampler num_samples / B, R#3). */
+int sand_view_iterations(const sand_view* v, uint64_t epoch, uint32_t rank, uint64_t* n);
+
+typedef struct {
+  uint64_t iteration;                 /* the {iteration} of the view path (Table 1)   */
+  sand_stream_t stream;               /* all device work is ordered on this stream    */
+  void* data[SAND_MAX_VIEWS];         /* device outputs, 16 B aligned, see output_desc */
+} sand_batch_out;
+
+/* read(): materialise batch (epoch, rank, out->iteration) of every view into
+ * out->data[k], asynchronously on out->stream. The epoch's plan is built on the host
+ * on first use (or ahead of time by sand_view_prefetch_epoch) and uploaded once.
+ * Errors (synchronous): EINVAL (null/misaligned outputs, rank >= world_size),
+ * ERANGE (iteration), ENOENT (a planned frame is absent), ECUDA (launch failure). */
+int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank, const sand_batch_out* out);
+
+/* Plan an epoch ahead of time on a background host thread (the plan analogue of
+ * the paper's pre-materialisation threads). Returns immediately. */
+int sand_view_prefetch_epoch(sand_view* v, uint64_t epoch, uint32_t rank);
+
+/* getxattr(): per-clip metadata of a batch (frame indices, crop boxes, flip,
+ * rotation, blur), written to out[0..B). Fields per group are indexed by group id. */
+typedef struct {
+  uint32_t clip;          /* global clip id (video index * S + sample) */
+  uint32_t video, sample, pool_start;
+  uint32_t frames[SAND_MAX_VIEWS][SAND_MAX_T];
+  int32_t box[SAND_MAX_GROUPS][4];   /* RRC: x0,y0,w,h ; SHORTSIDE: x_off,y_off,W',H' */
+  uint32_t flip[SAND_MAX_GROUPS], rot_on[SAND_MAX_GROUPS], blur_on[SAND_MAX_GROUPS],
+      blur_r[SAND_MAX_GROUPS];
+  double theta[SAND_MAX_GROUPS], sigma[SAND_MAX_GROUPS];
+} sand_clip_meta;
+int sand_view_get_meta(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration,
+                       sand_clip_meta* out);
+
+/* Algorithmic bytes of one batch: distinct 32 B sectors of source
+ * rows touched by bilinear taps (deduplicated across views and groups) and output
+ * bytes; plus the reuse counts the batch adds. */
+typedef struct {
+  uint64_t src_sectors, src_bytes, out_bytes, fetches, uses;
+} sand_batch_bytes;
+int sand_view_batch_bytes(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration,
+                          sand_batch_bytes* out);
+
+/* Launch statistics of a view group: kernels launched and batches read so far. */
+typedef struct {
+  uint64_t batches, kernel_launches, plans_built, work_items;
+} sand_view_stats;
+int sand_view_get_stats(const sand_view* v, sand_view_stats* out);
+
+/* close(): free the view group (waits for its in-flight work). */
+int sand_view_destroy(sand_view* v);
+
+/* Thread-local description of the last error on this thread ("" if none). */
+const char* sand_last_error(void);
+
+/* Library version string. */
+const char* sand_version(void);
+
+/* sizeof of the public structs, for binding layout checks: sizes[0..7] =
+ * sand_frame_layout, sand_counters, sand_view_desc, sand_view_spec, sand_tensor_desc,
+ * sand_batch_out, sand_clip_meta, sand_batch_bytes. Returns the count written (8). */
+int sand_abi_sizes(uint64_t sizes[8]);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SAND_H */

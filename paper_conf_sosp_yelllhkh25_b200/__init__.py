@@ -1,0 +1,176 @@
+"""B200-native SAND per-batch view materialisation (Python binding over libsand.so).
+
+Thin marshalling over the C-ABI in ``include/sand.h`` (names match the C
+functions). torch supplies device memory, streams and process groups only; every
+step of the path runs in libsand.so's CUDA kernels. There is no CPU fallback:
+constructing a ``Store`` without the library or a CUDA device raises.
+
+    store = Store(device=0, capacity_bytes=...)
+    store.add_video(v, n_frames, W, H); store.put_frames(...)   # decoded NV12
+    view = View(store, spec)                                       # open()
+    outs = view.alloc_outputs()                                    # torch tensors
+    view.read_batch(epoch, rank, iteration, outs)                  # read()
+    metas = view.get_meta(epoch, rank, iteration)                  # getxattr()
+    view.close(); store.close()                                    # close()
+"""
+from __future__ import annotations
+
+import ctypes
+
+from . import _abi
+from ._abi import (BF16, F32, GEOM_RRC, GEOM_SHORTSIDE_CROP, MAX_GROUPS, MAX_T, MAX_VIEWS, U8, SandError,
+                   check, lib)
+from .configs import Spec, ViewSpec, Workload
+
+__all__ = ["Store", "View", "Spec", "ViewSpec", "Workload", "SandError", "lib", "make_spec",
+           "U8", "BF16", "F32", "GEOM_RRC", "GEOM_SHORTSIDE_CROP"]
+
+_TORCH_DTYPE = None
+
+
+def _torch_dtype(d: int):
+    import torch
+    return {U8: torch.uint8, BF16: torch.bfloat16, F32: torch.float32}[d]
+
+
+def make_spec(spec: Spec, videos) -> tuple[_abi.sand_view_spec, object]:
+    """Marshal a Spec into sand_view_spec. Returns (struct, keepalive video array)."""
+    s = _abi.sand_view_spec()
+    s.seed = spec.seed
+    s.world_size = spec.world_size
+    s.batch_size = spec.batch_size
+    s.samples_per_video = spec.samples_per_video
+    s.drop_last = int(spec.drop_last)
+    arr = (ctypes.c_uint32 * len(videos))(*videos)
+    s.videos = ctypes.cast(arr, ctypes.POINTER(ctypes.c_uint32))
+    s.n_videos = len(videos)
+    s.n_views = len(spec.views)
+    s.shared_window = int(spec.shared_window)
+    for i, v in enumerate(spec.views):
+        o = s.views[i]
+        o.clip_len, o.stride, o.pool_offset, o.spatial_group = v.clip_len, v.stride, v.pool_offset, v.spatial_group
+        o.geom = v.geom
+        o.scale_min, o.scale_max = v.scale
+        o.ratio_min, o.ratio_max = v.ratio
+        o.short_side, o.out_h, o.out_w = v.short_side, v.out_h, v.out_w
+        o.flip_p, o.rot_p, o.rot_max_deg = v.flip_p, v.rot_p, v.rot_max_deg
+        o.blur_p, (o.sigma_min, o.sigma_max) = v.blur_p, v.sigma
+        o.blur_ksize, o.blur_truncate = v.blur_ksize, v.blur_truncate
+        for c in range(3):
+            o.mean[c] = v.mean[c]
+            o.std[c] = v.std[c]
+        o.out_dtype = v.out_dtype
+    return s, arr
+
+
+class Store:
+    """HBM decoded-frame store keyed by (video, frame) (sand_store_*)."""
+
+    def __init__(self, device: int = 0, capacity_bytes: int = 1 << 30):
+        self._h = ctypes.c_void_p()
+        check(lib().sand_store_create(device, capacity_bytes, ctypes.byref(self._h)), "sand_store_create")
+        self.device = device
+
+    @property
+    def handle(self):
+        return self._h
+
+    def add_video(self, video: int, n_frames: int, width: int, height: int) -> None:
+        check(lib().sand_store_add_video(self._h, video, n_frames, width, height), "sand_store_add_video")
+
+    def put_frames(self, video: int, first_frame: int, n_frames: int, y_ptr: int, y_pitch: int,
+                   y_frame_stride: int, uv_ptr: int, uv_pitch: int, uv_frame_stride: int,
+                   src_on_device: bool, stream: int = 0) -> None:
+        check(lib().sand_store_put_frames(self._h, video, first_frame, n_frames, y_ptr, y_pitch, y_frame_stride,
+                                          uv_ptr, uv_pitch, uv_frame_stride, int(src_on_device), stream),
+              "sand_store_put_frames")
+
+    def frame_layout(self, video: int, frame: int) -> _abi.sand_frame_layout:
+        out = _abi.sand_frame_layout()
+        check(lib().sand_store_frame_layout(self._h, video, frame, ctypes.byref(out)), "sand_store_frame_layout")
+        return out
+
+    def mark_present(self, video: int, first_frame: int, n_frames: int) -> None:
+        check(lib().sand_store_mark_present(self._h, video, first_frame, n_frames), "sand_store_mark_present")
+
+    def counters(self) -> _abi.sand_counters:
+        out = _abi.sand_counters()
+        check(lib().sand_store_counters(self._h, ctypes.byref(out)), "sand_store_counters")
+        return out
+
+    def frame_counters(self, video: int, first: int, n: int):
+        f = (ctypes.c_uint64 * n)()
+        u = (ctypes.c_uint64 * n)()
+        check(lib().sand_store_frame_counters(self._h, video, first, n, f, u), "sand_store_frame_counters")
+        return list(f), list(u)
+
+    def close(self) -> None:
+        if self._h:
+            check(lib().sand_store_destroy(self._h), "sand_store_destroy")
+            self._h = ctypes.c_void_p()
+
+
+class View:
+    """A view group over one clip stream (sand_view_*): open / read / getxattr / close."""
+
+    def __init__(self, store: Store, spec: Spec, videos):
+        self.spec = spec
+        self.store = store
+        self._spec_c, self._keep = make_spec(spec, list(videos))
+        self._h = ctypes.c_void_p()
+        check(lib().sand_view_create(store.handle, ctypes.byref(self._spec_c), ctypes.byref(self._h)),
+              "sand_view_create")
+
+    def output_desc(self, k: int) -> _abi.sand_tensor_desc:
+        d = _abi.sand_tensor_desc()
+        check(lib().sand_view_output_desc(self._h, k, ctypes.byref(d)), "sand_view_output_desc")
+        return d
+
+    def alloc_outputs(self, device=None):
+        import torch
+        outs = []
+        for k in range(len(self.spec.views)):
+            d = self.output_desc(k)
+            outs.append(torch.empty(tuple(d.dims), dtype=_torch_dtype(d.dtype),
+                                    device=device if device is not None else f"cuda:{self.store.device}"))
+        return outs
+
+    def iterations(self, epoch: int = 0, rank: int = 0) -> int:
+        n = ctypes.c_uint64()
+        check(lib().sand_view_iterations(self._h, epoch, rank, ctypes.byref(n)), "sand_view_iterations")
+        return n.value
+
+    def read_batch(self, epoch: int, rank: int, iteration: int, outs, stream: int | None = None) -> None:
+        o = _abi.sand_batch_out()
+        o.iteration = iteration
+        if stream is None:
+            import torch
+            stream = torch.cuda.current_stream(self.store.device).cuda_stream
+        o.stream = stream
+        for k, t in enumerate(outs):
+            o.data[k] = t.data_ptr() if hasattr(t, "data_ptr") else int(t)
+        check(lib().sand_view_read_batch(self._h, epoch, rank, ctypes.byref(o)), "sand_view_read_batch")
+
+    def prefetch_epoch(self, epoch: int, rank: int = 0) -> None:
+        check(lib().sand_view_prefetch_epoch(self._h, epoch, rank), "sand_view_prefetch_epoch")
+
+    def get_meta(self, epoch: int, rank: int, iteration: int):
+        out = (_abi.sand_clip_meta * self.spec.batch_size)()
+        check(lib().sand_view_get_meta(self._h, epoch, rank, iteration, out), "sand_view_get_meta")
+        return list(out)
+
+    def batch_bytes(self, epoch: int, rank: int, iteration: int) -> _abi.sand_batch_bytes:
+        out = _abi.sand_batch_bytes()
+        check(lib().sand_view_batch_bytes(self._h, epoch, rank, iteration, ctypes.byref(out)),
+              "sand_view_batch_bytes")
+        return out
+
+    def stats(self) -> _abi.sand_view_stats:
+        out = _abi.sand_view_stats()
+        check(lib().sand_view_get_stats(self._h, ctypes.byref(out)), "sand_view_get_stats")
+        return out
+
+    def close(self) -> None:
+        if self._h:
+            check(lib().sand_view_destroy(self._h), "sand_view_destroy")
+            self._h = ctypes.c_void_p()

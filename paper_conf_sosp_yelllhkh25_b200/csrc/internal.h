@@ -1,0 +1,108 @@
+// internal.h — host runtime objects behind the C-ABI (store, view group, plans).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <condition_variable>
+#include <cstdint>
+#include <deque>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <unordered_map>
+#include <vector>
+
+#include "plan_types.h"
+#include "planner.h"
+#include "sand.h"
+
+namespace sand {
+
+// thread-local error message; every ABI function sets it before returning an error
+int set_error(int code, const std::string& msg);
+int cuda_error(cudaError_t e, const char* what);
+
+// ------------------------------------------------------------------ HBM frame store (D4)
+struct VideoEntry {
+  uint32_t id, n_frames, width, height, pitch;
+  uint64_t offset;         // slab offset of frame 0
+  uint64_t frame_stride;   // bytes between frames
+  std::vector<uint8_t> present;
+  std::vector<uint64_t> fetches, uses;   // reuse accounting (a12)
+};
+
+}  // namespace sand
+
+struct sand_store {
+  int device = 0;
+  uint8_t* slab = nullptr;
+  uint64_t capacity = 0, used = 0;
+  std::unordered_map<uint32_t, sand::VideoEntry> videos;
+  std::atomic<int> live_views{0};
+  uint64_t batches = 0;
+  std::mutex mu;   // guards counters updated by read_batch (views may live on several threads)
+};
+
+namespace sand {
+
+// ------------------------------------------------------------------ epoch plan (D8)
+struct EpochPlan {
+  uint64_t epoch = 0;
+  uint32_t rank = 0;
+  uint64_t iterations = 0;
+  std::vector<sand_clip_meta> metas;          // iterations * B
+  std::vector<GroupParams> groups;            // iterations * B * n_groups
+  std::vector<WorkItem> items;
+  std::vector<uint32_t> dests;
+  std::vector<uint32_t> item_begin;           // iterations + 1
+  std::vector<uint8_t> batch_stencil;         // per iteration: any item needs rotation/blur
+  // reuse accounting per iteration: unique (video, frame) keys and their use counts
+  std::vector<uint32_t> fetch_begin;          // iterations + 1
+  std::vector<std::pair<uint32_t, uint32_t>> fetch_keys;   // (video, frame)
+  std::vector<uint32_t> fetch_uses;
+  // device copy
+  void* d_buf = nullptr;
+  void* h_stage = nullptr;
+  size_t d_bytes = 0;
+  GroupParams* d_groups = nullptr;
+  WorkItem* d_items = nullptr;
+  uint32_t* d_dests = nullptr;
+  bool uploaded = false;
+  cudaEvent_t last_use = nullptr;
+  uint64_t last_touch = 0;
+};
+
+}  // namespace sand
+
+struct sand_view {
+  sand_store* store = nullptr;
+  sand::SpecInfo info;
+  sand::ViewConst vconst[sand::kMaxViews];
+  std::vector<uint32_t> video_slot;   // dataset index -> unused (dims live in info)
+  // plan cache, keyed by (epoch, rank)
+  std::mutex mu;
+  std::condition_variable cv;
+  std::map<std::pair<uint64_t, uint32_t>, std::shared_ptr<sand::EpochPlan>> plans;
+  std::map<std::pair<uint64_t, uint32_t>, bool> pending;   // being built by the worker
+  std::deque<std::pair<uint64_t, uint32_t>> queue;
+  std::thread worker;
+  bool stop = false;
+  uint64_t touch = 0;
+  // stats
+  uint64_t batches = 0, launches = 0, plans_built = 0, work_items = 0;
+  size_t stencil_smem = 0;   // dynamic smem of the stencil path (0 if no view rotates/blurs)
+};
+
+namespace sand {
+
+std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32_t rank);
+
+// kernels (materialize.cu)
+size_t stencil_smem_bytes(int max_h, int max_w, int max_r);
+int configure_kernels(size_t stencil_smem);
+int launch_materialize(const LaunchParams& p, bool stencil, size_t stencil_smem, cudaStream_t stream,
+                       int* n_launched);
+
+}  // namespace sand

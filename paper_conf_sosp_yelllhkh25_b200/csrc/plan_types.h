@@ -1,0 +1,75 @@
+// plan_types.h — device-visible materialisation plan (host planner -> CUDA kernels).
+//
+// A batch (epoch, rank, iteration) is a list of WORK ITEMS. A work item is one
+// (clip slot b, source frame f, spatial group q) triple: the source frame is read
+// once and every (view, t) of group q that selected frame f is written from it
+// (multi-view fan-out; node merging). Items of
+// the same (b, f) are adjacent so the groups of one frame share its lines in L2.
+#pragma once
+#include <stdint.h>
+
+#if defined(__CUDACC__)
+#define SAND_HD __host__ __device__
+#else
+#define SAND_HD
+#endif
+
+namespace sand {
+
+constexpr int kMaxViews = 8;
+constexpr int kMaxGroups = 8;
+constexpr int kMaxT = 64;
+constexpr int kMaxTaps = 23;  // blur taps (k <= 23)
+
+// Geometry + augmentation of one (clip slot, group). Source coordinate of output
+// column ox (after the flip mirror ox' = flip ? Wo-1-ox : ox):
+//   s = max(sc_x * ((float)(off_x + ox') + 0.5f) - 0.5f, 0);  i0 = (int)s;
+//   i1 = min(i0 + 1, lim_x - 1);  taps at org_x + i0, org_x + i1      (R#12)
+// RRC: org = crop origin, off = 0, lim = crop size, sc = (float)w / Wo.
+// SHORTSIDE_CROP: org = 0, off = crop offset in the resized frame, lim = frame size,
+// sc = (float)W / W'.
+struct alignas(16) GroupParams {
+  int32_t org_x, org_y, off_x, off_y;
+  int32_t lim_x, lim_y, out_w, out_h;
+  float sc_x, sc_y, rot_c, rot_s;
+  int32_t flip, rot_on, blur_on, blur_r;
+  float blur_w[24];
+};
+
+struct alignas(16) WorkItem {
+  uint64_t y_off;        // byte offset of the source frame's Y plane in the slab
+  uint32_t pitch;        // row pitch of Y and UV planes (UV plane at y_off + pitch*src_h)
+  uint32_t src_w, src_h;
+  uint32_t gp;           // GroupParams index (absolute within the epoch plan)
+  uint32_t dest_begin;   // first destination (absolute within the epoch plan)
+  uint32_t n_dest;
+  uint32_t clip_slot;    // b
+  uint32_t group;        // q
+  uint32_t flags;        // bit0: needs the stencil path (rotation or blur)
+  uint32_t pad;
+};
+
+// destination packing: view (8 bits) << 24 | t (8 bits) << 16 | b (16 bits)
+SAND_HD inline uint32_t pack_dest(uint32_t view, uint32_t t, uint32_t b) {
+  return (view << 24) | (t << 16) | b;
+}
+
+struct ViewConst {
+  float a[3], b[3];      // y = fmaf(q, a_c, b_c)  (R#17)
+  int32_t dtype;         // SAND_U8 / SAND_BF16 / SAND_F32
+  int32_t T, out_h, out_w;
+};
+
+struct LaunchParams {
+  const uint8_t* slab;
+  const WorkItem* items;   // this batch's items
+  uint32_t n_items;
+  const GroupParams* groups;
+  const uint32_t* dests;
+  void* out[kMaxViews];
+  ViewConst views[kMaxViews];
+  uint32_t n_views;
+  uint32_t batch;          // B
+};
+
+}  // namespace sand

@@ -79,3 +79,17 @@ def fill_device(family: int, seed: int, video: int, first_frame: int, n_frames: 
                                     y_ptr, y_pitch, uv_ptr, uv_pitch, frame_stride, stream)
     if rc != 0:
         raise RuntimeError(f"synth_fill_frames_cuda failed ({rc})")
+
+
+def fill_store(store, videos, family: int, seed: int, stream: int = 0) -> None:
+    """Write synthetic frames straight into a product frame store (zero-copy).
+
+    ``store`` is a paper_conf_sosp_yelllhkh25_b200.Store; ``videos`` is a list of
+    (video_id, n_frames, width, height). Uses only the store's public layout query
+    (sand_store_frame_layout) and mark_present; the bytes come from this module.
+    """
+    for vid, F, W, H in videos:
+        store.add_video(vid, F, W, H)
+        lay = store.frame_layout(vid, 0)
+        fill_device(family, seed, vid, 0, F, W, H, lay.y, lay.pitch, lay.uv, lay.pitch, lay.frame_stride, stream)
+        store.mark_present(vid, 0, F)

@@ -1,0 +1,242 @@
+"""GPU parity: the CUDA path through the C-ABI against the oracle (pytest -m gpu).
+
+For every BASELINE.json workload: (1) the plan (clip ids, frame indices, crop
+boxes, flip / rotation / blur draws) is compared BIT-EXACTLY through
+sand_view_get_meta; (2) materialised outputs are compared element by element
+with oracle renders on the same synthetic frames — whole batches on reduced
+stores the oracle finishes in seconds, and sampled frames at the full
+BASELINE.json store sizes in the launch configuration bench.py times; (3)
+invariants the paper fixes (SlowFast slow == fast[::4], world-size invariance,
+exactly-once coverage, reuse accounting) and the error paths.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+from paper_conf_sosp_yelllhkh25_b200 import configs
+import paper_conf_sosp_yelllhkh25_b200 as sand
+
+from helpers import compare, meta_fields, oracle_render, out_numpy, to_oracle, videos_of
+
+pytestmark = pytest.mark.gpu
+SEED = 1234
+
+
+def _setup(workload, n_videos=None, family=synth.UNIFORM, spec=None):
+    vids = videos_of(workload, n_videos)
+    per_frame = (workload.width + 63) // 64 * 64 * workload.height * 3 // 2 + 256
+    cap = len(vids) * workload.n_frames * per_frame + (1 << 20)
+    store = sand.Store(0, cap)
+    synth.fill_store(store, vids, family, SEED)
+    torch.cuda.synchronize()
+    spec = spec or workload.spec
+    view = sand.View(store, spec, [v[0] for v in vids])
+    ospec = to_oracle(spec)
+    ods = oracle.make_dataset(vids)
+    return store, view, ospec, ods, vids
+
+
+def _teardown(store, view):
+    view.close()
+    store.close()
+
+
+def _check_meta(view, spec, ospec, ods, n, epoch, rank, it):
+    got = [meta_fields(spec, m) for m in view.get_meta(epoch, rank, it)]
+    ref = [meta_fields(spec, m) for m in oracle.plan_batch(ospec, ods, n, epoch, rank, it)]
+    assert got == ref
+
+
+def _check_outputs(view, spec, ospec, ods, vids, epoch, rank, it, samples=None, family=synth.UNIFORM):
+    outs = view.alloc_outputs()
+    view.read_batch(epoch, rank, it, outs)
+    torch.cuda.synchronize()
+    ometas = oracle.plan_batch(ospec, ods, len(vids), epoch, rank, it)
+    W, H = vids[0][2], vids[0][3]
+    if samples is None:
+        samples = [(b, k, t) for b in range(spec.batch_size) for k, v in enumerate(spec.views)
+                   for t in range(v.clip_len)]
+    stats = []
+    for b, k, t in samples:
+        ref = oracle_render(ospec, ometas[b], k, t, family, SEED, W, H)
+        got = out_numpy(outs[k][b, :, t])
+        stats.append(compare(got, ref, spec.views[k].out_dtype))
+    # bit-identical by construction (R#20): report exact-match fraction
+    exact = float(np.mean([s["exact"] for s in stats]))
+    assert exact == 1.0, f"exact-match fraction {exact}"
+    return outs
+
+
+# ------------------------------------------------------------------ tiny (configs[0]): whole batches
+
+@pytest.mark.parametrize("dtype", [configs.U8, configs.BF16, configs.F32])
+@pytest.mark.parametrize("family", [synth.UNIFORM, synth.SMOOTH])
+def test_tiny_all_epochs_exact(dtype, family):
+    w = configs.tiny()
+    w.spec.views[0].out_dtype = dtype
+    store, view, ospec, ods, vids = _setup(w, family=family)
+    try:
+        for epoch in range(6):
+            _check_meta(view, w.spec, ospec, ods, 1, epoch, 0, 0)
+            _check_outputs(view, w.spec, ospec, ods, vids, epoch, 0, 0, family=family)
+    finally:
+        _teardown(store, view)
+
+
+# ------------------------------------------------------------------ reduced stores: whole batches
+
+@pytest.mark.parametrize("name,n_videos", [("k400", 40), ("slowfast", 20), ("ray", 6)])
+def test_reduced_store_whole_batch(name, n_videos):
+    w = configs.get(name)
+    store, view, ospec, ods, vids = _setup(w, n_videos)
+    try:
+        n_it = view.iterations(0, 0)
+        assert n_it == oracle.iterations(ospec, n_videos)
+        for it in range(n_it):
+            _check_meta(view, w.spec, ospec, ods, n_videos, 0, 0, it)
+        _check_outputs(view, w.spec, ospec, ods, vids, 0, 0, 0)
+    finally:
+        _teardown(store, view)
+
+
+def test_twoview_rotate_blur_sampled_clips():
+    w = configs.twoview()
+    w.spec.batch_size = 8
+    store, view, ospec, ods, vids = _setup(w, 24)
+    try:
+        for it in range(view.iterations(0, 0)):
+            _check_meta(view, w.spec, ospec, ods, 24, 1, 0, it)
+        metas = oracle.plan_batch(ospec, ods, 24, 1, 0, 0)
+        assert any(m.rot_on[0] or m.rot_on[1] for m in metas) and any(m.blur_on[0] or m.blur_on[1] for m in metas)
+        samples = [(b, k, t) for b in range(8) for k in range(2) for t in (0, 7, 15)]
+        _check_outputs(view, w.spec, ospec, ods, vids, 1, 0, 0, samples=samples)
+    finally:
+        _teardown(store, view)
+
+
+# ------------------------------------------------------------------ full BASELINE.json sizes, sampled
+
+@pytest.mark.parametrize("name", ["k400", "slowfast", "twoview", "ray"])
+def test_full_size_sampled(name):
+    w = configs.get(name)
+    store, view, ospec, ods, vids = _setup(w)
+    try:
+        rng = np.random.default_rng(7)
+        n_it = view.iterations(0, 0)
+        for it in (0, n_it - 1):
+            _check_meta(view, w.spec, ospec, ods, len(vids), 2, 0, it)
+        samples = [(int(rng.integers(w.spec.batch_size)), k, int(rng.integers(v.clip_len)))
+                   for k, v in enumerate(w.spec.views) for _ in range(6)]
+        _check_outputs(view, w.spec, ospec, ods, vids, 2, 0, n_it - 1, samples=samples)
+    finally:
+        _teardown(store, view)
+
+
+# ------------------------------------------------------------------ invariants
+
+def test_slowfast_slow_is_fast_every_fourth_frame():
+    w = configs.slowfast()
+    store, view, ospec, ods, vids = _setup(w, 16)
+    try:
+        outs = view.alloc_outputs()
+        view.read_batch(0, 0, 0, outs)
+        torch.cuda.synchronize()
+        fast, slow = outs
+        assert torch.equal(slow, fast[:, :, ::4])
+    finally:
+        _teardown(store, view)
+
+
+def test_world_size_invariance_and_exactly_once():
+    w = configs.k400()
+    w.spec.batch_size = 4
+    store, view1, ospec, ods, vids = _setup(w, 32)
+    spec8 = configs.k400().spec
+    spec8.batch_size = 4
+    spec8.world_size = 8
+    view8 = sand.View(store, spec8, [v[0] for v in vids])
+    try:
+        by_clip = {}
+        for it in range(view1.iterations(0, 0)):
+            outs = view1.alloc_outputs()
+            view1.read_batch(0, 0, it, outs)
+            for b, m in enumerate(view1.get_meta(0, 0, it)):
+                by_clip[m.clip] = outs[0][b].clone()
+        assert sorted(by_clip) == list(range(32))        # P:L285 exactly once per epoch
+        seen = []
+        for r in range(8):
+            for it in range(view8.iterations(0, r)):
+                outs = view8.alloc_outputs()
+                view8.read_batch(0, r, it, outs)
+                for b, m in enumerate(view8.get_meta(0, r, it)):
+                    assert torch.equal(outs[0][b], by_clip[m.clip])
+                    seen.append(m.clip)
+        assert sorted(seen) == list(range(32))
+    finally:
+        view8.close()
+        _teardown(store, view1)
+
+
+def test_reuse_accounting_and_batch_bytes_match_oracle():
+    w = configs.slowfast()
+    store, view, ospec, ods, vids = _setup(w, 16)
+    try:
+        outs = view.alloc_outputs()
+        view.read_batch(0, 0, 0, outs)
+        torch.cuda.synchronize()
+        bb = view.batch_bytes(0, 0, 0)
+        ob = oracle.batch_bytes(ospec, ods, 16, 0, 0, 0)
+        assert (bb.src_sectors, bb.out_bytes, bb.fetches, bb.uses) == \
+            (ob.src_sectors, ob.out_bytes, ob.fetches, ob.uses)
+        c = store.counters()
+        assert (c.fetches, c.uses, c.batches) == (ob.fetches, ob.uses, 1)
+    finally:
+        _teardown(store, view)
+    for name in ("k400", "ray", "twoview"):
+        w = configs.get(name)
+        store, view, ospec, ods, vids = _setup(w, 6 if name == "ray" else 70)
+        try:
+            bb = view.batch_bytes(0, 0, 0)
+            ob = oracle.batch_bytes(ospec, ods, len(vids), 0, 0, 0)
+            assert (bb.src_sectors, bb.out_bytes, bb.fetches, bb.uses) == \
+                (ob.src_sectors, ob.out_bytes, ob.fetches, ob.uses), name
+        finally:
+            _teardown(store, view)
+
+
+# ------------------------------------------------------------------ error paths
+
+def test_error_paths():
+    w = configs.tiny()
+    vids = videos_of(w)
+    store = sand.Store(0, 1 << 24)
+    store.add_video(vids[0][0], 16, 64, 64)      # reserved but no frame put yet
+    view = sand.View(store, w.spec, [vids[0][0]])
+    try:
+        outs = view.alloc_outputs()
+        with pytest.raises(sand.SandError) as e:
+            view.read_batch(0, 0, 0, outs)
+        assert e.value.code == sand._abi.ENOENT
+        synth.fill_store(store, vids, synth.UNIFORM, SEED)
+        view.read_batch(0, 0, 0, outs)
+        with pytest.raises(sand.SandError) as e:
+            view.read_batch(0, 0, 1, outs)
+        assert e.value.code == sand._abi.ERANGE
+        with pytest.raises(sand.SandError) as e:
+            view.read_batch(0, 0, 0, [outs[0].view(-1)[1:].data_ptr()])
+        assert e.value.code == sand._abi.EINVAL
+        with pytest.raises(sand.SandError) as e:
+            store.close()
+        assert e.value.code == sand._abi.EBUSY
+        bad = configs.tiny().spec
+        bad.views[0].blur_ksize = 4
+        with pytest.raises(sand.SandError):
+            sand.View(store, bad, [vids[0][0]])
+        with pytest.raises(sand.SandError) as e:
+            sand.View(store, w.spec, [999999])
+        assert e.value.code == sand._abi.ERANGE
+    finally:
+        view.close()
+        store.close()
