@@ -57,7 +57,7 @@ struct EpochPlan {
   std::vector<WorkItem> items;
   std::vector<uint32_t> dests;
   std::vector<uint32_t> item_begin;           // iterations + 1
-  std::vector<uint8_t> batch_stencil;         // per iteration: any item needs rotation/blur
+  std::vector<BatchShape> shapes;             // per iteration: launch shape
   // reuse accounting per iteration: unique (video, frame) keys and their use counts
   std::vector<uint32_t> fetch_begin;          // iterations + 1
   std::vector<std::pair<uint32_t, uint32_t>> fetch_keys;   // (video, frame)
@@ -102,7 +102,7 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
 // kernels (materialize.cu)
 size_t stencil_smem_bytes(int max_h, int max_w, int max_r);
 int configure_kernels(size_t stencil_smem);
-int launch_materialize(const LaunchParams& p, bool stencil, size_t stencil_smem, cudaStream_t stream,
+int launch_materialize(const LaunchParams& p, const BatchShape& shape, size_t stencil_smem, cudaStream_t stream,
                        int* n_launched);
 
 }  // namespace sand

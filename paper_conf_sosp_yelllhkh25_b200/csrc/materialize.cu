@@ -1,10 +1,8 @@
 // materialize.cu — sm_100a kernels of the materialisation path.
 //
-// v1 (first correct path): one CTA per work item (clip slot, source frame, group).
-//  * k_direct : items without rotation/blur. Thread per output pixel: 4 bilinear taps
-//               read from the NV12 frame in HBM, converted to RGB on the fly (Q1),
-//               lerped in fp32 (Q2), normalised and stored to every destination.
-//  * k_stencil: items with rotation and/or blur. Per channel: Q2 plane in shared
+//  * k_tapgrid (k_tapgrid.cuh): items without rotation/blur — banded tap-grid resample,
+//               one CTA per (work item, band of output rows).
+//  * k_stencil: items with rotation and/or blur, one CTA per work item. Per channel: Q2 plane in shared
 //               memory -> rotated Q3 plane -> separable blur in row strips (fp32
 //               horizontal pass kept in shared memory) -> normalise -> store.
 // Arithmetic follows DESIGN.md R#11-R#17 with explicit IEEE-rounded intrinsics
@@ -13,6 +11,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <algorithm>
+#include <cmath>
 #include <string>
 
 #include "plan_types.h"
@@ -29,23 +29,6 @@ constexpr int kStripRows = 32;     // output rows per blur strip
 
 // ---------------------------------------------------------------- a5: NV12 -> RGB (R#11)
 __device__ __forceinline__ int clamp_u8(int v) { return min(max(v, 0), 255); }
-
-struct Taps {       // one bilinear tap position in the source frame
-  const uint8_t* y;
-  const uint8_t* uv;
-};
-
-__device__ __forceinline__ void nv12_rgb(const uint8_t* __restrict__ Yp, const uint8_t* __restrict__ UVp,
-                                         uint32_t pitch, int x, int y, int rgb[3]) {
-  const int Yv = __ldg(Yp + (size_t)y * pitch + x);
-  const uint8_t* uvr = UVp + (size_t)(y >> 1) * pitch + (x & ~1);
-  const int u = (int)__ldg(uvr) - 128;
-  const int v = (int)__ldg(uvr + 1) - 128;
-  const int yy = max(Yv - 16, 0) * 1220542 + (1 << 19);
-  rgb[0] = clamp_u8((yy + 1673527 * v) >> 20);
-  rgb[1] = clamp_u8((yy - 852492 * v - 409993 * u) >> 20);
-  rgb[2] = clamp_u8((yy + 2116026 * u) >> 20);
-}
 
 __device__ __forceinline__ int nv12_chan(const uint8_t* __restrict__ Yp, const uint8_t* __restrict__ UVp,
                                          uint32_t pitch, int x, int y, int c) {
@@ -87,41 +70,6 @@ __device__ __forceinline__ void store_value(const LaunchParams& p, uint32_t dest
       static_cast<__nv_bfloat16*>(p.out[k])[idx] = __float2bfloat16_rn(y);
     else
       static_cast<float*>(p.out[k])[idx] = y;
-  }
-}
-
-// ---------------------------------------------------------------- k_direct
-__global__ void __launch_bounds__(256) k_direct(const LaunchParams p) {
-  const WorkItem w = p.items[blockIdx.x];
-  if (w.flags & 1u) return;
-  const GroupParams& g = p.groups[w.gp];
-  const uint8_t* Yp = p.slab + w.y_off;
-  const uint8_t* UVp = Yp + (size_t)w.pitch * w.src_h;
-  const int Wo = g.out_w, Ho = g.out_h;
-  for (int pix = threadIdx.x; pix < Ho * Wo; pix += blockDim.x) {
-    const int oy = pix / Wo, ox = pix - (pix / Wo) * Wo;
-    const int oxm = g.flip ? Wo - 1 - ox : ox;        // a7: flip mirrors the output column
-    int x0, x1, y0, y1;
-    float lx, ly;
-    src_tap(g.sc_x, g.off_x, oxm, g.lim_x, g.org_x, x0, x1, lx);
-    src_tap(g.sc_y, g.off_y, oy, g.lim_y, g.org_y, y0, y1, ly);
-    int p00[3], p01[3], p10[3], p11[3];
-    nv12_rgb(Yp, UVp, w.pitch, x0, y0, p00);
-    nv12_rgb(Yp, UVp, w.pitch, x1, y0, p01);
-    nv12_rgb(Yp, UVp, w.pitch, x0, y1, p10);
-    nv12_rgb(Yp, UVp, w.pitch, x1, y1, p11);
-    int q[3];
-#pragma unroll
-    for (int c = 0; c < 3; ++c) {
-      const float h0 = lerp_rn(lx, (float)p00[c], (float)p01[c]);
-      const float h1 = lerp_rn(lx, (float)p10[c], (float)p11[c]);
-      q[c] = quant(lerp_rn(ly, h0, h1));
-    }
-    for (uint32_t d = 0; d < w.n_dest; ++d) {
-      const uint32_t dest = p.dests[w.dest_begin + d];
-#pragma unroll
-      for (int c = 0; c < 3; ++c) store_value(p, dest, c, oy, ox, q[c]);
-    }
   }
 }
 
@@ -217,6 +165,28 @@ __global__ void __launch_bounds__(512) k_stencil(const LaunchParams p) {
 }
 
 }  // namespace
+}  // namespace sand
+
+#include "k_tapgrid.cuh"
+
+namespace sand {
+
+namespace {
+constexpr size_t kTgSmemBudget = 55 * 1024;   // 4 CTAs / SM
+
+// band height R and dynamic shared memory of k_tapgrid for a batch shape
+void choose_tapgrid(const BatchShape& sh, int* R, size_t* smem) {
+  static const int kCands[] = {64, 48, 32, 24, 16, 8, 4, 2, 1};
+  for (int r : kCands) {
+    const int span = static_cast<int>(std::ceil(static_cast<double>(sh.max_scy) * r)) + 3;   // row bitmap span
+    const int rows = std::min(2 * r, span);
+    const size_t bytes = tg::table_bytes(sh.max_wo, r) + (size_t)rows * sh.cols_bound * 4;
+    *R = r;
+    *smem = bytes;
+    if ((bytes <= kTgSmemBudget && span <= 32 * tg::kRowWords) || r == 1) return;
+  }
+}
+}  // namespace
 
 size_t stencil_smem_bytes(int max_h, int max_w, int max_r) {
   const size_t n = ((size_t)max_h * max_w + 15) & ~(size_t)15;
@@ -224,6 +194,10 @@ size_t stencil_smem_bytes(int max_h, int max_w, int max_r) {
 }
 
 int configure_kernels(size_t stencil_smem) {
+  {
+    cudaError_t e = cudaFuncSetAttribute(k_tapgrid, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    if (e != cudaSuccess) return cuda_error(e, "cudaFuncSetAttribute(k_tapgrid)");
+  }
   if (stencil_smem > 0) {
     if (stencil_smem > 227 * 1024) return set_error(SAND_EINVAL, "stencil shared memory exceeds 227 KB");
     cudaError_t e = cudaFuncSetAttribute(k_stencil, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)stencil_smem);
@@ -232,19 +206,29 @@ int configure_kernels(size_t stencil_smem) {
   return SAND_OK;
 }
 
-int launch_materialize(const LaunchParams& p, bool stencil, size_t stencil_smem, cudaStream_t stream,
+int launch_materialize(const LaunchParams& p, const BatchShape& shape, size_t stencil_smem, cudaStream_t stream,
                        int* n_launched) {
   *n_launched = 0;
   if (p.n_items == 0) return SAND_OK;
-  k_direct<<<p.n_items, 256, 0, stream>>>(p);
-  cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess) return cuda_error(e, "k_direct launch");
-  *n_launched = 1;
-  if (stencil) {
+  if (shape.has_direct) {
+    int R;
+    size_t smem;
+    choose_tapgrid(shape, &R, &smem);
+    if (smem > 227 * 1024) return set_error(SAND_EINVAL, "tap grid exceeds shared memory (source crop too large)");
+    const int nbands = (shape.max_ho + R - 1) / R;
+    const int pairs = (shape.max_wo + 1) / 2;
+    const int threads = std::min(256, ((2 * pairs + 31) / 32) * 32);
+    const uint64_t blocks = (uint64_t)p.n_items * nbands;
+    k_tapgrid<<<(unsigned)blocks, threads, smem, stream>>>(p, R, nbands, shape.max_wo);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_error(e, "k_tapgrid launch");
+    ++*n_launched;
+  }
+  if (shape.has_stencil) {
     k_stencil<<<p.n_items, 512, stencil_smem, stream>>>(p);
-    e = cudaGetLastError();
+    cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_error(e, "k_stencil launch");
-    *n_launched = 2;
+    ++*n_launched;
   }
   return SAND_OK;
 }

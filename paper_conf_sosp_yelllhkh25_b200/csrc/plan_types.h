@@ -60,6 +60,14 @@ struct ViewConst {
   int32_t T, out_h, out_w;
 };
 
+// Per-batch launch shape of the direct (no rotation/blur) items, from the plan.
+struct BatchShape {
+  int32_t has_direct, has_stencil;
+  int32_t max_wo, max_ho;
+  int32_t cols_bound;     // upper bound of distinct tapped source columns of any item
+  float max_scy;          // largest vertical source step (rows per output row)
+};
+
 struct LaunchParams {
   const uint8_t* slab;
   const WorkItem* items;   // this batch's items

@@ -43,6 +43,7 @@ extern "C" int sand_store_add_video(sand_store* s, uint32_t video, uint32_t n_fr
   if (!s) return sand::set_error(SAND_EINVAL, "store is null");
   if (width == 0 || height == 0 || (width & 1u) || (height & 1u) || n_frames == 0)
     return sand::set_error(SAND_EINVAL, "NV12 frames need even, non-zero width/height and n_frames > 0");
+  if (width > 4096 || height > 4096) return sand::set_error(SAND_EINVAL, "frames larger than 4096x4096");
   std::lock_guard<std::mutex> lk(s->mu);
   auto it = s->videos.find(video);
   if (it != s->videos.end()) {

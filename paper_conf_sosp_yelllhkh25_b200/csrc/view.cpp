@@ -91,7 +91,7 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
   plan->item_begin.push_back(0);
   plan->fetch_begin.push_back(0);
   for (uint64_t it = 0; it < plan->iterations; ++it) {
-    bool stencil = false;
+    BatchShape shape{};
     std::vector<std::pair<uint64_t, uint32_t>> fetch;   // ((video<<32)|frame, uses)
     for (uint32_t b = 0; b < B; ++b) {
       const uint64_t slot = it * B + b;
@@ -132,7 +132,16 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
           w.group = q;
           const GroupParams& g = plan->groups[w.gp];
           w.flags = (g.rot_on || g.blur_on) ? 1u : 0u;
-          stencil = stencil || w.flags;
+          if (w.flags) {
+            shape.has_stencil = 1;
+          } else {
+            shape.has_direct = 1;
+            shape.max_wo = std::max(shape.max_wo, g.out_w);
+            shape.max_ho = std::max(shape.max_ho, g.out_h);
+            const int cols = std::min(2 * g.out_w, static_cast<int>(std::ceil(static_cast<double>(g.sc_x) * g.out_w)) + 3);
+            shape.cols_bound = std::max(shape.cols_bound, cols);
+            shape.max_scy = std::max(shape.max_scy, g.sc_y);
+          }
           plan->items.push_back(w);
         }
         fetch.push_back({(static_cast<uint64_t>(dim.id) << 32) | f, uses});
@@ -150,7 +159,7 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
     }
     plan->fetch_begin.push_back(static_cast<uint32_t>(plan->fetch_keys.size()));
     plan->item_begin.push_back(static_cast<uint32_t>(plan->items.size()));
-    plan->batch_stencil.push_back(stencil ? 1 : 0);
+    plan->shapes.push_back(shape);
   }
   return plan;
 }
@@ -397,9 +406,8 @@ extern "C" int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank,
     lp.out[k] = out->data[k];
     lp.views[k] = v->vconst[k];
   }
-  const bool stencil = plan->batch_stencil[it] != 0;
   int launched = 0;
-  int rc = sand::launch_materialize(lp, stencil, v->stencil_smem, stream, &launched);
+  int rc = sand::launch_materialize(lp, plan->shapes[it], v->stencil_smem, stream, &launched);
   if (rc != SAND_OK) return rc;
   e = cudaEventRecord(plan->last_use, stream);
   if (e != cudaSuccess) return sand::cuda_error(e, "cudaEventRecord");

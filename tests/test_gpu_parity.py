@@ -87,16 +87,19 @@ def test_tiny_all_epochs_exact(dtype, family):
 
 # ------------------------------------------------------------------ reduced stores: whole batches
 
-@pytest.mark.parametrize("name,n_videos", [("k400", 40), ("slowfast", 20), ("ray", 6)])
-def test_reduced_store_whole_batch(name, n_videos):
+@pytest.mark.parametrize("name,n_videos,clips", [("k400", 40, None), ("slowfast", 20, None), ("ray", 20, 3)])
+def test_reduced_store_whole_batch(name, n_videos, clips):
     w = configs.get(name)
     store, view, ospec, ods, vids = _setup(w, n_videos)
     try:
         n_it = view.iterations(0, 0)
-        assert n_it == oracle.iterations(ospec, n_videos)
+        assert n_it == oracle.iterations(ospec, n_videos) >= 1
         for it in range(n_it):
             _check_meta(view, w.spec, ospec, ods, n_videos, 0, 0, it)
-        _check_outputs(view, w.spec, ospec, ods, vids, 0, 0, 0)
+        samples = None
+        if clips is not None:   # whole clips (every view and frame) of the first `clips` batch slots
+            samples = [(b, k, t) for b in range(clips) for k, v in enumerate(w.spec.views) for t in range(v.clip_len)]
+        _check_outputs(view, w.spec, ospec, ods, vids, 0, 0, 0, samples=samples)
     finally:
         _teardown(store, view)
 
