@@ -199,7 +199,7 @@ def test_reuse_accounting_and_batch_bytes_match_oracle():
         _teardown(store, view)
     for name in ("k400", "ray", "twoview"):
         w = configs.get(name)
-        store, view, ospec, ods, vids = _setup(w, 6 if name == "ray" else 70)
+        store, view, ospec, ods, vids = _setup(w, 16 if name == "ray" else 70)
         try:
             bb = view.batch_bytes(0, 0, 0)
             ob = oracle.batch_bytes(ospec, ods, len(vids), 0, 0, 0)
