@@ -1,0 +1,484 @@
+// k_resample.cuh — fused resample kernel for items without rotation/blur
+// (DESIGN.md §7).
+//
+// One CTA = one work item (clip slot, source frame, group) x one band of R output rows.
+//  1. Separable tap tables: output column j -> (x0, x1, lambda_x); band row -> (y0, y1,
+//     lambda_y) with the exact fp32 rule of R#12.
+//  2. Source -> shared memory, two modes chosen per batch by the host:
+//     RAW    (scale <= ~2, Kinetics/SlowFast): the band's NV12 footprint (Y rows + UV rows,
+//            16 B aligned column span) is copied with cp.async (LDGSTS, all requests in
+//            flight at once), then converted in shared memory to packed RGBx, two pixels
+//            per thread sharing one chroma sample (a4, a5, Q1).
+//     GATHER (heavy down-scaling, 1080p Ray trials): only the tapped source columns and
+//            rows are touched: bitmaps + popcount prefix give a compact tap grid, whose
+//            pixels are gathered from HBM with 4 independent loads in flight per thread
+//            and converted (a4, a5).
+//  3. Two row-walker groups; each thread owns two adjacent output columns, walks down its
+//     half of the band and keeps the horizontal lerps of the two current source rows in
+//     registers, so each (source row, column) lerp is computed once (a6). Flip is the
+//     column mirror (a7). Vertical lerp, rint, normalise and packing run as FFMA2/FADD2
+//     pairs (sm_100a packed fp32), then one 4-byte store per (row, channel, destination)
+//     through per-destination pointers computed once (a10); every destination view of the
+//     group is written from the same registers (a11, node merging P:L277).
+// Every fp32 operation is the R#12/R#17 op sequence with IEEE rounding, so results are
+// bit-identical to the oracle (byte->float via the 2^23 exponent trick and rint via
+// +1.5*2^23 are exact for values in [0, 256)).
+#pragma once
+
+namespace sand {
+namespace rs {
+
+constexpr int kColWords = 128;             // GATHER: source column span <= 4096
+constexpr int kRowWords = 32;              // GATHER: band source row span <= 1024
+constexpr int kInlineDests = 2;            // destinations kept in registers
+constexpr float kBias = 8388608.0f;        // 2^23
+constexpr float kRound = 12582912.0f;      // 1.5 * 2^23
+
+__host__ __device__ inline size_t a16(size_t x) { return (x + 15) & ~size_t(15); }
+
+// --- shared layout: [tables][mode data] -----------------------------------------------
+struct Tables {
+  uint32_t* ctab_i;   // per output column j: x0 | x1 << 16 (grid-relative)
+  float* ctab_l;
+  uint32_t* rtab_i;   // per band row: y0 | y1 << 16 (grid-relative)
+  float* rtab_l;
+  int* misc;          // [0] grid width (words), [1] grid rows
+};
+
+__host__ __device__ inline size_t tables_bytes(int maxWo, int R) {
+  return 2 * a16((size_t)maxWo * 4) + 2 * a16((size_t)R * 4) + 16;
+}
+
+__device__ inline Tables carve_tables(uint8_t*& p, int maxWo, int R) {
+  Tables t;
+  t.ctab_i = reinterpret_cast<uint32_t*>(p); p += a16((size_t)maxWo * 4);
+  t.ctab_l = reinterpret_cast<float*>(p); p += a16((size_t)maxWo * 4);
+  t.rtab_i = reinterpret_cast<uint32_t*>(p); p += a16((size_t)R * 4);
+  t.rtab_l = reinterpret_cast<float*>(p); p += a16((size_t)R * 4);
+  t.misc = reinterpret_cast<int*>(p); p += 16;
+  return t;
+}
+
+// GATHER-mode bookkeeping
+__host__ __device__ inline size_t gather_meta_bytes(int maxWo, int R) {
+  return a16(kColWords * 4) + a16(kRowWords * 4) + a16(kColWords * 2) + a16(kRowWords * 2) +
+         a16((size_t)2 * maxWo * 2) + a16((size_t)2 * R * 2);
+}
+
+// source tap of output index o (R#12): s = max(sc*((float)(off+o)+0.5f)-0.5f, 0)
+__device__ __forceinline__ void tap(float sc, int off, int o, int lim, int org, int& i0, int& i1, float& lam) {
+  float s = __fadd_rn(__fmul_rn(sc, __fadd_rn((float)(off + o), 0.5f)), -0.5f);
+  s = fmaxf(s, 0.f);
+  const int i = (int)s;
+  lam = __fsub_rn(s, (float)i);
+  i0 = org + i;
+  i1 = org + min(i + 1, lim - 1);
+}
+
+__device__ __forceinline__ int tap0(float sc, int off, int o, int org) {
+  float s = __fadd_rn(__fmul_rn(sc, __fadd_rn((float)(off + o), 0.5f)), -0.5f);
+  return org + (int)fmaxf(s, 0.f);
+}
+
+// chroma terms of one (U,V) pair, shared by the pixels of a 2x2 block (R#11)
+struct Chroma {
+  int r, g, b;
+};
+__device__ __forceinline__ Chroma chroma(uint32_t uvpair) {
+  const int u = (int)(uvpair & 0xffu) - 128;
+  const int v = (int)((uvpair >> 8) & 0xffu) - 128;
+  return {1673527 * v, -852492 * v - 409993 * u, 2116026 * u};
+}
+__device__ __forceinline__ int sat8(int x) { return min(max(x, 0), 255); }
+__device__ __forceinline__ uint32_t rgbx(int Y, const Chroma& c) {
+  const int yy = max(Y - 16, 0) * 1220542 + (1 << 19);
+  return (uint32_t)sat8((yy + c.r) >> 20) | ((uint32_t)sat8((yy + c.g) >> 20) << 8) |
+         ((uint32_t)sat8((yy + c.b) >> 20) << 16);
+}
+
+// byte c of an RGBx word as the float 2^23 + byte (exact)
+__device__ __forceinline__ float biased(uint32_t w, int c) {
+  return __int_as_float((int)__byte_perm(w, 0x4B000000u, 0x7540u | (uint32_t)c));
+}
+
+struct Row3 {
+  float2 h[3];   // horizontal lerps of (column a, column b) per channel
+};
+
+__device__ __forceinline__ Row3 hrow(const uint32_t* __restrict__ grow, uint32_t ca, uint32_t cb, float2 lx) {
+  const uint32_t a0 = grow[ca & 0xffffu], a1 = grow[ca >> 16];
+  const uint32_t b0 = grow[cb & 0xffffu], b1 = grow[cb >> 16];
+  Row3 r;
+#pragma unroll
+  for (int c = 0; c < 3; ++c) {
+    const float2 P0 = make_float2(biased(a0, c), biased(b0, c));
+    const float2 P1 = make_float2(biased(a1, c), biased(b1, c));
+    const float2 d = __ffma2_rn(P0, make_float2(-1.f, -1.f), P1);          // p1 - p0 (exact)
+    const float2 p0 = __fadd2_rn(P0, make_float2(-kBias, -kBias));          // p0 (exact)
+    r.h[c] = __ffma2_rn(lx, d, p0);                                         // fmaf(l, p1 - p0, p0)
+  }
+  return r;
+}
+
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+  const uint32_t s = (uint32_t)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() {
+  asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
+}
+
+// One destination (view k, time t, clip b) of the thread's two columns.
+struct Dest {
+  uint8_t* row;         // element (c=0, oy=current row, ox) of this destination
+  uint32_t cstride;     // bytes between channel planes
+  uint32_t rstride;     // bytes between rows
+  float a[3], b[3];
+};
+
+__device__ __forceinline__ Dest make_dest(const LaunchParams& p, uint32_t dest, int oy, int ox) {
+  const uint32_t k = dest >> 24, t = (dest >> 16) & 0xffu, b = dest & 0xffffu;
+  const ViewConst& vc = p.views[k];
+  Dest d;
+  const size_t es = vc.dtype == SAND_U8 ? 1 : (vc.dtype == SAND_BF16 ? 2 : 4);
+  const size_t plane = (size_t)vc.out_h * vc.out_w;
+  d.cstride = (uint32_t)((size_t)vc.T * plane * es);
+  d.rstride = (uint32_t)((size_t)vc.out_w * es);
+  d.row = static_cast<uint8_t*>(p.out[k]) + ((((size_t)b * 3) * vc.T + t) * plane + (size_t)oy * vc.out_w + ox) * es;
+#pragma unroll
+  for (int c = 0; c < 3; ++c) {
+    d.a[c] = vc.a[c];
+    d.b[c] = vc.b[c];
+  }
+  return d;
+}
+
+// store quantised pair q of channel c; DT < 0: dtype read at run time
+template <int DT>
+__device__ __forceinline__ void put(const Dest& d, int dtype, int c, float2 q, bool vec, bool has_b) {
+  const int dt = DT >= 0 ? DT : dtype;
+  uint8_t* o = d.row + (size_t)c * d.cstride;
+  if (dt == SAND_BF16) {
+    const float2 y = __ffma2_rn(q, make_float2(d.a[c], d.a[c]), make_float2(d.b[c], d.b[c]));
+    if (vec) {
+      *reinterpret_cast<__nv_bfloat162*>(o) = __floats2bfloat162_rn(y.x, y.y);
+    } else {
+      reinterpret_cast<__nv_bfloat16*>(o)[0] = __float2bfloat16_rn(y.x);
+      if (has_b) reinterpret_cast<__nv_bfloat16*>(o)[1] = __float2bfloat16_rn(y.y);
+    }
+  } else if (dt == SAND_F32) {
+    const float2 y = __ffma2_rn(q, make_float2(d.a[c], d.a[c]), make_float2(d.b[c], d.b[c]));
+    if (vec) {
+      *reinterpret_cast<float2*>(o) = y;
+    } else {
+      reinterpret_cast<float*>(o)[0] = y.x;
+      if (has_b) reinterpret_cast<float*>(o)[1] = y.y;
+    }
+  } else {
+    if (vec) {
+      *reinterpret_cast<uint16_t*>(o) = (uint16_t)((uint32_t)q.x | ((uint32_t)q.y << 8));
+    } else {
+      o[0] = (uint8_t)q.x;
+      if (has_b) o[1] = (uint8_t)q.y;
+    }
+  }
+}
+
+// The row walk (step 3), shared by both modes. grid: RGBx rows of gw words.
+template <int DT>
+__device__ __forceinline__ void walk(const LaunchParams& p, const WorkItem& w, const GroupParams& g,
+                                     const Tables& t, const uint32_t* __restrict__ grid, int gw, int oy_lo,
+                                     int nrows) {
+  const int Wo = g.out_w;
+  const int pairs = (Wo + 1) >> 1;
+  const int P = blockDim.x >> 1;                       // threads per walker
+  const int walker = threadIdx.x / P;
+  if (walker >= 2) return;
+  const int half = (nrows + 1) >> 1;
+  const int rr_lo = walker * half, rr_hi = min(nrows, rr_lo + half);
+  const int nd = (int)w.n_dest;
+  const uint32_t* dests = p.dests + w.dest_begin;
+  for (int pair = threadIdx.x - walker * P; pair < pairs; pair += P) {
+    const int ox = 2 * pair;
+    const bool has_b = ox + 1 < Wo;
+    const bool vec = has_b && !(Wo & 1);
+    const int ja = g.flip ? Wo - 1 - ox : ox;
+    const int jb = has_b ? (g.flip ? Wo - 2 - ox : ox + 1) : ja;
+    const uint32_t ca = t.ctab_i[ja], cb = t.ctab_i[jb];
+    const float2 lx = make_float2(t.ctab_l[ja], t.ctab_l[jb]);
+    Dest dl[kInlineDests];
+    int dt[kInlineDests];
+#pragma unroll
+    for (int d = 0; d < kInlineDests; ++d)
+      if (d < nd) {
+        dl[d] = make_dest(p, dests[d], oy_lo + rr_lo, ox);
+        dt[d] = DT >= 0 ? DT : p.views[dests[d] >> 24].dtype;
+      }
+    int ra = -1, rb = -1;
+    Row3 Ha, Hb;
+    for (int rr = rr_lo; rr < rr_hi; ++rr) {
+      const uint32_t rt = t.rtab_i[rr];
+      const int r0 = (int)(rt & 0xffffu), r1 = (int)(rt >> 16);
+      const float ly1 = t.rtab_l[rr];
+      Row3 H0, H1;
+      if (r0 == rb) H0 = Hb;
+      else if (r0 == ra) H0 = Ha;
+      else H0 = hrow(grid + (size_t)r0 * gw, ca, cb, lx);
+      if (r1 == r0) H1 = H0;
+      else if (r1 == rb) H1 = Hb;
+      else H1 = hrow(grid + (size_t)r1 * gw, ca, cb, lx);
+      ra = r0; Ha = H0;
+      rb = r1; Hb = H1;
+      const float2 ly = make_float2(ly1, ly1);
+      float2 q[3];
+#pragma unroll
+      for (int c = 0; c < 3; ++c) {
+        const float2 dv = __ffma2_rn(H0.h[c], make_float2(-1.f, -1.f), H1.h[c]);   // h1 - h0
+        const float2 v = __ffma2_rn(ly, dv, H0.h[c]);                              // fmaf(ly, h1-h0, h0)
+        const float2 tq = __fadd2_rn(v, make_float2(kRound, kRound));              // rint (RNE)
+        q[c] = __fadd2_rn(tq, make_float2(-kRound, -kRound));
+      }
+#pragma unroll
+      for (int d = 0; d < kInlineDests; ++d) {
+        if (d < nd) {
+#pragma unroll
+          for (int c = 0; c < 3; ++c) put<DT>(dl[d], dt[d], c, q[c], vec, has_b);
+          dl[d].row += dl[d].rstride;
+        }
+      }
+      for (int d = kInlineDests; d < nd; ++d) {       // rare: more destinations than registers
+        const Dest e = make_dest(p, dests[d], oy_lo + rr, ox);
+        const int et = DT >= 0 ? DT : p.views[dests[d] >> 24].dtype;
+#pragma unroll
+        for (int c = 0; c < 3; ++c) put<DT>(e, et, c, q[c], vec, has_b);
+      }
+    }
+  }
+}
+
+}  // namespace rs
+
+// RAW mode: p launch params; R band rows; nbands; maxWo table sizing.
+template <int DT>
+__global__ void __launch_bounds__(224, 4) k_resample_raw(const LaunchParams p, int R, int nbands, int maxWo) {
+  extern __shared__ __align__(16) uint8_t smem_raw[];
+  using namespace rs;
+  const int item_idx = blockIdx.x / nbands;
+  const int band = blockIdx.x - item_idx * nbands;
+  const WorkItem w = p.items[item_idx];
+  if (w.flags & 1u) return;
+  const GroupParams& g = p.groups[w.gp];
+  const int Wo = g.out_w, Ho = g.out_h;
+  const int oy_lo = band * R;
+  if (oy_lo >= Ho) return;
+  const int nrows = min(R, Ho - oy_lo);
+  uint8_t* sp = smem_raw;
+  const Tables t = carve_tables(sp, maxWo, R);
+  const int tid = threadIdx.x, nthr = blockDim.x;
+
+  // footprint: monotone taps -> first/last output column and row bound it
+  const int x_lo = tap0(g.sc_x, g.off_x, 0, g.org_x);
+  int x_hi, y_lo, y_hi, dmy;
+  float fl;
+  tap(g.sc_x, g.off_x, Wo - 1, g.lim_x, g.org_x, dmy, x_hi, fl);
+  y_lo = tap0(g.sc_y, g.off_y, oy_lo, g.org_y);
+  tap(g.sc_y, g.off_y, oy_lo + nrows - 1, g.lim_y, g.org_y, dmy, y_hi, fl);
+  const int x16 = x_lo & ~15;
+  const int gw = ((x_hi + 16) & ~15) - x16;        // grid / raw row width (bytes of Y, words of RGBx)
+  const int ny = y_hi - y_lo + 1;
+  const int uv_lo = y_lo >> 1;
+  const int nuv = (y_hi >> 1) - uv_lo + 1;
+  uint8_t* rawY = sp;
+  uint8_t* rawUV = rawY + (size_t)ny * gw;
+  uint32_t* grid = reinterpret_cast<uint32_t*>(rawUV + a16((size_t)nuv * gw));
+
+  // 1. async copy of the NV12 footprint (16 B requests)
+  const uint8_t* Yp = p.slab + w.y_off;
+  const uint8_t* UVp = Yp + (size_t)w.pitch * w.src_h;
+  const int chunks = gw >> 4;
+  for (int e = tid; e < (ny + nuv) * chunks; e += nthr) {
+    const int r = e / chunks, k = e - r * chunks;
+    if (r < ny)
+      cp_async16(rawY + (size_t)r * gw + k * 16, Yp + (size_t)(y_lo + r) * w.pitch + x16 + k * 16);
+    else
+      cp_async16(rawUV + (size_t)(r - ny) * gw + k * 16, UVp + (size_t)(uv_lo + r - ny) * w.pitch + x16 + k * 16);
+  }
+  // 2. tap tables, grid-relative (overlaps the copy)
+  for (int j = tid; j < Wo; j += nthr) {
+    int x0, x1;
+    float lx;
+    tap(g.sc_x, g.off_x, j, g.lim_x, g.org_x, x0, x1, lx);
+    t.ctab_i[j] = (uint32_t)(x0 - x16) | ((uint32_t)(x1 - x16) << 16);
+    t.ctab_l[j] = lx;
+  }
+  for (int r = tid; r < nrows; r += nthr) {
+    int y0, y1;
+    float ly;
+    tap(g.sc_y, g.off_y, oy_lo + r, g.lim_y, g.org_y, y0, y1, ly);
+    t.rtab_i[r] = (uint32_t)(y0 - y_lo) | ((uint32_t)(y1 - y_lo) << 16);
+    t.rtab_l[r] = ly;
+  }
+  cp_async_wait_all();
+  __syncthreads();
+
+  // 3. NV12 -> RGBx in shared memory, two pixels (one chroma sample) per thread
+  const int hp = gw >> 1;
+  for (int e = tid; e < ny * hp; e += nthr) {
+    const int r = e / hp, k = e - r * hp;
+    const uint32_t ypair = *reinterpret_cast<const uint16_t*>(rawY + (size_t)r * gw + 2 * k);
+    const uint32_t uv = *reinterpret_cast<const uint16_t*>(rawUV + (size_t)(((y_lo + r) >> 1) - uv_lo) * gw + 2 * k);
+    const Chroma ch = chroma(uv);
+    uint2 o;
+    o.x = rgbx((int)(ypair & 0xffu), ch);
+    o.y = rgbx((int)(ypair >> 8), ch);
+    *reinterpret_cast<uint2*>(grid + (size_t)r * gw + 2 * k) = o;
+  }
+  __syncthreads();
+
+  // 4. row walk
+  walk<DT>(p, w, g, t, grid, gw, oy_lo, nrows);
+}
+
+// GATHER mode (heavy down-scaling): compact tap grid gathered from HBM.
+template <int DT>
+__global__ void __launch_bounds__(224, 4) k_resample_gather(const LaunchParams p, int R, int nbands, int maxWo) {
+  extern __shared__ __align__(16) uint8_t smem_raw[];
+  using namespace rs;
+  const int item_idx = blockIdx.x / nbands;
+  const int band = blockIdx.x - item_idx * nbands;
+  const WorkItem w = p.items[item_idx];
+  if (w.flags & 1u) return;
+  const GroupParams& g = p.groups[w.gp];
+  const int Wo = g.out_w, Ho = g.out_h;
+  const int oy_lo = band * R;
+  if (oy_lo >= Ho) return;
+  const int nrows = min(R, Ho - oy_lo);
+  uint8_t* sp = smem_raw;
+  const Tables t = carve_tables(sp, maxWo, R);
+  uint32_t* colbits = reinterpret_cast<uint32_t*>(sp); sp += a16(kColWords * 4);
+  uint32_t* rowbits = reinterpret_cast<uint32_t*>(sp); sp += a16(kRowWords * 4);
+  uint16_t* colpref = reinterpret_cast<uint16_t*>(sp); sp += a16(kColWords * 2);
+  uint16_t* rowpref = reinterpret_cast<uint16_t*>(sp); sp += a16(kRowWords * 2);
+  uint16_t* xs = reinterpret_cast<uint16_t*>(sp); sp += a16((size_t)2 * maxWo * 2);
+  uint16_t* ys = reinterpret_cast<uint16_t*>(sp); sp += a16((size_t)2 * R * 2);
+  uint32_t* grid = reinterpret_cast<uint32_t*>(sp);
+  const int tid = threadIdx.x, nthr = blockDim.x;
+  const int warp = tid >> 5, lane = tid & 31;
+
+  for (int i = tid; i < kColWords + kRowWords; i += nthr) {
+    if (i < kColWords) colbits[i] = 0u;
+    else rowbits[i - kColWords] = 0u;
+  }
+  const int cbase = tap0(g.sc_x, g.off_x, 0, g.org_x);
+  const int rbase = tap0(g.sc_y, g.off_y, oy_lo, g.org_y);
+  __syncthreads();
+  for (int j = tid; j < Wo; j += nthr) {
+    int x0, x1;
+    float lx;
+    tap(g.sc_x, g.off_x, j, g.lim_x, g.org_x, x0, x1, lx);
+    const int r0 = x0 - cbase, r1 = x1 - cbase;
+    t.ctab_i[j] = (uint32_t)r0 | ((uint32_t)r1 << 16);
+    t.ctab_l[j] = lx;
+    atomicOr(&colbits[r0 >> 5], 1u << (r0 & 31));
+    atomicOr(&colbits[r1 >> 5], 1u << (r1 & 31));
+  }
+  for (int r = tid; r < nrows; r += nthr) {
+    int y0, y1;
+    float ly;
+    tap(g.sc_y, g.off_y, oy_lo + r, g.lim_y, g.org_y, y0, y1, ly);
+    const int r0 = y0 - rbase, r1 = y1 - rbase;
+    t.rtab_i[r] = (uint32_t)r0 | ((uint32_t)r1 << 16);
+    t.rtab_l[r] = ly;
+    atomicOr(&rowbits[r0 >> 5], 1u << (r0 & 31));
+    atomicOr(&rowbits[r1 >> 5], 1u << (r1 & 31));
+  }
+  __syncthreads();
+  if (warp == 0) {   // exclusive popcount prefix of the column bitmap
+    uint32_t c[kColWords / 32];
+    uint32_t sum = 0;
+#pragma unroll
+    for (int k = 0; k < kColWords / 32; ++k) {
+      c[k] = __popc(colbits[lane * (kColWords / 32) + k]);
+      sum += c[k];
+    }
+    uint32_t incl = sum;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t o = __shfl_up_sync(0xffffffffu, incl, d);
+      if (lane >= d) incl += o;
+    }
+    uint32_t run = incl - sum;
+#pragma unroll
+    for (int k = 0; k < kColWords / 32; ++k) {
+      colpref[lane * (kColWords / 32) + k] = (uint16_t)run;
+      run += c[k];
+    }
+    if (lane == 31) t.misc[0] = (int)incl;
+  }
+  if (warp == (nthr > 32 ? 1 : 0)) {   // ... and of the row bitmap
+    const uint32_t c = __popc(rowbits[lane]);
+    uint32_t incl = c;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t o = __shfl_up_sync(0xffffffffu, incl, d);
+      if (lane >= d) incl += o;
+    }
+    rowpref[lane] = (uint16_t)(incl - c);
+    if (lane == 31) t.misc[1] = (int)incl;
+  }
+  __syncthreads();
+  for (int wd = tid; wd < kColWords + kRowWords; wd += nthr) {
+    const bool col = wd < kColWords;
+    const int k0 = col ? wd : wd - kColWords;
+    uint32_t b = col ? colbits[k0] : rowbits[k0];
+    int k = col ? colpref[k0] : rowpref[k0];
+    const int base = (col ? cbase : rbase) + k0 * 32;
+    uint16_t* dst = col ? xs : ys;
+    while (b) {
+      const int bit = __ffs(b) - 1;
+      b &= b - 1;
+      dst[k++] = (uint16_t)(base + bit);
+    }
+  }
+  auto cidx = [&](const uint32_t* bits, const uint16_t* pref, int r) -> uint32_t {
+    return pref[r >> 5] + __popc(bits[r >> 5] & ((1u << (r & 31)) - 1u));
+  };
+  for (int j = tid; j < Wo; j += nthr) {
+    const uint32_t v = t.ctab_i[j];
+    t.ctab_i[j] = cidx(colbits, colpref, (int)(v & 0xffffu)) | (cidx(colbits, colpref, (int)(v >> 16)) << 16);
+  }
+  for (int r = tid; r < nrows; r += nthr) {
+    const uint32_t v = t.rtab_i[r];
+    t.rtab_i[r] = cidx(rowbits, rowpref, (int)(v & 0xffffu)) | (cidx(rowbits, rowpref, (int)(v >> 16)) << 16);
+  }
+  __syncthreads();
+
+  // gather-convert with 4 independent loads in flight per thread
+  const int nX = t.misc[0], nY = t.misc[1];
+  const uint8_t* Yp = p.slab + w.y_off;
+  const uint8_t* UVp = Yp + (size_t)w.pitch * w.src_h;
+  const int total = nX * nY;
+  for (int e0 = tid; e0 < total; e0 += 4 * nthr) {
+    int yv[4];
+    uint32_t uvv[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int e = e0 + u * nthr;
+      if (e < total) {
+        const int i = e / nX, jj = e - i * nX;
+        const int x = xs[jj], y = ys[i];
+        yv[u] = __ldg(Yp + (size_t)y * w.pitch + x);
+        uvv[u] = __ldg(reinterpret_cast<const uint16_t*>(UVp + (size_t)(y >> 1) * w.pitch + (x & ~1)));
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int e = e0 + u * nthr;
+      if (e < total) grid[e] = rgbx(yv[u], chroma(uvv[u]));
+    }
+  }
+  __syncthreads();
+  walk<DT>(p, w, g, t, grid, nX, oy_lo, nrows);
+}
+
+}  // namespace sand

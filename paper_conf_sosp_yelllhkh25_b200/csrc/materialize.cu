@@ -1,6 +1,6 @@
 // materialize.cu — sm_100a kernels of the materialisation path.
 //
-//  * k_tapgrid (k_tapgrid.cuh): items without rotation/blur — banded tap-grid resample,
+//  * k_resample_{raw,gather} (k_resample.cuh): items without rotation/blur — banded resample,
 //               one CTA per (work item, band of output rows).
 //  * k_stencil: items with rotation and/or blur, one CTA per work item. Per channel: Q2 plane in shared
 //               memory -> rotated Q3 plane -> separable blur in row strips (fp32
@@ -13,6 +13,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <string>
 
 #include "plan_types.h"
@@ -167,24 +168,70 @@ __global__ void __launch_bounds__(512) k_stencil(const LaunchParams p) {
 }  // namespace
 }  // namespace sand
 
-#include "k_tapgrid.cuh"
+#include "k_resample.cuh"
 
 namespace sand {
 
 namespace {
-constexpr size_t kTgSmemBudget = 55 * 1024;   // 4 CTAs / SM
+// Shared-memory budget per resample CTA: 4 CTAs of 7 warps per SM (tunable for experiments).
+size_t smem_budget() {
+  static size_t b = [] {
+    const char* e = getenv("SAND_SMEM_BUDGET_KB");
+    return (size_t)(e ? atoi(e) : 55) * 1024;
+  }();
+  return b;
+}
 
-// band height R and dynamic shared memory of k_tapgrid for a batch shape
-void choose_tapgrid(const BatchShape& sh, int* R, size_t* smem) {
-  static const int kCands[] = {64, 48, 32, 24, 16, 8, 4, 2, 1};
-  for (int r : kCands) {
-    const int span = static_cast<int>(std::ceil(static_cast<double>(sh.max_scy) * r)) + 3;   // row bitmap span
-    const int rows = std::min(2 * r, span);
-    const size_t bytes = tg::table_bytes(sh.max_wo, r) + (size_t)rows * sh.cols_bound * 4;
-    *R = r;
-    *smem = bytes;
-    if ((bytes <= kTgSmemBudget && span <= 32 * tg::kRowWords) || r == 1) return;
+struct ResampleCfg {
+  bool raw;
+  int R;
+  size_t smem;
+};
+
+// mode, band height and dynamic shared memory of the resample kernel for a batch shape
+ResampleCfg choose_resample(const BatchShape& sh) {
+  static const int kCands[] = {64, 48, 32, 24, 16, 12, 8, 4, 2, 1};
+  const bool mild = sh.cols_bound <= 2 * sh.max_wo + 16 && sh.max_scy <= 2.0f;
+  const size_t gwb = rs::a16((size_t)sh.cols_bound) + 16;
+  if (mild) {
+    for (int r : kCands) {
+      const size_t rows = (size_t)std::ceil((double)sh.max_scy * r) + 3;
+      const size_t bytes = rs::tables_bytes(sh.max_wo, r) + rows * gwb + rs::a16((rows / 2 + 2) * gwb) + rows * gwb * 4;
+      if (bytes <= smem_budget() || (r <= 8 && bytes <= 200 * 1024)) return {true, r, bytes};
+    }
   }
+  for (int r : kCands) {
+    const int span = (int)std::ceil((double)sh.max_scy * r) + 3;
+    const size_t rows = (size_t)std::min(2 * r, span);
+    const size_t cols = (size_t)std::min(2 * sh.max_wo, sh.cols_bound);
+    const size_t bytes = rs::tables_bytes(sh.max_wo, r) + rs::gather_meta_bytes(sh.max_wo, r) + rows * cols * 4;
+    if ((bytes <= smem_budget() && span <= 32 * rs::kRowWords) || r == 1) return {false, r, bytes};
+  }
+  return {false, 1, 0};
+}
+
+template <int DT>
+int launch_resample_dt(const LaunchParams& p, const BatchShape& sh, cudaStream_t stream) {
+  const ResampleCfg cfg = choose_resample(sh);
+  if (cfg.smem > 227 * 1024) return set_error(SAND_EINVAL, "resample tile exceeds shared memory (source crop too large)");
+  const int nbands = (sh.max_ho + cfg.R - 1) / cfg.R;
+  const int pairs = (sh.max_wo + 1) / 2;
+  const int threads = std::min(224, ((2 * pairs + 31) / 32) * 32);
+  const unsigned blocks = (unsigned)((uint64_t)p.n_items * nbands);
+  if (cfg.raw)
+    k_resample_raw<DT><<<blocks, threads, cfg.smem, stream>>>(p, cfg.R, nbands, sh.max_wo);
+  else
+    k_resample_gather<DT><<<blocks, threads, cfg.smem, stream>>>(p, cfg.R, nbands, sh.max_wo);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_error(e, "k_resample launch");
+  return SAND_OK;
+}
+
+template <typename K>
+cudaError_t allow_smem(K kernel) {
+  cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(kernel, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
 }
 }  // namespace
 
@@ -195,8 +242,13 @@ size_t stencil_smem_bytes(int max_h, int max_w, int max_r) {
 
 int configure_kernels(size_t stencil_smem) {
   {
-    cudaError_t e = cudaFuncSetAttribute(k_tapgrid, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-    if (e != cudaSuccess) return cuda_error(e, "cudaFuncSetAttribute(k_tapgrid)");
+    cudaError_t e = cudaSuccess;
+    for (cudaError_t r : {allow_smem(k_resample_raw<-1>), allow_smem(k_resample_raw<SAND_U8>),
+                          allow_smem(k_resample_raw<SAND_BF16>), allow_smem(k_resample_raw<SAND_F32>),
+                          allow_smem(k_resample_gather<-1>), allow_smem(k_resample_gather<SAND_U8>),
+                          allow_smem(k_resample_gather<SAND_BF16>), allow_smem(k_resample_gather<SAND_F32>)})
+      if (r != cudaSuccess) e = r;
+    if (e != cudaSuccess) return cuda_error(e, "cudaFuncSetAttribute(k_resample)");
   }
   if (stencil_smem > 0) {
     if (stencil_smem > 227 * 1024) return set_error(SAND_EINVAL, "stencil shared memory exceeds 227 KB");
@@ -211,17 +263,14 @@ int launch_materialize(const LaunchParams& p, const BatchShape& shape, size_t st
   *n_launched = 0;
   if (p.n_items == 0) return SAND_OK;
   if (shape.has_direct) {
-    int R;
-    size_t smem;
-    choose_tapgrid(shape, &R, &smem);
-    if (smem > 227 * 1024) return set_error(SAND_EINVAL, "tap grid exceeds shared memory (source crop too large)");
-    const int nbands = (shape.max_ho + R - 1) / R;
-    const int pairs = (shape.max_wo + 1) / 2;
-    const int threads = std::min(256, ((2 * pairs + 31) / 32) * 32);
-    const uint64_t blocks = (uint64_t)p.n_items * nbands;
-    k_tapgrid<<<(unsigned)blocks, threads, smem, stream>>>(p, R, nbands, shape.max_wo);
-    cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) return cuda_error(e, "k_tapgrid launch");
+    int rc;
+    switch (shape.dtype) {
+      case SAND_U8: rc = launch_resample_dt<SAND_U8>(p, shape, stream); break;
+      case SAND_BF16: rc = launch_resample_dt<SAND_BF16>(p, shape, stream); break;
+      case SAND_F32: rc = launch_resample_dt<SAND_F32>(p, shape, stream); break;
+      default: rc = launch_resample_dt<-1>(p, shape, stream); break;
+    }
+    if (rc != SAND_OK) return rc;
     ++*n_launched;
   }
   if (shape.has_stencil) {

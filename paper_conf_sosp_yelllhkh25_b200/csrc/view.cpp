@@ -90,8 +90,12 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
   plan->groups.resize(n_clips * nG);
   plan->item_begin.push_back(0);
   plan->fetch_begin.push_back(0);
+  int32_t common_dtype = s.views[0].out_dtype;
+  for (uint32_t k = 1; k < s.n_views; ++k)
+    if (s.views[k].out_dtype != common_dtype) common_dtype = -1;
   for (uint64_t it = 0; it < plan->iterations; ++it) {
     BatchShape shape{};
+    shape.dtype = common_dtype;
     std::vector<std::pair<uint64_t, uint32_t>> fetch;   // ((video<<32)|frame, uses)
     for (uint32_t b = 0; b < B; ++b) {
       const uint64_t slot = it * B + b;
