@@ -38,23 +38,19 @@ __host__ __device__ inline size_t a16(size_t x) { return (x + 15) & ~size_t(15);
 
 // --- shared layout: [tables][mode data] -----------------------------------------------
 struct Tables {
-  uint32_t* ctab_i;   // per output column j: x0 | x1 << 16 (grid-relative)
-  float* ctab_l;
-  uint32_t* rtab_i;   // per band row: y0 | y1 << 16 (grid-relative)
-  float* rtab_l;
-  int* misc;          // [0] grid width (words), [1] grid rows
+  uint2* ctab;        // per output column j: (x0 | x1 << 16 grid-relative, bits of lambda_x)
+  uint2* rtab;        // per band row: (y0 | y1 << 16 grid-relative, bits of lambda_y)
+  int* misc;          // GATHER: [0] tapped columns, [1] tapped rows
 };
 
 __host__ __device__ inline size_t tables_bytes(int maxWo, int R) {
-  return 2 * a16((size_t)maxWo * 4) + 2 * a16((size_t)R * 4) + 16;
+  return a16((size_t)maxWo * 8) + a16((size_t)R * 8) + 16;
 }
 
 __device__ inline Tables carve_tables(uint8_t*& p, int maxWo, int R) {
   Tables t;
-  t.ctab_i = reinterpret_cast<uint32_t*>(p); p += a16((size_t)maxWo * 4);
-  t.ctab_l = reinterpret_cast<float*>(p); p += a16((size_t)maxWo * 4);
-  t.rtab_i = reinterpret_cast<uint32_t*>(p); p += a16((size_t)R * 4);
-  t.rtab_l = reinterpret_cast<float*>(p); p += a16((size_t)R * 4);
+  t.ctab = reinterpret_cast<uint2*>(p); p += a16((size_t)maxWo * 8);
+  t.rtab = reinterpret_cast<uint2*>(p); p += a16((size_t)R * 8);
   t.misc = reinterpret_cast<int*>(p); p += 16;
   return t;
 }
@@ -185,6 +181,61 @@ __device__ __forceinline__ void put(const Dest& d, int dtype, int c, float2 q, b
 }
 
 // The row walk (step 3), shared by both modes. grid: RGBx rows of gw words.
+// Walk band rows [rr_lo, rr_hi) for the output column pair (ox, ox+1). ND: destinations in
+// registers (1, or 2 plus a loop over the rest). The pair of current source rows (r0c, r1c)
+// and their horizontal lerps (H0, H1) advance monotonically: y1 = min(y0+1, lim-1) is a
+// function of y0, so both change together; a shift by one row reuses H1 as the new H0.
+template <int DT, int ND>
+__device__ __forceinline__ void walk_rows(const LaunchParams& p, const uint32_t* __restrict__ dests, int nd,
+                                          const uint2* __restrict__ rtab, const uint32_t* __restrict__ grid,
+                                          int gw, int oy0, int rr_lo, int rr_hi, int ox, uint32_t ca, uint32_t cb,
+                                          float2 lx, bool vec, bool has_b) {
+  Dest dl[ND];
+  int dt[ND];
+#pragma unroll
+  for (int d = 0; d < ND; ++d) {
+    dl[d] = make_dest(p, dests[d], oy0 + rr_lo, ox);
+    dt[d] = DT >= 0 ? DT : p.views[dests[d] >> 24].dtype;
+  }
+  int r0c = -1, r1c = -1;
+  Row3 H0, H1;
+  for (int rr = rr_lo; rr < rr_hi; ++rr) {
+    const uint2 rt = rtab[rr];
+    const int r0 = (int)(rt.x & 0xffffu), r1 = (int)(rt.x >> 16);
+    if (r0 != r0c) {
+      if (r0 == r1c) H0 = H1;
+      else H0 = hrow(grid + (size_t)r0 * gw, ca, cb, lx);
+      if (r1 == r0) H1 = H0;
+      else H1 = hrow(grid + (size_t)r1 * gw, ca, cb, lx);
+      r0c = r0;
+      r1c = r1;
+    }
+    const float l = __uint_as_float(rt.y);
+    const float2 ly = make_float2(l, l);
+    float2 q[3];
+#pragma unroll
+    for (int c = 0; c < 3; ++c) {
+      const float2 dv = __ffma2_rn(H0.h[c], make_float2(-1.f, -1.f), H1.h[c]);   // h1 - h0
+      const float2 v = __ffma2_rn(ly, dv, H0.h[c]);                              // fmaf(ly, h1-h0, h0)
+      const float2 tq = __fadd2_rn(v, make_float2(kRound, kRound));              // rint (RNE)
+      q[c] = __fadd2_rn(tq, make_float2(-kRound, -kRound));
+    }
+#pragma unroll
+    for (int d = 0; d < ND; ++d) {
+#pragma unroll
+      for (int c = 0; c < 3; ++c) put<DT>(dl[d], dt[d], c, q[c], vec, has_b);
+      dl[d].row += dl[d].rstride;
+    }
+    for (int d = ND; d < nd; ++d) {       // rare: more destinations than registers
+      const Dest e = make_dest(p, dests[d], oy0 + rr, ox);
+      const int et = DT >= 0 ? DT : p.views[dests[d] >> 24].dtype;
+#pragma unroll
+      for (int c = 0; c < 3; ++c) put<DT>(e, et, c, q[c], vec, has_b);
+    }
+  }
+}
+
+// The row walk (step 3), shared by both modes. grid: RGBx rows of gw words.
 template <int DT>
 __device__ __forceinline__ void walk(const LaunchParams& p, const WorkItem& w, const GroupParams& g,
                                      const Tables& t, const uint32_t* __restrict__ grid, int gw, int oy_lo,
@@ -192,67 +243,25 @@ __device__ __forceinline__ void walk(const LaunchParams& p, const WorkItem& w, c
   const int Wo = g.out_w;
   const int pairs = (Wo + 1) >> 1;
   const int P = blockDim.x >> 1;                       // threads per walker
-  const int walker = threadIdx.x / P;
-  if (walker >= 2) return;
+  const int walker = threadIdx.x >= P ? 1 : 0;
   const int half = (nrows + 1) >> 1;
   const int rr_lo = walker * half, rr_hi = min(nrows, rr_lo + half);
   const int nd = (int)w.n_dest;
   const uint32_t* dests = p.dests + w.dest_begin;
+  const uint2* rtab = reinterpret_cast<const uint2*>(t.rtab);
   for (int pair = threadIdx.x - walker * P; pair < pairs; pair += P) {
     const int ox = 2 * pair;
     const bool has_b = ox + 1 < Wo;
     const bool vec = has_b && !(Wo & 1);
     const int ja = g.flip ? Wo - 1 - ox : ox;
     const int jb = has_b ? (g.flip ? Wo - 2 - ox : ox + 1) : ja;
-    const uint32_t ca = t.ctab_i[ja], cb = t.ctab_i[jb];
-    const float2 lx = make_float2(t.ctab_l[ja], t.ctab_l[jb]);
-    Dest dl[kInlineDests];
-    int dt[kInlineDests];
-#pragma unroll
-    for (int d = 0; d < kInlineDests; ++d)
-      if (d < nd) {
-        dl[d] = make_dest(p, dests[d], oy_lo + rr_lo, ox);
-        dt[d] = DT >= 0 ? DT : p.views[dests[d] >> 24].dtype;
-      }
-    int ra = -1, rb = -1;
-    Row3 Ha, Hb;
-    for (int rr = rr_lo; rr < rr_hi; ++rr) {
-      const uint32_t rt = t.rtab_i[rr];
-      const int r0 = (int)(rt & 0xffffu), r1 = (int)(rt >> 16);
-      const float ly1 = t.rtab_l[rr];
-      Row3 H0, H1;
-      if (r0 == rb) H0 = Hb;
-      else if (r0 == ra) H0 = Ha;
-      else H0 = hrow(grid + (size_t)r0 * gw, ca, cb, lx);
-      if (r1 == r0) H1 = H0;
-      else if (r1 == rb) H1 = Hb;
-      else H1 = hrow(grid + (size_t)r1 * gw, ca, cb, lx);
-      ra = r0; Ha = H0;
-      rb = r1; Hb = H1;
-      const float2 ly = make_float2(ly1, ly1);
-      float2 q[3];
-#pragma unroll
-      for (int c = 0; c < 3; ++c) {
-        const float2 dv = __ffma2_rn(H0.h[c], make_float2(-1.f, -1.f), H1.h[c]);   // h1 - h0
-        const float2 v = __ffma2_rn(ly, dv, H0.h[c]);                              // fmaf(ly, h1-h0, h0)
-        const float2 tq = __fadd2_rn(v, make_float2(kRound, kRound));              // rint (RNE)
-        q[c] = __fadd2_rn(tq, make_float2(-kRound, -kRound));
-      }
-#pragma unroll
-      for (int d = 0; d < kInlineDests; ++d) {
-        if (d < nd) {
-#pragma unroll
-          for (int c = 0; c < 3; ++c) put<DT>(dl[d], dt[d], c, q[c], vec, has_b);
-          dl[d].row += dl[d].rstride;
-        }
-      }
-      for (int d = kInlineDests; d < nd; ++d) {       // rare: more destinations than registers
-        const Dest e = make_dest(p, dests[d], oy_lo + rr, ox);
-        const int et = DT >= 0 ? DT : p.views[dests[d] >> 24].dtype;
-#pragma unroll
-        for (int c = 0; c < 3; ++c) put<DT>(e, et, c, q[c], vec, has_b);
-      }
-    }
+    const uint2 ta = t.ctab[ja], tb = t.ctab[jb];
+    const float2 lx = make_float2(__uint_as_float(ta.y), __uint_as_float(tb.y));
+    if (nd == 1)
+      walk_rows<DT, 1>(p, dests, nd, rtab, grid, gw, oy_lo, rr_lo, rr_hi, ox, ta.x, tb.x, lx, vec, has_b);
+    else
+      walk_rows<DT, kInlineDests>(p, dests, nd, rtab, grid, gw, oy_lo, rr_lo, rr_hi, ox, ta.x, tb.x, lx, vec,
+                                  has_b);
   }
 }
 
@@ -296,42 +305,62 @@ __global__ void __launch_bounds__(224, 4) k_resample_raw(const LaunchParams p, i
   const uint8_t* Yp = p.slab + w.y_off;
   const uint8_t* UVp = Yp + (size_t)w.pitch * w.src_h;
   const int chunks = gw >> 4;
-  for (int e = tid; e < (ny + nuv) * chunks; e += nthr) {
-    const int r = e / chunks, k = e - r * chunks;
-    if (r < ny)
-      cp_async16(rawY + (size_t)r * gw + k * 16, Yp + (size_t)(y_lo + r) * w.pitch + x16 + k * 16);
-    else
-      cp_async16(rawUV + (size_t)(r - ny) * gw + k * 16, UVp + (size_t)(uv_lo + r - ny) * w.pitch + x16 + k * 16);
+  {
+    // thread -> (row slot, chunk): rows advance by nthr / chunks per pass, no division in the loop
+    const int rows_per_pass = max(1, nthr / chunks);
+    const int k = tid % chunks, r0 = tid / chunks;
+    if (r0 < rows_per_pass)
+      for (int r = r0; r < ny + nuv; r += rows_per_pass) {
+        if (r < ny)
+          cp_async16(rawY + (size_t)r * gw + k * 16, Yp + (size_t)(y_lo + r) * w.pitch + x16 + k * 16);
+        else
+          cp_async16(rawUV + (size_t)(r - ny) * gw + k * 16, UVp + (size_t)(uv_lo + r - ny) * w.pitch + x16 + k * 16);
+      }
+    for (int kk = k + nthr; kk < chunks; kk += nthr)     // only if a row has more chunks than threads
+      for (int r = 0; r < ny + nuv; ++r) {
+        if (r < ny)
+          cp_async16(rawY + (size_t)r * gw + kk * 16, Yp + (size_t)(y_lo + r) * w.pitch + x16 + kk * 16);
+        else
+          cp_async16(rawUV + (size_t)(r - ny) * gw + kk * 16, UVp + (size_t)(uv_lo + r - ny) * w.pitch + x16 + kk * 16);
+      }
   }
   // 2. tap tables, grid-relative (overlaps the copy)
   for (int j = tid; j < Wo; j += nthr) {
     int x0, x1;
     float lx;
     tap(g.sc_x, g.off_x, j, g.lim_x, g.org_x, x0, x1, lx);
-    t.ctab_i[j] = (uint32_t)(x0 - x16) | ((uint32_t)(x1 - x16) << 16);
-    t.ctab_l[j] = lx;
+    t.ctab[j] = make_uint2((uint32_t)(x0 - x16) | ((uint32_t)(x1 - x16) << 16), __float_as_uint(lx));
   }
   for (int r = tid; r < nrows; r += nthr) {
     int y0, y1;
     float ly;
     tap(g.sc_y, g.off_y, oy_lo + r, g.lim_y, g.org_y, y0, y1, ly);
-    t.rtab_i[r] = (uint32_t)(y0 - y_lo) | ((uint32_t)(y1 - y_lo) << 16);
-    t.rtab_l[r] = ly;
+    t.rtab[r] = make_uint2((uint32_t)(y0 - y_lo) | ((uint32_t)(y1 - y_lo) << 16), __float_as_uint(ly));
   }
   cp_async_wait_all();
   __syncthreads();
 
-  // 3. NV12 -> RGBx in shared memory, two pixels (one chroma sample) per thread
+  // 3. NV12 -> RGBx in shared memory: a thread takes one chroma sample and the (up to) 2x2
+  //    luma pixels that share it; warps walk chroma rows, lanes walk chroma columns
   const int hp = gw >> 1;
-  for (int e = tid; e < ny * hp; e += nthr) {
-    const int r = e / hp, k = e - r * hp;
-    const uint32_t ypair = *reinterpret_cast<const uint16_t*>(rawY + (size_t)r * gw + 2 * k);
-    const uint32_t uv = *reinterpret_cast<const uint16_t*>(rawUV + (size_t)(((y_lo + r) >> 1) - uv_lo) * gw + 2 * k);
-    const Chroma ch = chroma(uv);
-    uint2 o;
-    o.x = rgbx((int)(ypair & 0xffu), ch);
-    o.y = rgbx((int)(ypair >> 8), ch);
-    *reinterpret_cast<uint2*>(grid + (size_t)r * gw + 2 * k) = o;
+  const int nwarps = nthr >> 5, lane = tid & 31;
+  for (int u = tid >> 5; u < nuv; u += nwarps) {
+    const int ytop = 2 * (uv_lo + u) - y_lo;      // grid rows ytop, ytop+1 (may fall outside)
+    const bool top = ytop >= 0, bot = ytop + 1 < ny;
+    const uint8_t* uvrow = rawUV + (size_t)u * gw;
+    for (int k = lane; k < hp; k += 32) {
+      const Chroma ch = chroma(*reinterpret_cast<const uint16_t*>(uvrow + 2 * k));
+      if (top) {
+        const uint32_t yp = *reinterpret_cast<const uint16_t*>(rawY + (size_t)ytop * gw + 2 * k);
+        *reinterpret_cast<uint2*>(grid + (size_t)ytop * gw + 2 * k) =
+            make_uint2(rgbx((int)(yp & 0xffu), ch), rgbx((int)(yp >> 8), ch));
+      }
+      if (bot) {
+        const uint32_t yp = *reinterpret_cast<const uint16_t*>(rawY + (size_t)(ytop + 1) * gw + 2 * k);
+        *reinterpret_cast<uint2*>(grid + (size_t)(ytop + 1) * gw + 2 * k) =
+            make_uint2(rgbx((int)(yp & 0xffu), ch), rgbx((int)(yp >> 8), ch));
+      }
+    }
   }
   __syncthreads();
 
@@ -377,8 +406,7 @@ __global__ void __launch_bounds__(224, 4) k_resample_gather(const LaunchParams p
     float lx;
     tap(g.sc_x, g.off_x, j, g.lim_x, g.org_x, x0, x1, lx);
     const int r0 = x0 - cbase, r1 = x1 - cbase;
-    t.ctab_i[j] = (uint32_t)r0 | ((uint32_t)r1 << 16);
-    t.ctab_l[j] = lx;
+    t.ctab[j] = make_uint2((uint32_t)r0 | ((uint32_t)r1 << 16), __float_as_uint(lx));
     atomicOr(&colbits[r0 >> 5], 1u << (r0 & 31));
     atomicOr(&colbits[r1 >> 5], 1u << (r1 & 31));
   }
@@ -387,8 +415,7 @@ __global__ void __launch_bounds__(224, 4) k_resample_gather(const LaunchParams p
     float ly;
     tap(g.sc_y, g.off_y, oy_lo + r, g.lim_y, g.org_y, y0, y1, ly);
     const int r0 = y0 - rbase, r1 = y1 - rbase;
-    t.rtab_i[r] = (uint32_t)r0 | ((uint32_t)r1 << 16);
-    t.rtab_l[r] = ly;
+    t.rtab[r] = make_uint2((uint32_t)r0 | ((uint32_t)r1 << 16), __float_as_uint(ly));
     atomicOr(&rowbits[r0 >> 5], 1u << (r0 & 31));
     atomicOr(&rowbits[r1 >> 5], 1u << (r1 & 31));
   }
@@ -444,12 +471,12 @@ __global__ void __launch_bounds__(224, 4) k_resample_gather(const LaunchParams p
     return pref[r >> 5] + __popc(bits[r >> 5] & ((1u << (r & 31)) - 1u));
   };
   for (int j = tid; j < Wo; j += nthr) {
-    const uint32_t v = t.ctab_i[j];
-    t.ctab_i[j] = cidx(colbits, colpref, (int)(v & 0xffffu)) | (cidx(colbits, colpref, (int)(v >> 16)) << 16);
+    const uint32_t v = t.ctab[j].x;
+    t.ctab[j].x = cidx(colbits, colpref, (int)(v & 0xffffu)) | (cidx(colbits, colpref, (int)(v >> 16)) << 16);
   }
   for (int r = tid; r < nrows; r += nthr) {
-    const uint32_t v = t.rtab_i[r];
-    t.rtab_i[r] = cidx(rowbits, rowpref, (int)(v & 0xffffu)) | (cidx(rowbits, rowpref, (int)(v >> 16)) << 16);
+    const uint32_t v = t.rtab[r].x;
+    t.rtab[r].x = cidx(rowbits, rowpref, (int)(v & 0xffffu)) | (cidx(rowbits, rowpref, (int)(v >> 16)) << 16);
   }
   __syncthreads();
 
@@ -457,24 +484,29 @@ __global__ void __launch_bounds__(224, 4) k_resample_gather(const LaunchParams p
   const int nX = t.misc[0], nY = t.misc[1];
   const uint8_t* Yp = p.slab + w.y_off;
   const uint8_t* UVp = Yp + (size_t)w.pitch * w.src_h;
-  const int total = nX * nY;
-  for (int e0 = tid; e0 < total; e0 += 4 * nthr) {
-    int yv[4];
-    uint32_t uvv[4];
+  const int nwarps = nthr >> 5;
+  for (int i = warp; i < nY; i += nwarps) {
+    const int y = ys[i];
+    const uint8_t* yrow = Yp + (size_t)y * w.pitch;
+    const uint8_t* uvrow = UVp + (size_t)(y >> 1) * w.pitch;
+    uint32_t* grow = grid + (size_t)i * nX;
+    for (int j0 = lane; j0 < nX; j0 += 128) {
+      int yv[4];
+      uint32_t uvv[4];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const int e = e0 + u * nthr;
-      if (e < total) {
-        const int i = e / nX, jj = e - i * nX;
-        const int x = xs[jj], y = ys[i];
-        yv[u] = __ldg(Yp + (size_t)y * w.pitch + x);
-        uvv[u] = __ldg(reinterpret_cast<const uint16_t*>(UVp + (size_t)(y >> 1) * w.pitch + (x & ~1)));
+      for (int u = 0; u < 4; ++u) {
+        const int jj = j0 + 32 * u;
+        if (jj < nX) {
+          const int x = xs[jj];
+          yv[u] = __ldg(yrow + x);
+          uvv[u] = __ldg(reinterpret_cast<const uint16_t*>(uvrow + (x & ~1)));
+        }
       }
-    }
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const int e = e0 + u * nthr;
-      if (e < total) grid[e] = rgbx(yv[u], chroma(uvv[u]));
+      for (int u = 0; u < 4; ++u) {
+        const int jj = j0 + 32 * u;
+        if (jj < nX) grow[jj] = rgbx(yv[u], chroma(uvv[u]));
+      }
     }
   }
   __syncthreads();

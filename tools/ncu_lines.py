@@ -17,6 +17,18 @@ import sys
 import tempfile
 
 
+def mangled_match(kernel, line):
+    """kernel like 'k_resample_raw<1>' matches the mangled '14k_resample_rawILi1EE...'."""
+    m = re.match(r"(\w+)(?:<(-?\d+)>)?", kernel)
+    name, targ = m.group(1), m.group(2)
+    if name not in line:
+        return False
+    if targ is None:
+        return True
+    t = ("Lin" + targ[1:]) if targ.startswith("-") else ("Li" + targ)
+    return f"{name}I{t}E" in line
+
+
 def sass_lines(obj, kernel):
     d = tempfile.mkdtemp()
     if obj.endswith(".o") or obj.endswith(".so"):
@@ -31,7 +43,7 @@ def sass_lines(obj, kernel):
         infn = False
         for ln in txt.splitlines():
             if ln.startswith("//----") and ".text." in ln:
-                infn = kernel in ln
+                infn = mangled_match(kernel, ln)
                 continue
             if not infn:
                 continue
@@ -62,7 +74,7 @@ def main():
             hdr = r
         elif cur is not None and hdr and len(r) >= len(hdr) - 1:
             cur["rows"].append(r)
-    blk = next(b for b in blocks if kernel in b["name"])
+    blk = next(b for b in blocks if kernel in b["name"].replace(" ", "").replace("(int)", ""))
     ie, st, src = hdr.index("Instructions Executed"), hdr.index("Warp Stall Sampling (All Samples)"), hdr.index("Source")
 
     def f(x):
