@@ -86,34 +86,42 @@ __device__ __forceinline__ Chroma chroma(uint32_t uvpair) {
   return {1673527 * v, -852492 * v - 409993 * u, 2116026 * u};
 }
 __device__ __forceinline__ int sat8(int x) { return min(max(x, 0), 255); }
+// RGBx word: R | G << 8 | B << 16 | 0x4B << 24. The top byte is the exponent byte of 2^23,
+// so a channel becomes the float 2^23 + value with one byte permute (see biased()).
 __device__ __forceinline__ uint32_t rgbx(int Y, const Chroma& c) {
   const int yy = max(Y - 16, 0) * 1220542 + (1 << 19);
   return (uint32_t)sat8((yy + c.r) >> 20) | ((uint32_t)sat8((yy + c.g) >> 20) << 8) |
-         ((uint32_t)sat8((yy + c.b) >> 20) << 16);
+         ((uint32_t)sat8((yy + c.b) >> 20) << 16) | 0x4B000000u;
 }
 
-// byte c of an RGBx word as the float 2^23 + byte (exact)
-__device__ __forceinline__ float biased(uint32_t w, int c) {
-  return __int_as_float((int)__byte_perm(w, 0x4B000000u, 0x7540u | (uint32_t)c));
+// byte C of an RGBx word as the float 2^23 + byte (exact): result bytes = [w.C, 0, 0, w.3]
+template <int C>
+__device__ __forceinline__ float biased(uint32_t w) {
+  uint32_t r;
+  asm("prmt.b32 %0, %1, 0, %2;" : "=r"(r) : "r"(w), "n"(0x3440 | C));
+  return __uint_as_float(r);
 }
 
 struct Row3 {
   float2 h[3];   // horizontal lerps of (column a, column b) per channel
 };
 
-__device__ __forceinline__ Row3 hrow(const uint32_t* __restrict__ grow, uint32_t ca, uint32_t cb, float2 lx) {
+template <int C>
+__device__ __forceinline__ float2 hlerp(uint32_t a0, uint32_t a1, uint32_t b0, uint32_t b1, float2 lx) {
+  const float2 P0 = make_float2(biased<C>(a0), biased<C>(b0));
+  const float2 P1 = make_float2(biased<C>(a1), biased<C>(b1));
+  const float2 d = __ffma2_rn(P0, make_float2(-1.f, -1.f), P1);          // p1 - p0 (exact)
+  const float2 p0 = __fadd2_rn(P0, make_float2(-kBias, -kBias));          // p0 (exact)
+  return __ffma2_rn(lx, d, p0);                                           // fmaf(l, p1 - p0, p0)
+}
+
+__device__ __forceinline__ void hrow(Row3& r, const uint32_t* __restrict__ grow, uint32_t ca, uint32_t cb,
+                                     float2 lx) {
   const uint32_t a0 = grow[ca & 0xffffu], a1 = grow[ca >> 16];
   const uint32_t b0 = grow[cb & 0xffffu], b1 = grow[cb >> 16];
-  Row3 r;
-#pragma unroll
-  for (int c = 0; c < 3; ++c) {
-    const float2 P0 = make_float2(biased(a0, c), biased(b0, c));
-    const float2 P1 = make_float2(biased(a1, c), biased(b1, c));
-    const float2 d = __ffma2_rn(P0, make_float2(-1.f, -1.f), P1);          // p1 - p0 (exact)
-    const float2 p0 = __fadd2_rn(P0, make_float2(-kBias, -kBias));          // p0 (exact)
-    r.h[c] = __ffma2_rn(lx, d, p0);                                         // fmaf(l, p1 - p0, p0)
-  }
-  return r;
+  r.h[0] = hlerp<0>(a0, a1, b0, b1, lx);
+  r.h[1] = hlerp<1>(a0, a1, b0, b1, lx);
+  r.h[2] = hlerp<2>(a0, a1, b0, b1, lx);
 }
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
@@ -150,8 +158,10 @@ __device__ __forceinline__ Dest make_dest(const LaunchParams& p, uint32_t dest, 
 }
 
 // store quantised pair q of channel c; DT < 0: dtype read at run time
-template <int DT>
-__device__ __forceinline__ void put(const Dest& d, int dtype, int c, float2 q, bool vec, bool has_b) {
+template <int DT, bool VEC>
+__device__ __forceinline__ void put(const Dest& d, int dtype, int c, float2 q, bool vec_rt, bool has_b) {
+  const bool vec = VEC || vec_rt;
+  // q holds integers 0..255; y = fmaf(q, a_c, b_c) per element (R#17)
   const int dt = DT >= 0 ? DT : dtype;
   uint8_t* o = d.row + (size_t)c * d.cstride;
   if (dt == SAND_BF16) {
@@ -180,12 +190,41 @@ __device__ __forceinline__ void put(const Dest& d, int dtype, int c, float2 q, b
   }
 }
 
-// The row walk (step 3), shared by both modes. grid: RGBx rows of gw words.
+// Vertical lerp + rint + stores of one output row from the horizontal lerps of its two
+// source rows (top = y0, bot = y1): v = fmaf(ly, h1 - h0, h0), q = rint(v) (R#12).
+template <int DT, int ND, bool VEC>
+__device__ __forceinline__ void emit(const Row3& top, const Row3& bot, float l, Dest (&dl)[ND], const int (&dt)[ND],
+                                     const LaunchParams& p, const uint32_t* __restrict__ dests, int nd, int oy,
+                                     int ox, bool vec, bool has_b) {
+  const float2 ly = make_float2(l, l);
+  float2 q[3];
+#pragma unroll
+  for (int c = 0; c < 3; ++c) {
+    const float2 dv = __ffma2_rn(top.h[c], make_float2(-1.f, -1.f), bot.h[c]);   // h1 - h0
+    const float2 v = __ffma2_rn(ly, dv, top.h[c]);                               // fmaf(ly, h1-h0, h0)
+    const float2 tq = __fadd2_rn(v, make_float2(kRound, kRound));                // rint (RNE)
+    q[c] = __fadd2_rn(tq, make_float2(-kRound, -kRound));
+  }
+#pragma unroll
+  for (int d = 0; d < ND; ++d) {
+#pragma unroll
+    for (int c = 0; c < 3; ++c) put<DT, VEC>(dl[d], dt[d], c, q[c], vec, has_b);
+    dl[d].row += dl[d].rstride;
+  }
+  for (int d = ND; d < nd; ++d) {       // rare: more destinations than registers
+    const Dest e = make_dest(p, dests[d], oy, ox);
+    const int et = DT >= 0 ? DT : p.views[dests[d] >> 24].dtype;
+#pragma unroll
+    for (int c = 0; c < 3; ++c) put<DT, VEC>(e, et, c, q[c], vec, has_b);
+  }
+}
+
 // Walk band rows [rr_lo, rr_hi) for the output column pair (ox, ox+1). ND: destinations in
-// registers (1, or 2 plus a loop over the rest). The pair of current source rows (r0c, r1c)
-// and their horizontal lerps (H0, H1) advance monotonically: y1 = min(y0+1, lim-1) is a
-// function of y0, so both change together; a shift by one row reuses H1 as the new H0.
-template <int DT, int ND>
+// registers (1, or 2 plus a loop over the rest). Horizontal lerps of source rows live in two
+// register slots indexed by row parity: y1 = y0 + 1 (or y0 at the clamp), so the two rows an
+// output row needs are always in different slots and each source row's lerp is computed
+// once, with no register copies between rows (the branches on parity are warp-uniform).
+template <int DT, int ND, bool VEC>
 __device__ __forceinline__ void walk_rows(const LaunchParams& p, const uint32_t* __restrict__ dests, int nd,
                                           const uint2* __restrict__ rtab, const uint32_t* __restrict__ grid,
                                           int gw, int oy0, int rr_lo, int rr_hi, int ox, uint32_t ca, uint32_t cb,
@@ -197,46 +236,34 @@ __device__ __forceinline__ void walk_rows(const LaunchParams& p, const uint32_t*
     dl[d] = make_dest(p, dests[d], oy0 + rr_lo, ox);
     dt[d] = DT >= 0 ? DT : p.views[dests[d] >> 24].dtype;
   }
-  int r0c = -1, r1c = -1;
-  Row3 H0, H1;
+  int have0 = -1, have1 = -1;      // source row held in slot 0 (even rows) / slot 1 (odd rows)
+  Row3 S0, S1;
   for (int rr = rr_lo; rr < rr_hi; ++rr) {
     const uint2 rt = rtab[rr];
     const int r0 = (int)(rt.x & 0xffffu), r1 = (int)(rt.x >> 16);
-    if (r0 != r0c) {
-      if (r0 == r1c) H0 = H1;
-      else H0 = hrow(grid + (size_t)r0 * gw, ca, cb, lx);
-      if (r1 == r0) H1 = H0;
-      else H1 = hrow(grid + (size_t)r1 * gw, ca, cb, lx);
-      r0c = r0;
-      r1c = r1;
-    }
     const float l = __uint_as_float(rt.y);
-    const float2 ly = make_float2(l, l);
-    float2 q[3];
-#pragma unroll
-    for (int c = 0; c < 3; ++c) {
-      const float2 dv = __ffma2_rn(H0.h[c], make_float2(-1.f, -1.f), H1.h[c]);   // h1 - h0
-      const float2 v = __ffma2_rn(ly, dv, H0.h[c]);                              // fmaf(ly, h1-h0, h0)
-      const float2 tq = __fadd2_rn(v, make_float2(kRound, kRound));              // rint (RNE)
-      q[c] = __fadd2_rn(tq, make_float2(-kRound, -kRound));
-    }
-#pragma unroll
-    for (int d = 0; d < ND; ++d) {
-#pragma unroll
-      for (int c = 0; c < 3; ++c) put<DT>(dl[d], dt[d], c, q[c], vec, has_b);
-      dl[d].row += dl[d].rstride;
-    }
-    for (int d = ND; d < nd; ++d) {       // rare: more destinations than registers
-      const Dest e = make_dest(p, dests[d], oy0 + rr, ox);
-      const int et = DT >= 0 ? DT : p.views[dests[d] >> 24].dtype;
-#pragma unroll
-      for (int c = 0; c < 3; ++c) put<DT>(e, et, c, q[c], vec, has_b);
+    if (r0 & 1) {
+      if (have1 != r0) { hrow(S1, grid + (size_t)r0 * gw, ca, cb, lx); have1 = r0; }
+      if (r1 != r0) {
+        if (have0 != r1) { hrow(S0, grid + (size_t)r1 * gw, ca, cb, lx); have0 = r1; }
+        emit<DT, ND, VEC>(S1, S0, l, dl, dt, p, dests, nd, oy0 + rr, ox, vec, has_b);
+      } else {
+        emit<DT, ND, VEC>(S1, S1, l, dl, dt, p, dests, nd, oy0 + rr, ox, vec, has_b);
+      }
+    } else {
+      if (have0 != r0) { hrow(S0, grid + (size_t)r0 * gw, ca, cb, lx); have0 = r0; }
+      if (r1 != r0) {
+        if (have1 != r1) { hrow(S1, grid + (size_t)r1 * gw, ca, cb, lx); have1 = r1; }
+        emit<DT, ND, VEC>(S0, S1, l, dl, dt, p, dests, nd, oy0 + rr, ox, vec, has_b);
+      } else {
+        emit<DT, ND, VEC>(S0, S0, l, dl, dt, p, dests, nd, oy0 + rr, ox, vec, has_b);
+      }
     }
   }
 }
 
 // The row walk (step 3), shared by both modes. grid: RGBx rows of gw words.
-template <int DT>
+template <int DT, bool VEC>
 __device__ __forceinline__ void walk(const LaunchParams& p, const WorkItem& w, const GroupParams& g,
                                      const Tables& t, const uint32_t* __restrict__ grid, int gw, int oy_lo,
                                      int nrows) {
@@ -258,9 +285,9 @@ __device__ __forceinline__ void walk(const LaunchParams& p, const WorkItem& w, c
     const uint2 ta = t.ctab[ja], tb = t.ctab[jb];
     const float2 lx = make_float2(__uint_as_float(ta.y), __uint_as_float(tb.y));
     if (nd == 1)
-      walk_rows<DT, 1>(p, dests, nd, rtab, grid, gw, oy_lo, rr_lo, rr_hi, ox, ta.x, tb.x, lx, vec, has_b);
+      walk_rows<DT, 1, VEC>(p, dests, nd, rtab, grid, gw, oy_lo, rr_lo, rr_hi, ox, ta.x, tb.x, lx, vec, has_b);
     else
-      walk_rows<DT, kInlineDests>(p, dests, nd, rtab, grid, gw, oy_lo, rr_lo, rr_hi, ox, ta.x, tb.x, lx, vec,
+      walk_rows<DT, kInlineDests, VEC>(p, dests, nd, rtab, grid, gw, oy_lo, rr_lo, rr_hi, ox, ta.x, tb.x, lx, vec,
                                   has_b);
   }
 }
@@ -268,8 +295,8 @@ __device__ __forceinline__ void walk(const LaunchParams& p, const WorkItem& w, c
 }  // namespace rs
 
 // RAW mode: p launch params; R band rows; nbands; maxWo table sizing.
-template <int DT>
-__global__ void __launch_bounds__(224, 4) k_resample_raw(const LaunchParams p, int R, int nbands, int maxWo) {
+template <int DT, bool VEC>
+__global__ void __launch_bounds__(224, 3) k_resample_raw(const LaunchParams p, int R, int nbands, int maxWo) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   using namespace rs;
   const int item_idx = blockIdx.x / nbands;
@@ -365,12 +392,12 @@ __global__ void __launch_bounds__(224, 4) k_resample_raw(const LaunchParams p, i
   __syncthreads();
 
   // 4. row walk
-  walk<DT>(p, w, g, t, grid, gw, oy_lo, nrows);
+  walk<DT, VEC>(p, w, g, t, grid, gw, oy_lo, nrows);
 }
 
 // GATHER mode (heavy down-scaling): compact tap grid gathered from HBM.
-template <int DT>
-__global__ void __launch_bounds__(224, 4) k_resample_gather(const LaunchParams p, int R, int nbands, int maxWo) {
+template <int DT, bool VEC>
+__global__ void __launch_bounds__(224, 3) k_resample_gather(const LaunchParams p, int R, int nbands, int maxWo) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   using namespace rs;
   const int item_idx = blockIdx.x / nbands;
@@ -510,7 +537,7 @@ __global__ void __launch_bounds__(224, 4) k_resample_gather(const LaunchParams p
     }
   }
   __syncthreads();
-  walk<DT>(p, w, g, t, grid, nX, oy_lo, nrows);
+  walk<DT, VEC>(p, w, g, t, grid, nX, oy_lo, nrows);
 }
 
 }  // namespace sand

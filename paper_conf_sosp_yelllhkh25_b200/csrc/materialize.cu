@@ -210,7 +210,7 @@ ResampleCfg choose_resample(const BatchShape& sh) {
   return {false, 1, 0};
 }
 
-template <int DT>
+template <int DT, bool VEC>
 int launch_resample_dt(const LaunchParams& p, const BatchShape& sh, cudaStream_t stream) {
   const ResampleCfg cfg = choose_resample(sh);
   if (cfg.smem > 227 * 1024) return set_error(SAND_EINVAL, "resample tile exceeds shared memory (source crop too large)");
@@ -219,9 +219,9 @@ int launch_resample_dt(const LaunchParams& p, const BatchShape& sh, cudaStream_t
   const int threads = std::min(224, ((2 * pairs + 31) / 32) * 32);
   const unsigned blocks = (unsigned)((uint64_t)p.n_items * nbands);
   if (cfg.raw)
-    k_resample_raw<DT><<<blocks, threads, cfg.smem, stream>>>(p, cfg.R, nbands, sh.max_wo);
+    k_resample_raw<DT, VEC><<<blocks, threads, cfg.smem, stream>>>(p, cfg.R, nbands, sh.max_wo);
   else
-    k_resample_gather<DT><<<blocks, threads, cfg.smem, stream>>>(p, cfg.R, nbands, sh.max_wo);
+    k_resample_gather<DT, VEC><<<blocks, threads, cfg.smem, stream>>>(p, cfg.R, nbands, sh.max_wo);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_error(e, "k_resample launch");
   return SAND_OK;
@@ -243,10 +243,10 @@ size_t stencil_smem_bytes(int max_h, int max_w, int max_r) {
 int configure_kernels(size_t stencil_smem) {
   {
     cudaError_t e = cudaSuccess;
-    for (cudaError_t r : {allow_smem(k_resample_raw<-1>), allow_smem(k_resample_raw<SAND_U8>),
-                          allow_smem(k_resample_raw<SAND_BF16>), allow_smem(k_resample_raw<SAND_F32>),
-                          allow_smem(k_resample_gather<-1>), allow_smem(k_resample_gather<SAND_U8>),
-                          allow_smem(k_resample_gather<SAND_BF16>), allow_smem(k_resample_gather<SAND_F32>)})
+    for (cudaError_t r : {allow_smem(k_resample_raw<-1, false>), allow_smem(k_resample_raw<SAND_U8, true>),
+                          allow_smem(k_resample_raw<SAND_BF16, true>), allow_smem(k_resample_raw<SAND_F32, true>),
+                          allow_smem(k_resample_gather<-1, false>), allow_smem(k_resample_gather<SAND_U8, true>),
+                          allow_smem(k_resample_gather<SAND_BF16, true>), allow_smem(k_resample_gather<SAND_F32, true>)})
       if (r != cudaSuccess) e = r;
     if (e != cudaSuccess) return cuda_error(e, "cudaFuncSetAttribute(k_resample)");
   }
@@ -264,11 +264,13 @@ int launch_materialize(const LaunchParams& p, const BatchShape& shape, size_t st
   if (p.n_items == 0) return SAND_OK;
   if (shape.has_direct) {
     int rc;
-    switch (shape.dtype) {
-      case SAND_U8: rc = launch_resample_dt<SAND_U8>(p, shape, stream); break;
-      case SAND_BF16: rc = launch_resample_dt<SAND_BF16>(p, shape, stream); break;
-      case SAND_F32: rc = launch_resample_dt<SAND_F32>(p, shape, stream); break;
-      default: rc = launch_resample_dt<-1>(p, shape, stream); break;
+    // specialised instantiations: one dtype for every view and even output widths (the
+    // 4-byte pair stores are aligned); anything else takes the generic instantiation
+    switch (shape.even_wo ? shape.dtype : -1) {
+      case SAND_U8: rc = launch_resample_dt<SAND_U8, true>(p, shape, stream); break;
+      case SAND_BF16: rc = launch_resample_dt<SAND_BF16, true>(p, shape, stream); break;
+      case SAND_F32: rc = launch_resample_dt<SAND_F32, true>(p, shape, stream); break;
+      default: rc = launch_resample_dt<-1, false>(p, shape, stream); break;
     }
     if (rc != SAND_OK) return rc;
     ++*n_launched;

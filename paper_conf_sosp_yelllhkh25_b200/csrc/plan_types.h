@@ -67,6 +67,7 @@ struct BatchShape {
   int32_t cols_bound;     // upper bound of distinct tapped source columns of any item
   float max_scy;          // largest vertical source step (rows per output row)
   int32_t dtype;          // output dtype shared by every view, or -1 if mixed
+  int32_t even_wo;        // every view's out_w is even
 };
 
 struct LaunchParams {

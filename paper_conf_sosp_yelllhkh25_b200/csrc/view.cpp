@@ -91,11 +91,15 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
   plan->item_begin.push_back(0);
   plan->fetch_begin.push_back(0);
   int32_t common_dtype = s.views[0].out_dtype;
-  for (uint32_t k = 1; k < s.n_views; ++k)
+  int32_t even_wo = 1;
+  for (uint32_t k = 0; k < s.n_views; ++k) {
     if (s.views[k].out_dtype != common_dtype) common_dtype = -1;
+    if (s.views[k].out_w & 1u) even_wo = 0;
+  }
   for (uint64_t it = 0; it < plan->iterations; ++it) {
     BatchShape shape{};
     shape.dtype = common_dtype;
+    shape.even_wo = even_wo;
     std::vector<std::pair<uint64_t, uint32_t>> fetch;   // ((video<<32)|frame, uses)
     for (uint32_t b = 0; b < B; ++b) {
       const uint64_t slot = it * B + b;
@@ -388,6 +392,15 @@ extern "C" int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank,
   }
   const uint64_t it = out->iteration;
   const uint32_t ib = plan->item_begin[it], ie = plan->item_begin[it + 1];
+  // plan the next epoch on the worker while this one is consumed (pre-materialisation of the
+  // plan, the analogue of the paper's pre-materialisation threads)
+  if (it == 0) {
+    const auto next = std::make_pair(epoch + 1, rank);
+    if (!v->plans.count(next) && !v->pending.count(next)) {
+      v->queue.push_back(next);
+      v->cv.notify_all();
+    }
+  }
   sand_store* st = v->store;
   {
     std::lock_guard<std::mutex> slk(st->mu);
