@@ -255,9 +255,8 @@ def run_sand(args):
     def step_id(s):
         return s // iters, s % iters
 
-    # plan ahead (pre-materialisation of plans)
-    for e in range(0, (args.warmup + args.steps) // iters + 2):
-        view.prefetch_epoch(e, rank)
+    # the library plans epoch e+1 on its worker when epoch e's first batch is read
+    view.prefetch_epoch(0, rank)
 
     s = 0
     for _ in range(args.warmup):
