@@ -207,9 +207,11 @@ __device__ __forceinline__ void emit(const Row3& top, const Row3& bot, float l, 
   }
 #pragma unroll
   for (int d = 0; d < ND; ++d) {
+    if (d == 0 || d < nd) {
 #pragma unroll
-    for (int c = 0; c < 3; ++c) put<DT, VEC>(dl[d], dt[d], c, q[c], vec, has_b);
-    dl[d].row += dl[d].rstride;
+      for (int c = 0; c < 3; ++c) put<DT, VEC>(dl[d], dt[d], c, q[c], vec, has_b);
+      dl[d].row += dl[d].rstride;
+    }
   }
   for (int d = ND; d < nd; ++d) {       // rare: more destinations than registers
     const Dest e = make_dest(p, dests[d], oy, ox);

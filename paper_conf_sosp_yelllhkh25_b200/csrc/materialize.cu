@@ -169,6 +169,7 @@ __global__ void __launch_bounds__(512) k_stencil(const LaunchParams p) {
 }  // namespace sand
 
 #include "k_resample.cuh"
+#include "k_stream.cuh"
 
 namespace sand {
 
@@ -183,21 +184,39 @@ size_t smem_budget() {
 }
 
 struct ResampleCfg {
-  bool raw;
+  int mode;         // 0 gather, 1 raw bands, 2 stream
   int R;
   size_t smem;
+  st::Shape st;
 };
+
+int env_int(const char* name, int dflt) {
+  const char* e = getenv(name);
+  return e ? atoi(e) : dflt;
+}
 
 // mode, band height and dynamic shared memory of the resample kernel for a batch shape
 ResampleCfg choose_resample(const BatchShape& sh) {
   static const int kCands[] = {64, 48, 32, 24, 16, 12, 8, 4, 2, 1};
   const bool mild = sh.cols_bound <= 2 * sh.max_wo + 16 && sh.max_scy <= 2.0f;
   const size_t gwb = rs::a16((size_t)sh.cols_bound) + 16;
-  if (mild) {
+  static const int forced = env_int("SAND_RESAMPLE_MODE", -1);
+  if (mild && sh.max_wo <= 512 && forced != 1 && forced != 0) {
+    st::Shape s;
+    s.S = env_int("SAND_STREAM_S", 8);
+    s.SB = env_int("SAND_STREAM_SB", 56);
+    s.nsb = (sh.max_ho + s.SB - 1) / s.SB;
+    s.ring = (int)std::ceil((double)sh.max_scy * s.S) + 3;
+    s.raw_rows = s.ring + s.ring / 2 + 2;
+    s.gw = (int)gwb;
+    ResampleCfg c{2, 0, st::smem_bytes(s, sh.max_wo), s};
+    if (s.ring <= 255 && c.smem <= 200 * 1024) return c;
+  }
+  if (mild && forced != 0) {
     for (int r : kCands) {
       const size_t rows = (size_t)std::ceil((double)sh.max_scy * r) + 3;
       const size_t bytes = rs::tables_bytes(sh.max_wo, r) + rows * gwb + rs::a16((rows / 2 + 2) * gwb) + rows * gwb * 4;
-      if (bytes <= smem_budget() || (r <= 8 && bytes <= 200 * 1024)) return {true, r, bytes};
+      if (bytes <= smem_budget() || (r <= 8 && bytes <= 200 * 1024)) return {1, r, bytes, {}};
     }
   }
   for (int r : kCands) {
@@ -205,20 +224,28 @@ ResampleCfg choose_resample(const BatchShape& sh) {
     const size_t rows = (size_t)std::min(2 * r, span);
     const size_t cols = (size_t)std::min(2 * sh.max_wo, sh.cols_bound);
     const size_t bytes = rs::tables_bytes(sh.max_wo, r) + rs::gather_meta_bytes(sh.max_wo, r) + rows * cols * 4;
-    if ((bytes <= smem_budget() && span <= 32 * rs::kRowWords) || r == 1) return {false, r, bytes};
+    if ((bytes <= smem_budget() && span <= 32 * rs::kRowWords) || r == 1) return {0, r, bytes, {}};
   }
-  return {false, 1, 0};
+  return {0, 1, 0, {}};
 }
 
 template <int DT, bool VEC>
 int launch_resample_dt(const LaunchParams& p, const BatchShape& sh, cudaStream_t stream) {
   const ResampleCfg cfg = choose_resample(sh);
   if (cfg.smem > 227 * 1024) return set_error(SAND_EINVAL, "resample tile exceeds shared memory (source crop too large)");
-  const int nbands = (sh.max_ho + cfg.R - 1) / cfg.R;
   const int pairs = (sh.max_wo + 1) / 2;
+  if (cfg.mode == 2) {
+    const int threads = ((pairs + 31) / 32) * 32;
+    const unsigned blocks = (unsigned)((uint64_t)p.n_items * cfg.st.nsb);
+    k_stream<DT, VEC><<<blocks, threads, cfg.smem, stream>>>(p, cfg.st, sh.max_wo);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_error(e, "k_stream launch");
+    return SAND_OK;
+  }
+  const int nbands = (sh.max_ho + cfg.R - 1) / cfg.R;
   const int threads = std::min(224, ((2 * pairs + 31) / 32) * 32);
   const unsigned blocks = (unsigned)((uint64_t)p.n_items * nbands);
-  if (cfg.raw)
+  if (cfg.mode == 1)
     k_resample_raw<DT, VEC><<<blocks, threads, cfg.smem, stream>>>(p, cfg.R, nbands, sh.max_wo);
   else
     k_resample_gather<DT, VEC><<<blocks, threads, cfg.smem, stream>>>(p, cfg.R, nbands, sh.max_wo);
@@ -246,7 +273,9 @@ int configure_kernels(size_t stencil_smem) {
     for (cudaError_t r : {allow_smem(k_resample_raw<-1, false>), allow_smem(k_resample_raw<SAND_U8, true>),
                           allow_smem(k_resample_raw<SAND_BF16, true>), allow_smem(k_resample_raw<SAND_F32, true>),
                           allow_smem(k_resample_gather<-1, false>), allow_smem(k_resample_gather<SAND_U8, true>),
-                          allow_smem(k_resample_gather<SAND_BF16, true>), allow_smem(k_resample_gather<SAND_F32, true>)})
+                          allow_smem(k_resample_gather<SAND_BF16, true>), allow_smem(k_resample_gather<SAND_F32, true>),
+                          allow_smem(k_stream<-1, false>), allow_smem(k_stream<SAND_U8, true>),
+                          allow_smem(k_stream<SAND_BF16, true>), allow_smem(k_stream<SAND_F32, true>)})
       if (r != cudaSuccess) e = r;
     if (e != cudaSuccess) return cuda_error(e, "cudaFuncSetAttribute(k_resample)");
   }

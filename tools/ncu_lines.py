@@ -1,7 +1,7 @@
 #!/usr/bin/env python
 """Aggregate an ncu SASS source page by CUDA source line.
 
-    python tools/ncu_lines.py <report.ncu-rep> <object.o|.cubin> <kernel-substring> [top]
+    python tools/ncu_lines.py <report.ncu-rep> <object.o|.cubin> <ncu-name-substring> [top] [raw:<mangled-substring>]
 
 Runs `ncu -i --page source --print-source sass --csv` and `nvdisasm -g` on the cubin of the
 same build, matches instructions by order, and prints instructions executed and warp-stall
@@ -18,15 +18,25 @@ import tempfile
 
 
 def mangled_match(kernel, line):
+    if kernel.startswith("raw:"):
+        return kernel[4:] in line
     """kernel like 'k_resample_raw<1>' matches the mangled '14k_resample_rawILi1EE...'."""
-    m = re.match(r"(\w+)(?:<(-?\d+)>)?", kernel)
-    name, targ = m.group(1), m.group(2)
+    m = re.match(r"(\w+)(?:<([^>]*)>)?", kernel)
+    name, targs = m.group(1), m.group(2)
     if name not in line:
         return False
-    if targ is None:
+    if targs is None:
         return True
-    t = ("Lin" + targ[1:]) if targ.startswith("-") else ("Li" + targ)
-    return f"{name}I{t}E" in line
+    enc = ""
+    for a in targs.split(","):
+        a = a.strip()
+        if a in ("true", "false"):
+            enc += "Lb" + ("1" if a == "true" else "0") + "E"
+        elif a.startswith("-"):
+            enc += "Lin" + a[1:] + "E"
+        else:
+            enc += "Li" + a + "E"
+    return f"{name}I{enc}" in line
 
 
 def sass_lines(obj, kernel):
@@ -61,6 +71,7 @@ def sass_lines(obj, kernel):
 def main():
     rep, obj, kernel = sys.argv[1:4]
     top = int(sys.argv[4]) if len(sys.argv) > 4 else 40
+    mangled = sys.argv[5] if len(sys.argv) > 5 else kernel
     csvtxt = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
                             capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(csvtxt)))
@@ -74,7 +85,7 @@ def main():
             hdr = r
         elif cur is not None and hdr and len(r) >= len(hdr) - 1:
             cur["rows"].append(r)
-    blk = next(b for b in blocks if kernel in b["name"].replace(" ", "").replace("(int)", ""))
+    blk = next(b for b in blocks if kernel in b["name"].replace(" ", "").replace("(int)", "").replace("(bool)", "").replace("true", "1").replace("false", "0"))
     ie, st, src = hdr.index("Instructions Executed"), hdr.index("Warp Stall Sampling (All Samples)"), hdr.index("Source")
 
     def f(x):
@@ -83,7 +94,7 @@ def main():
         except ValueError:
             return 0.0
 
-    lines = sass_lines(obj, kernel)
+    lines = sass_lines(obj, mangled)
     n = min(len(lines), len(blk["rows"]))
     if len(lines) != len(blk["rows"]):
         print(f"warning: {len(lines)} disassembled vs {len(blk['rows'])} profiled instructions", file=sys.stderr)
