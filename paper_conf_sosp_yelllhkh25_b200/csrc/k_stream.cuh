@@ -5,15 +5,17 @@
 // rows, processed as sub-bands of S rows:
 //   * the NV12 rows a sub-band adds are copied HBM -> shared memory with cp.async one
 //     sub-band ahead (double-buffered raw staging, all 16 B requests in flight; a4);
-//   * they are converted once to RGBx words in a shared-memory ring of source rows, a
-//     thread taking one chroma sample's 2x(4) luma pixels (a5, Q1);
+//   * they are converted once to RGBx words in a shared-memory ring of source rows; a
+//     thread takes one UV word (two chroma samples) and the 2x4 luma pixels sharing it,
+//     with the clamp folded into DPX add-max (VIADDMNMX) and bytes packed by PRMT (a5, Q1);
 //   * each thread owns an output column pair for the whole super-band and keeps the
 //     horizontal lerps of the current two source rows in registers across sub-bands (a6),
 //     mirrored for flip (a7); vertical lerp, rint, normalise and the 4-byte stores to every
 //     destination view follow (a10, a11).
-// Per-CTA setup (tap tables, destination pointers) is amortised over SB rows and no source
-// row is converted twice inside a super-band. Arithmetic is the R#12/R#17 op sequence with
-// IEEE rounding at each step: bit-identical to the oracle.
+// Shared memory is addressed with 32-bit shared-window addresses (ld/st.shared) so the hot
+// loops carry no generic-address arithmetic. Per-CTA setup is amortised over SB rows and
+// no source row is converted twice inside a super-band. Arithmetic is the R#11/R#12/R#17
+// op sequence with IEEE rounding at each step: bit-identical to the oracle.
 #pragma once
 
 namespace sand {
@@ -25,55 +27,112 @@ struct Shape {      // host-chosen launch shape
   int SB;           // output rows per CTA
   int nsb;          // super-bands per item (ceil(maxHo / SB))
   int S;            // output rows per sub-band
-  int ring;         // ring capacity in source rows (<= 255)
+  int ring;         // ring capacity in source rows
   int raw_rows;     // raw staging capacity in rows (Y + UV) per buffer
   int gw;           // max row width in bytes of Y (= words of RGBx), multiple of 16
 };
 
 __host__ __device__ inline size_t smem_bytes(const Shape& s, int maxWo) {
-  return a16((size_t)maxWo * 8) + a16((size_t)s.SB * 8) + (size_t)s.ring * s.gw * 4 +
+  return a16((size_t)maxWo * 8) + a16((size_t)s.SB * 16) + (size_t)s.ring * s.gw * 4 +
          2 * a16((size_t)s.raw_rows * s.gw);
 }
 
-__device__ __forceinline__ void stage_rows(uint8_t* raw, const uint8_t* Yp, const uint8_t* UVp, uint32_t pitch,
+__device__ __forceinline__ uint32_t lds32(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ uint4 lds128(uint32_t a) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ void sts128(uint32_t a, uint4 v) {
+  asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async16s(uint32_t s, const void* gmem) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
+}
+
+// Y rows [ya, yb] then UV rows [ya>>1, yb>>1] -> raw (shared address), gw bytes from column x16
+__device__ __forceinline__ void stage_rows(uint32_t raw, const uint8_t* Yp, const uint8_t* UVp, uint32_t pitch,
                                            int x16, int gw, int ya, int yb, int tid, int nthr) {
-  // Y rows [ya, yb] then UV rows [ya>>1, yb>>1], each gw bytes from column x16
   const int ny = yb - ya + 1, u0 = ya >> 1, nuv = (yb >> 1) - u0 + 1;
   const int chunks = gw >> 4, total = (ny + nuv) * chunks;
   for (int e = tid; e < total; e += nthr) {
-    const int r = e / chunks, k = e - r * chunks;    // once per 16 B request, off the hot loop
+    const int r = e / chunks, k = e - r * chunks;    // once per 16 B request
     const uint8_t* src = r < ny ? Yp + (size_t)(ya + r) * pitch : UVp + (size_t)(u0 + r - ny) * pitch;
-    rs::cp_async16(raw + (size_t)r * gw + k * 16, src + x16 + k * 16);
+    cp_async16s(raw + (uint32_t)(r * gw + k * 16), src + x16 + k * 16);
   }
   asm volatile("cp.async.commit_group;\n" ::: "memory");
 }
 
-// convert staged rows [ya, yb] into ring slots (y - y_first) % ring
-__device__ __forceinline__ void convert_rows(uint32_t* ring, const uint8_t* raw, int gw, int ya, int yb, int y_first,
-                                             int ring_rows, int tid, int nthr) {
-  const int ny = yb - ya + 1, u0 = ya >> 1, nuv = (yb >> 1) - u0 + 1;
-  const uint8_t* rawUV = raw + (size_t)ny * gw;
-  const int q4 = gw >> 2;                       // 4-pixel groups per row
-  for (int e = tid; e < nuv * q4; e += nthr) {
-    const int u = e / q4, q = e - u * q4;
-    const uint32_t uv = *reinterpret_cast<const uint32_t*>(rawUV + (size_t)u * gw + 4 * q);
-    const rs::Chroma c0 = rs::chroma(uv & 0xffffu), c1 = rs::chroma(uv >> 16);
+// chroma terms (R#11) of the sample whose U is at bit SHIFT of the UV word
+struct Chroma3 {
+  int r, g, b;
+};
+template <int SHIFT>
+__device__ __forceinline__ Chroma3 chroma_at(uint32_t uv) {
+  const int u = (int)((uv >> SHIFT) & 0xffu) - 128;
+  const int v = (int)((uv >> (SHIFT + 8)) & 0xffu) - 128;
+  return {1673527 * v, -852492 * v - 409993 * u, 2116026 * u};
+}
+
+// RGBx word of luma Y with chroma c: sat((yy + term) >> 20) per channel (OpenCV integer
+// BT.601), computed as min(max(yy + term, 0), 2^28 - 1) >> 4, whose byte 2 is the channel;
+// PRMT gathers the three bytes and the exponent byte 0x4B tops the word (see rs::biased).
+__device__ __forceinline__ uint32_t rgbx_dpx(uint32_t Y, const Chroma3& c) {
+  const int yy = (int)max(Y, 16u) * 1220542 + ((1 << 19) - 16 * 1220542);
+  const int mr = min(__viaddmax_s32(yy, c.r, 0), 0x0FFFFFFF) >> 4;
+  const int mg = min(__viaddmax_s32(yy, c.g, 0), 0x0FFFFFFF) >> 4;
+  const int mb = min(__viaddmax_s32(yy, c.b, 0), 0x0FFFFFFF) >> 4;
+  const uint32_t rg = __byte_perm((uint32_t)mr, (uint32_t)mg, 0x0062);
+  return __byte_perm(rg, (uint32_t)mb, 0x7610) | 0x4B000000u;
+}
+
+// convert staged rows [ya, yb] into the ring (slot = (y - y_first) % ring_rows)
+__device__ __forceinline__ void convert_rows(uint32_t ring, uint32_t raw, int gw, int ya, int yb, int y_first,
+                                             int ring_rows, int warp, int nwarps, int lane) {
+  const int ny = yb - ya + 1;
+  if (ny <= 0) return;
+  const int u0 = ya >> 1, nuv = (yb >> 1) - u0 + 1;
+  const uint32_t rawUV = raw + (uint32_t)(ny * gw);
+  const int q4 = gw >> 2;                      // 4-pixel groups per row
+  const uint32_t rowbytes = (uint32_t)gw * 4u;
+  for (int u = warp; u < nuv; u += nwarps) {
     const int yt = 2 * (u0 + u);
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      const int y = yt + h;
-      if (y < ya || y > yb) continue;
-      const uint32_t yw = *reinterpret_cast<const uint32_t*>(raw + (size_t)(y - ya) * gw + 4 * q);
-      int slot = y - y_first;
-      slot = slot >= ring_rows ? slot % ring_rows : slot;
-      uint4 o;
-      o.x = rs::rgbx((int)(yw & 0xffu), c0);
-      o.y = rs::rgbx((int)((yw >> 8) & 0xffu), c0);
-      o.z = rs::rgbx((int)((yw >> 16) & 0xffu), c1);
-      o.w = rs::rgbx((int)(yw >> 24), c1);
-      *reinterpret_cast<uint4*>(ring + (size_t)slot * gw + 4 * q) = o;
+    const bool top = yt >= ya, bot = yt + 1 <= yb;
+    const int st = (yt - y_first + ring_rows) % ring_rows;   // yt may be y_first - 1
+    const int sb = st + 1 == ring_rows ? 0 : st + 1;
+    const uint32_t yrow_t = raw + (uint32_t)((yt - ya) * gw), yrow_b = raw + (uint32_t)((yt + 1 - ya) * gw);
+    const uint32_t out_t = ring + (uint32_t)st * rowbytes, out_b = ring + (uint32_t)sb * rowbytes;
+    const uint32_t uvrow = rawUV + (uint32_t)(u * gw);
+    for (int q = lane; q < q4; q += 32) {
+      const uint32_t uv = lds32(uvrow + 4 * q);
+      const Chroma3 c0 = chroma_at<0>(uv), c1 = chroma_at<16>(uv);
+      if (top) {
+        const uint32_t yw = lds32(yrow_t + 4 * q);
+        sts128(out_t + 16 * q, make_uint4(rgbx_dpx(yw & 0xffu, c0), rgbx_dpx((yw >> 8) & 0xffu, c0),
+                                          rgbx_dpx((yw >> 16) & 0xffu, c1), rgbx_dpx(yw >> 24, c1)));
+      }
+      if (bot) {
+        const uint32_t yw = lds32(yrow_b + 4 * q);
+        sts128(out_b + 16 * q, make_uint4(rgbx_dpx(yw & 0xffu, c0), rgbx_dpx((yw >> 8) & 0xffu, c0),
+                                          rgbx_dpx((yw >> 16) & 0xffu, c1), rgbx_dpx(yw >> 24, c1)));
+      }
     }
   }
+}
+
+// horizontal lerps of one ring row for the thread's column pair (R#12); col*: byte offsets
+__device__ __forceinline__ void hrow_s(rs::Row3& r, uint32_t rowaddr, uint32_t ca0, uint32_t ca1, uint32_t cb0,
+                                       uint32_t cb1, float2 lx) {
+  const uint32_t a0 = lds32(rowaddr + ca0), a1 = lds32(rowaddr + ca1);
+  const uint32_t b0 = lds32(rowaddr + cb0), b1 = lds32(rowaddr + cb1);
+  r.h[0] = rs::hlerp<0>(a0, a1, b0, b1, lx);
+  r.h[1] = rs::hlerp<1>(a0, a1, b0, b1, lx);
+  r.h[2] = rs::hlerp<2>(a0, a1, b0, b1, lx);
 }
 
 }  // namespace st
@@ -92,13 +151,15 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
   if (Y0 >= Ho) return;
   const int nr = min(sh.SB, Ho - Y0);
   const int tid = threadIdx.x, nthr = blockDim.x;
+  const int warp = tid >> 5, lane = tid & 31, nwarps = nthr >> 5;
 
-  uint8_t* sp = smem_raw;
-  uint2* ctab = reinterpret_cast<uint2*>(sp); sp += a16((size_t)maxWo * 8);
-  uint2* rtab = reinterpret_cast<uint2*>(sp); sp += a16((size_t)sh.SB * 8);
-  uint32_t* ring = reinterpret_cast<uint32_t*>(sp); sp += (size_t)sh.ring * sh.gw * 4;
-  const size_t rawcap = a16((size_t)sh.raw_rows * sh.gw);
-  uint8_t* const rawbase = sp;   // two raw staging buffers of rawcap bytes
+  uint2* ctab = reinterpret_cast<uint2*>(smem_raw);
+  uint4* rtab = reinterpret_cast<uint4*>(smem_raw + a16((size_t)maxWo * 8));
+  const uint32_t s_base = (uint32_t)__cvta_generic_to_shared(smem_raw);
+  const uint32_t s_rtab = s_base + (uint32_t)a16((size_t)maxWo * 8);
+  const uint32_t s_ring = s_rtab + (uint32_t)a16((size_t)sh.SB * 16);
+  const uint32_t s_raw = s_ring + (uint32_t)(sh.ring * sh.gw * 4);
+  const uint32_t rawcap = (uint32_t)a16((size_t)sh.raw_rows * sh.gw);
 
   // footprint of the super-band (monotone taps)
   const int x_lo = tap0(g.sc_x, g.off_x, 0, g.org_x);
@@ -107,12 +168,13 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
   tap(g.sc_x, g.off_x, Wo - 1, g.lim_x, g.org_x, dmy, x_hi, fl);
   const int x16 = x_lo & ~15;
   const int gw = ((x_hi + 16) & ~15) - x16;
+  const uint32_t rowbytes = (uint32_t)gw * 4u;
   const int y_first = tap0(g.sc_y, g.off_y, Y0, g.org_y);
   const uint8_t* Yp = p.slab + w.y_off;
   const uint8_t* UVp = Yp + (size_t)w.pitch * w.src_h;
 
-  // sub-band k covers output rows [k*S, min((k+1)*S, nr)); its new source rows are
-  // (last row of sub-band k-1, y1(last row of k)]
+  // sub-band k covers output rows [k*S, min((k+1)*S, nr)); it adds source rows
+  // (y1(last row of k-1), y1(last row of k)]
   auto last_src = [&](int k) {
     int a, b;
     float l;
@@ -121,9 +183,10 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
   };
   const int nsub = (nr + sh.S - 1) / sh.S;
   int ya = y_first, yb = last_src(0);
-  st::stage_rows(rawbase, Yp, UVp, w.pitch, x16, gw, ya, yb, tid, nthr);
+  st::stage_rows(s_raw, Yp, UVp, w.pitch, x16, gw, ya, yb, tid, nthr);
 
-  // tap tables (overlap the first copy)
+  // tap tables (overlap the first copy): columns (x0, x1, lambda); rows (byte offsets of
+  // the two ring rows, y0, lambda)
   for (int j = tid; j < Wo; j += nthr) {
     int x0, x1;
     float lx;
@@ -135,16 +198,16 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
     float ly;
     tap(g.sc_y, g.off_y, Y0 + r, g.lim_y, g.org_y, y0, y1, ly);
     const uint32_t s0 = (uint32_t)((y0 - y_first) % sh.ring), s1 = (uint32_t)((y1 - y_first) % sh.ring);
-    rtab[r] = make_uint2(s0 | (s1 << 8) | ((uint32_t)y0 << 16), __float_as_uint(ly));
+    rtab[r] = make_uint4(s0 * rowbytes, s1 * rowbytes, (uint32_t)y0, __float_as_uint(ly));
   }
 
-  // per-thread walker state: output column pair `pair`, kept for the whole super-band
+  // per-thread walker state: output columns (ox, ox+1) for the whole super-band
   const int pairs = (Wo + 1) >> 1;
   const bool walker = tid < pairs;
   const int ox = 2 * tid;
   const bool has_b = ox + 1 < Wo;
   const bool vec = has_b && !(Wo & 1);
-  uint32_t ca = 0, cb = 0;
+  uint32_t ca0 = 0, ca1 = 0, cb0 = 0, cb1 = 0;
   float2 lx = make_float2(0.f, 0.f);
   const int nd = (int)w.n_dest;
   const uint32_t* dests = p.dests + w.dest_begin;
@@ -156,20 +219,24 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
   for (int k = 0; k < nsub; ++k) {
     asm volatile("cp.async.wait_group 0;\n" ::: "memory");
     __syncthreads();                                 // raw[k&1] landed; walk(k-1) finished
-    st::convert_rows(ring, rawbase + (size_t)(k & 1) * rawcap, gw, ya, yb, y_first, sh.ring, tid, nthr);
+    st::convert_rows(s_ring, s_raw + (uint32_t)(k & 1) * rawcap, gw, ya, yb, y_first, sh.ring, warp, nwarps, lane);
     if (k + 1 < nsub) {                              // stage the next sub-band's new rows
       const int na = yb + 1, nb = last_src(k + 1);
-      if (nb >= na) st::stage_rows(rawbase + (size_t)((k + 1) & 1) * rawcap, Yp, UVp, w.pitch, x16, gw, na, nb, tid, nthr);
+      if (nb >= na)
+        st::stage_rows(s_raw + (uint32_t)((k + 1) & 1) * rawcap, Yp, UVp, w.pitch, x16, gw, na, nb, tid, nthr);
       ya = na;
       yb = max(nb, yb);
     }
     __syncthreads();                                 // ring holds every row of sub-band k
-    if (k == 0 && walker) {                          // tables are visible now
+    if (!walker) continue;
+    if (k == 0) {                                    // tables are visible now
       const int ja = g.flip ? Wo - 1 - ox : ox;
       const int jb = has_b ? (g.flip ? Wo - 2 - ox : ox + 1) : ja;
       const uint2 ta = ctab[ja], tb = ctab[jb];
-      ca = ta.x;
-      cb = tb.x;
+      ca0 = 4u * (ta.x & 0xffffu);
+      ca1 = 4u * (ta.x >> 16);
+      cb0 = 4u * (tb.x & 0xffffu);
+      cb1 = 4u * (tb.x >> 16);
       lx = make_float2(__uint_as_float(ta.y), __uint_as_float(tb.y));
 #pragma unroll
       for (int d = 0; d < kInlineDests; ++d)
@@ -178,30 +245,29 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
           dt[d] = DT >= 0 ? DT : p.views[dests[d] >> 24].dtype;
         }
     }
-    if (walker) {
-      const int r_lo = k * sh.S, r_hi = min(r_lo + sh.S, nr);
-      for (int rr = r_lo; rr < r_hi; ++rr) {
-        const uint2 rt = rtab[rr];
-        const int s0 = (int)(rt.x & 0xffu), s1 = (int)((rt.x >> 8) & 0xffu), y0 = (int)(rt.x >> 16);
-        const float l = __uint_as_float(rt.y);
-        const int oy = Y0 + rr;
-        // parity slots: rows y0 and y0+1 are held in different registers sets (R#12 taps)
-        if (y0 & 1) {
-          if (have1 != y0) { hrow(S1, ring + (size_t)s0 * gw, ca, cb, lx); have1 = y0; }
-          if (s1 != s0) {
-            if (have0 != y0 + 1) { hrow(S0, ring + (size_t)s1 * gw, ca, cb, lx); have0 = y0 + 1; }
-            emit<DT, kInlineDests, VEC>(S1, S0, l, dl, dt, p, dests, nd, oy, ox, vec, has_b);
-          } else {
-            emit<DT, kInlineDests, VEC>(S1, S1, l, dl, dt, p, dests, nd, oy, ox, vec, has_b);
-          }
+    const int r_lo = k * sh.S, r_hi = min(r_lo + sh.S, nr);
+    for (int rr = r_lo; rr < r_hi; ++rr) {
+      const uint4 rt = st::lds128(s_rtab + 16u * rr);
+      const uint32_t o0 = s_ring + rt.x, o1 = s_ring + rt.y;
+      const int y0 = (int)rt.z;
+      const float l = __uint_as_float(rt.w);
+      const int oy = Y0 + rr;
+      // parity slots: rows y0 and y0+1 are held in different register sets (R#12 taps)
+      if (y0 & 1) {
+        if (have1 != y0) { st::hrow_s(S1, o0, ca0, ca1, cb0, cb1, lx); have1 = y0; }
+        if (o1 != o0) {
+          if (have0 != y0 + 1) { st::hrow_s(S0, o1, ca0, ca1, cb0, cb1, lx); have0 = y0 + 1; }
+          emit<DT, kInlineDests, VEC>(S1, S0, l, dl, dt, p, dests, nd, oy, ox, vec, has_b);
         } else {
-          if (have0 != y0) { hrow(S0, ring + (size_t)s0 * gw, ca, cb, lx); have0 = y0; }
-          if (s1 != s0) {
-            if (have1 != y0 + 1) { hrow(S1, ring + (size_t)s1 * gw, ca, cb, lx); have1 = y0 + 1; }
-            emit<DT, kInlineDests, VEC>(S0, S1, l, dl, dt, p, dests, nd, oy, ox, vec, has_b);
-          } else {
-            emit<DT, kInlineDests, VEC>(S0, S0, l, dl, dt, p, dests, nd, oy, ox, vec, has_b);
-          }
+          emit<DT, kInlineDests, VEC>(S1, S1, l, dl, dt, p, dests, nd, oy, ox, vec, has_b);
+        }
+      } else {
+        if (have0 != y0) { st::hrow_s(S0, o0, ca0, ca1, cb0, cb1, lx); have0 = y0; }
+        if (o1 != o0) {
+          if (have1 != y0 + 1) { st::hrow_s(S1, o1, ca0, ca1, cb0, cb1, lx); have1 = y0 + 1; }
+          emit<DT, kInlineDests, VEC>(S0, S1, l, dl, dt, p, dests, nd, oy, ox, vec, has_b);
+        } else {
+          emit<DT, kInlineDests, VEC>(S0, S0, l, dl, dt, p, dests, nd, oy, ox, vec, has_b);
         }
       }
     }
