@@ -59,11 +59,12 @@ __device__ __forceinline__ void cp_async16s(uint32_t s, const void* gmem) {
 __device__ __forceinline__ void stage_rows(uint32_t raw, const uint8_t* Yp, const uint8_t* UVp, uint32_t pitch,
                                            int x16, int gw, int ya, int yb, int tid, int nthr) {
   const int ny = yb - ya + 1, u0 = ya >> 1, nuv = (yb >> 1) - u0 + 1;
-  const int chunks = gw >> 4, total = (ny + nuv) * chunks;
-  for (int e = tid; e < total; e += nthr) {
-    const int r = e / chunks, k = e - r * chunks;    // once per 16 B request
-    const uint8_t* src = r < ny ? Yp + (size_t)(ya + r) * pitch : UVp + (size_t)(u0 + r - ny) * pitch;
-    cp_async16s(raw + (uint32_t)(r * gw + k * 16), src + x16 + k * 16);
+  const int chunks = gw >> 4;
+  const int warp = tid >> 5, lane = tid & 31, nwarps = nthr >> 5;
+  for (int r = warp; r < ny + nuv; r += nwarps) {   // warps over rows, lanes over 16 B chunks
+    const uint8_t* src = (r < ny ? Yp + (size_t)(ya + r) * pitch : UVp + (size_t)(u0 + r - ny) * pitch) + x16;
+    const uint32_t dst = raw + (uint32_t)(r * gw);
+    for (int k = lane; k < chunks; k += 32) cp_async16s(dst + 16u * k, src + 16 * k);
   }
   asm volatile("cp.async.commit_group;\n" ::: "memory");
 }
@@ -155,7 +156,8 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
 
   uint2* ctab = reinterpret_cast<uint2*>(smem_raw);
   uint4* rtab = reinterpret_cast<uint4*>(smem_raw + a16((size_t)maxWo * 8));
-  const uint32_t s_base = (uint32_t)__cvta_generic_to_shared(smem_raw);
+  uint32_t s_base = (uint32_t)__cvta_generic_to_shared(smem_raw);
+  asm volatile("" : "+r"(s_base));   // materialise once: keeps the hot loops free of S2UR/LEA rebuilds
   const uint32_t s_rtab = s_base + (uint32_t)a16((size_t)maxWo * 8);
   const uint32_t s_ring = s_rtab + (uint32_t)a16((size_t)sh.SB * 16);
   const uint32_t s_raw = s_ring + (uint32_t)(sh.ring * sh.gw * 4);
