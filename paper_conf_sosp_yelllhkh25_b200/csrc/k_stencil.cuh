@@ -1,0 +1,391 @@
+// k_stencil.cuh — fused kernel for items with rotation and/or blur (two-view config;
+// SURVEY §8(a) a4-a10).
+//
+// One CTA (512 threads, ~200 KB shared memory) per work item:
+//  Phase 1  Q2 = resample(+flip) of the clip frame for all three channels into three uint8
+//           planes in shared memory, produced band by band with the staged machinery of
+//           k_resample/k_stream: cp.async of the band's NV12 footprint, conversion to an RGBx
+//           tap grid, row walkers (4 groups of column-pair threads) writing uint8 (a4-a7, Q2).
+//  Phase 2  per channel: rotation Q2 -> Q3 (bilinear inverse map, zero outside, rint; a8, Q3)
+//           then the separable blur in row strips: horizontal pass into an fp32 strip
+//           (register-blocked along x, FFMA2 over pairs of strip rows), vertical pass
+//           (FFMA2 over column pairs read as 64-bit words), rint (Q4), normalise and store to
+//           every destination (a9, a10). The free Q2 plane of the channel, or the band/Q3
+//           region, holds the fp32 strip.
+// Every fp32 operation follows R#12/R#15/R#16/R#17 with IEEE rounding in the oracle's order
+// (blur taps accumulated from 0 in tap order), so outputs are bit-identical to the oracle.
+#pragma once
+
+namespace sand {
+namespace sc {
+
+using rs::a16;
+
+struct Shape {
+  int R;            // Q2 band height (output rows)
+  int gw;           // max grid row width (bytes of Y / words of RGBx)
+  int grid_rows;    // grid / raw capacity in rows per band
+  size_t plane;     // bytes of one uint8 plane (Ho*Wo, 16-aligned)
+  size_t ubytes;    // bytes of the shared band/Q3 region
+};
+
+__host__ __device__ inline size_t band_bytes(int maxWo, int R, int grid_rows, int gw) {
+  return a16((size_t)maxWo * 8) + a16((size_t)R * 16) + (size_t)grid_rows * gw * 4 + a16((size_t)(grid_rows + grid_rows / 2 + 2) * gw);
+}
+
+__device__ __forceinline__ uint32_t ldsu8(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ void stsu8(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u8 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void stsu16(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u16 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void sts32(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void sts64f(uint32_t a, float2 v) {
+  asm volatile("st.shared.v2.f32 [%0], {%1, %2};" ::"r"(a), "f"(v.x), "f"(v.y) : "memory");
+}
+__device__ __forceinline__ float2 lds64f(uint32_t a) {
+  float2 v;
+  asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(v.x), "=f"(v.y) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ float u8f(uint32_t b) {    // exact float of a byte
+  return __fadd_rn(__uint_as_float(0x4B000000u | b), -rs::kBias);
+}
+__device__ __forceinline__ int reflect(int i, int n) { return i < 0 ? -i : (i >= n ? 2 * (n - 1) - i : i); }
+
+// destination base pointer of channel c for dest entry `dest` (element (0, 0) of the plane)
+__device__ __forceinline__ uint8_t* plane_ptr(const LaunchParams& p, uint32_t dest, int c, size_t& es) {
+  const uint32_t k = dest >> 24, t = (dest >> 16) & 0xffu, b = dest & 0xffffu;
+  const ViewConst& vc = p.views[k];
+  es = vc.dtype == SAND_U8 ? 1 : (vc.dtype == SAND_BF16 ? 2 : 4);
+  const size_t plane = (size_t)vc.out_h * vc.out_w;
+  return static_cast<uint8_t*>(p.out[k]) + (((size_t)b * 3 + c) * vc.T + t) * plane * es;
+}
+
+// normalise + store the quantised pair q (columns ox, ox+1 of row oy, channel c) to every
+// destination of the item (R#17)
+template <int DT, bool VEC>
+__device__ __forceinline__ void store_q(const LaunchParams& p, const uint32_t* dests, int nd, int c, int oy, int ox,
+                                        int Wo, float2 q, bool has_b) {
+  const bool vec = VEC || (has_b && !(Wo & 1));
+  for (int d = 0; d < nd; ++d) {
+    const uint32_t dest = dests[d];
+    const ViewConst& vc = p.views[dest >> 24];
+    const int dt = DT >= 0 ? DT : vc.dtype;
+    size_t es;
+    uint8_t* base = plane_ptr(p, dest, c, es);
+    uint8_t* o = base + ((size_t)oy * Wo + ox) * es;
+    if (dt == SAND_BF16) {
+      const float2 y = __ffma2_rn(q, make_float2(vc.a[c], vc.a[c]), make_float2(vc.b[c], vc.b[c]));
+      if (vec) {
+        *reinterpret_cast<__nv_bfloat162*>(o) = __floats2bfloat162_rn(y.x, y.y);
+      } else {
+        reinterpret_cast<__nv_bfloat16*>(o)[0] = __float2bfloat16_rn(y.x);
+        if (has_b) reinterpret_cast<__nv_bfloat16*>(o)[1] = __float2bfloat16_rn(y.y);
+      }
+    } else if (dt == SAND_F32) {
+      const float2 y = __ffma2_rn(q, make_float2(vc.a[c], vc.a[c]), make_float2(vc.b[c], vc.b[c]));
+      if (vec) {
+        *reinterpret_cast<float2*>(o) = y;
+      } else {
+        reinterpret_cast<float*>(o)[0] = y.x;
+        if (has_b) reinterpret_cast<float*>(o)[1] = y.y;
+      }
+    } else {
+      if (vec) {
+        *reinterpret_cast<uint16_t*>(o) = (uint16_t)((uint32_t)q.x | ((uint32_t)q.y << 8));
+      } else {
+        o[0] = (uint8_t)q.x;
+        if (has_b) o[1] = (uint8_t)q.y;
+      }
+    }
+  }
+}
+
+__device__ __forceinline__ float2 rint2(float2 v) {
+  return __fadd2_rn(__fadd2_rn(v, make_float2(rs::kRound, rs::kRound)), make_float2(-rs::kRound, -rs::kRound));
+}
+
+constexpr int kBX = 8;        // blur: outputs per thread along the blocked axis
+
+// Separable Gaussian blur of one channel plane with radius R (R#16): horizontal pass into
+// the fp32 scratch in row strips, vertical pass, rint (Q4), normalise and store.
+template <int DT, bool VEC, int R>
+__device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupParams& g, const uint32_t* dests, int nd,
+                                           int c, uint32_t src, uint32_t scratch, size_t plane, int Wo, int Ho,
+                                           int tid, int nthr) {
+  const int pairs = (Wo + 1) >> 1;
+  const int strip_rows = (int)(plane / ((size_t)Wo * 4));   // fp32 rows the scratch holds
+  const int S = strip_rows - 2 * R;
+  for (int ys = 0; ys < Ho; ys += S) {
+    const int ns = min(S, Ho - ys);
+    const int jrows = ns + 2 * R;          // strip row j <-> image row reflect(ys - R + j)
+    // horizontal pass: thread = (pair of strip rows j, j + half) x block of kBX columns
+    const int half = (jrows + 1) >> 1;
+    const int xblocks = (Wo + kBX - 1) / kBX;
+    for (int e = tid; e < half * xblocks; e += nthr) {
+      const int j = e / xblocks, xb = e - j * xblocks;
+      const int ja2 = j, jb2 = min(j + half, jrows - 1);
+      const uint32_t rowa = src + (uint32_t)(reflect(ys - R + ja2, Ho) * Wo);
+      const uint32_t rowb = src + (uint32_t)(reflect(ys - R + jb2, Ho) * Wo);
+      const int x0 = xb * kBX;
+      float2 win[kBX + 2 * R];
+      const bool interior = x0 - R >= 0 && x0 + kBX - 1 + R < Wo;
+#pragma unroll
+      for (int k = 0; k < kBX + 2 * R; ++k) {
+        const int xx = interior ? x0 - R + k : reflect(min(x0 - R + k, 2 * Wo - 2), Wo);
+        win[k] = make_float2(u8f(ldsu8(rowa + (uint32_t)xx)), u8f(ldsu8(rowb + (uint32_t)xx)));
+      }
+      float2 accs[kBX];
+#pragma unroll
+      for (int o = 0; o < kBX; ++o) accs[o] = make_float2(0.f, 0.f);
+#pragma unroll
+      for (int i = 0; i <= 2 * R; ++i) {           // taps in order: acc = fmaf(w_i, v, acc)
+        const float wi = g.blur_w[i];
+#pragma unroll
+        for (int o = 0; o < kBX; ++o) accs[o] = __ffma2_rn(make_float2(wi, wi), win[o + i], accs[o]);
+      }
+#pragma unroll
+      for (int o = 0; o < kBX; ++o) {
+        const float2 acc = accs[o];
+        if (x0 + o < Wo) {
+          asm volatile("st.shared.f32 [%0], %1;" ::"r"(scratch + 4u * (uint32_t)(ja2 * Wo + x0 + o)), "f"(acc.x)
+                       : "memory");
+          asm volatile("st.shared.f32 [%0], %1;" ::"r"(scratch + 4u * (uint32_t)(jb2 * Wo + x0 + o)), "f"(acc.y)
+                       : "memory");
+        }
+      }
+    }
+    __syncthreads();
+    // vertical pass: thread = column pair (x, x+1) x block of kBX output rows
+    const int rblocks = (ns + kBX - 1) / kBX;
+    for (int e = tid; e < pairs * rblocks; e += nthr) {
+      const int rb = e / pairs, pr2 = e - rb * pairs;
+      const int ox = 2 * pr2, y0 = rb * kBX;
+      const bool has_b = ox + 1 < Wo;
+      float2 win[kBX + 2 * R];
+#pragma unroll
+      for (int k = 0; k < kBX + 2 * R; ++k) {
+        win[k] = make_float2(0.f, 0.f);
+        if (y0 + k < jrows) {
+          const uint32_t a = scratch + 4u * (uint32_t)((y0 + k) * Wo + ox);
+          win[k] = has_b && !(Wo & 1) ? lds64f(a) : make_float2(__uint_as_float(st::lds32(a)),
+                                                                  has_b ? __uint_as_float(st::lds32(a + 4)) : 0.f);
+        }
+      }
+      float2 accs[kBX];
+#pragma unroll
+      for (int o = 0; o < kBX; ++o) accs[o] = make_float2(0.f, 0.f);
+#pragma unroll
+      for (int i = 0; i <= 2 * R; ++i) {
+        const float wi = g.blur_w[i];
+#pragma unroll
+        for (int o = 0; o < kBX; ++o) accs[o] = __ffma2_rn(make_float2(wi, wi), win[o + i], accs[o]);
+      }
+#pragma unroll
+      for (int o = 0; o < kBX; ++o) {
+        if (y0 + o >= ns) break;
+        store_q<DT, VEC>(p, dests, nd, c, ys + y0 + o, ox, Wo, rint2(accs[o]), has_b);
+      }
+    }
+    __syncthreads();
+  }
+}
+
+}  // namespace sc
+
+template <int DT, bool VEC>
+__global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::Shape sh, int maxWo) {
+  extern __shared__ __align__(16) uint8_t smem_raw[];
+  using namespace rs;
+  using namespace sc;
+  const WorkItem w = p.items[blockIdx.x];
+  if (!(w.flags & 1u)) return;
+  const GroupParams& g = p.groups[w.gp];
+  const int Wo = g.out_w, Ho = g.out_h;
+  const int tid = threadIdx.x, nthr = blockDim.x;
+  const int warp = tid >> 5, lane = tid & 31, nwarps = nthr >> 5;
+  uint32_t s_base = (uint32_t)__cvta_generic_to_shared(smem_raw);
+  asm volatile("" : "+r"(s_base));
+  const uint32_t q2 = s_base;                                  // 3 planes of sh.plane bytes
+  const uint32_t ureg = s_base + (uint32_t)(3 * sh.plane);     // band buffers / Q3 plane
+  uint2* ctab = reinterpret_cast<uint2*>(smem_raw + 3 * sh.plane);
+  uint4* rtab = reinterpret_cast<uint4*>(smem_raw + 3 * sh.plane + a16((size_t)maxWo * 8));
+  const uint32_t s_grid = ureg + (uint32_t)(a16((size_t)maxWo * 8) + a16((size_t)sh.R * 16));
+  const uint32_t s_rawb = s_grid + (uint32_t)(sh.grid_rows * sh.gw * 4);
+  const uint32_t* dests = p.dests + w.dest_begin;
+  const int nd = (int)w.n_dest;
+
+  // ------------------------------------------------------------- phase 1: Q2 planes
+  const int x_lo = tap0(g.sc_x, g.off_x, 0, g.org_x);
+  int x_hi, dmy;
+  float fl;
+  tap(g.sc_x, g.off_x, Wo - 1, g.lim_x, g.org_x, dmy, x_hi, fl);
+  const int x16 = x_lo & ~15;
+  const int gw = ((x_hi + 16) & ~15) - x16;
+  const uint32_t rowbytes = (uint32_t)gw * 4u;
+  const uint8_t* Yp = p.slab + w.y_off;
+  const uint8_t* UVp = Yp + (size_t)w.pitch * w.src_h;
+  for (int j = tid; j < Wo; j += nthr) {
+    int x0, x1;
+    float lx;
+    tap(g.sc_x, g.off_x, j, g.lim_x, g.org_x, x0, x1, lx);
+    ctab[j] = make_uint2((uint32_t)(x0 - x16) | ((uint32_t)(x1 - x16) << 16), __float_as_uint(lx));
+  }
+  const int pairs = (Wo + 1) >> 1;
+  const int groups = max(1, nthr / pairs);
+  const int grp = tid / pairs, pr = tid - grp * pairs;
+  for (int oy_lo = 0; oy_lo < Ho; oy_lo += sh.R) {
+    const int nr = min(sh.R, Ho - oy_lo);
+    const int y_lo = tap0(g.sc_y, g.off_y, oy_lo, g.org_y);
+    int y_hi;
+    tap(g.sc_y, g.off_y, oy_lo + nr - 1, g.lim_y, g.org_y, dmy, y_hi, fl);
+    __syncthreads();                          // previous band's walkers are done with the grid
+    st::stage_rows(s_rawb, Yp, UVp, w.pitch, x16, gw, y_lo, y_hi, tid, nthr);
+    for (int r = tid; r < nr; r += nthr) {
+      int y0, y1;
+      float ly;
+      tap(g.sc_y, g.off_y, oy_lo + r, g.lim_y, g.org_y, y0, y1, ly);
+      rtab[r] = make_uint4((uint32_t)(y0 - y_lo) * rowbytes, (uint32_t)(y1 - y_lo) * rowbytes, (uint32_t)y0,
+                           __float_as_uint(ly));
+    }
+    asm volatile("cp.async.wait_group 0;\n" ::: "memory");
+    __syncthreads();
+    st::convert_rows(s_grid, s_rawb, gw, y_lo, y_hi, y_lo, 1 << 30, warp, nwarps, lane);
+    __syncthreads();
+    if (grp < groups && pr < pairs) {
+      const int ox = 2 * pr;
+      const bool has_b = ox + 1 < Wo;
+      const int ja = g.flip ? Wo - 1 - ox : ox;
+      const int jb = has_b ? (g.flip ? Wo - 2 - ox : ox + 1) : ja;
+      const uint2 ta = ctab[ja], tb = ctab[jb];
+      const uint32_t ca0 = 4u * (ta.x & 0xffffu), ca1 = 4u * (ta.x >> 16);
+      const uint32_t cb0 = 4u * (tb.x & 0xffffu), cb1 = 4u * (tb.x >> 16);
+      const float2 lx = make_float2(__uint_as_float(ta.y), __uint_as_float(tb.y));
+      const int per = (nr + groups - 1) / groups;
+      const int r_lo = grp * per, r_hi = min(nr, r_lo + per);
+      int have0 = -1, have1 = -1;
+      Row3 S0, S1;
+      for (int rr = r_lo; rr < r_hi; ++rr) {
+        const uint4 rt = st::lds128((uint32_t)__cvta_generic_to_shared(rtab) + 16u * rr);
+        const uint32_t o0 = s_grid + rt.x, o1 = s_grid + rt.y;
+        const int y0 = (int)rt.z;
+        const float2 ly = make_float2(__uint_as_float(rt.w), __uint_as_float(rt.w));
+        const Row3* top;
+        const Row3* bot;
+        if (y0 & 1) {
+          if (have1 != y0) { st::hrow_s(S1, o0, ca0, ca1, cb0, cb1, lx); have1 = y0; }
+          top = &S1;
+          bot = &S1;
+          if (o1 != o0) {
+            if (have0 != y0 + 1) { st::hrow_s(S0, o1, ca0, ca1, cb0, cb1, lx); have0 = y0 + 1; }
+            bot = &S0;
+          }
+        } else {
+          if (have0 != y0) { st::hrow_s(S0, o0, ca0, ca1, cb0, cb1, lx); have0 = y0; }
+          top = &S0;
+          bot = &S0;
+          if (o1 != o0) {
+            if (have1 != y0 + 1) { st::hrow_s(S1, o1, ca0, ca1, cb0, cb1, lx); have1 = y0 + 1; }
+            bot = &S1;
+          }
+        }
+        const uint32_t pix = (uint32_t)((oy_lo + rr) * Wo + ox);
+#pragma unroll
+        for (int c = 0; c < 3; ++c) {
+          const float2 dv = __ffma2_rn(top->h[c], make_float2(-1.f, -1.f), bot->h[c]);
+          const float2 q = rint2(__ffma2_rn(ly, dv, top->h[c]));
+          const uint32_t plane = q2 + (uint32_t)(c * sh.plane) + pix;
+          if (has_b) stsu16(plane, (uint32_t)q.x | ((uint32_t)q.y << 8));
+          else stsu8(plane, (uint32_t)q.x);
+        }
+      }
+    }
+  }
+  __syncthreads();
+
+  // ------------------------------------------------------------- phase 2: per channel
+  const int n = Ho * Wo;
+  const int r = g.blur_on ? g.blur_r : 0;
+  const float cxo = (float)(Wo - 1) * 0.5f, cyo = (float)(Ho - 1) * 0.5f;
+  for (int c = 0; c < 3; ++c) {
+    uint32_t src = q2 + (uint32_t)(c * sh.plane);
+    uint32_t scratch = ureg;
+    if (g.rot_on) {                            // a8: Q3 = rotate(Q2) (R#15)
+      const uint32_t q3 = ureg;
+      for (int e = tid; e < (n + 1) / 2; e += nthr) {
+        const int pix = 2 * e;
+        const int oy = pix / Wo, ox = pix - oy * Wo;
+        // two horizontally adjacent outputs (the second may wrap to the next row)
+        const int oy2 = ox + 1 < Wo ? oy : oy + 1, ox2 = ox + 1 < Wo ? ox + 1 : 0;
+        const float2 xc = make_float2(__fsub_rn((float)ox, cxo), __fsub_rn((float)ox2, cxo));
+        const float2 yc = make_float2(__fsub_rn((float)oy, cyo), __fsub_rn((float)oy2, cyo));
+        const float2 sx = __fadd2_rn(__fadd2_rn(__fmul2_rn(make_float2(g.rot_c, g.rot_c), xc),
+                                                __fmul2_rn(make_float2(-g.rot_s, -g.rot_s), yc)),
+                                     make_float2(cxo, cxo));
+        const float2 sy = __fadd2_rn(__fadd2_rn(__fmul2_rn(make_float2(g.rot_s, g.rot_s), xc),
+                                                __fmul2_rn(make_float2(g.rot_c, g.rot_c), yc)),
+                                     make_float2(cyo, cyo));
+        float2 v;
+        float* vv = &v.x;
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const float fx = floorf(h ? sx.y : sx.x), fy = floorf(h ? sy.y : sy.x);
+          const float lxr = __fsub_rn(h ? sx.y : sx.x, fx), lyr = __fsub_rn(h ? sy.y : sy.x, fy);
+          const int x0 = (int)fx, y0 = (int)fy;
+          float t[2][2];
+#pragma unroll
+          for (int dy = 0; dy < 2; ++dy)
+#pragma unroll
+            for (int dx = 0; dx < 2; ++dx) {
+              const int xx = x0 + dx, yy = y0 + dy;
+              t[dy][dx] = (xx >= 0 && xx < Wo && yy >= 0 && yy < Ho) ? u8f(ldsu8(src + (uint32_t)(yy * Wo + xx))) : 0.f;
+            }
+          const float h0 = __fmaf_rn(lxr, __fsub_rn(t[0][1], t[0][0]), t[0][0]);
+          const float h1 = __fmaf_rn(lxr, __fsub_rn(t[1][1], t[1][0]), t[1][0]);
+          vv[h] = __fmaf_rn(lyr, __fsub_rn(h1, h0), h0);
+        }
+        const float2 q = rint2(v);
+        stsu8(q3 + (uint32_t)pix, (uint32_t)q.x);
+        if (pix + 1 < n) stsu8(q3 + (uint32_t)pix + 1, (uint32_t)q.y);
+      }
+      __syncthreads();
+      src = q3;
+      scratch = q2 + (uint32_t)(c * sh.plane);   // this channel's Q2 plane is free now
+    }
+    if (g.blur_on) {                           // a9: separable Gaussian in strips (R#16)
+      switch (r) {
+        case 0: blur_plane<DT, VEC, 0>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 1: blur_plane<DT, VEC, 1>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 2: blur_plane<DT, VEC, 2>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 3: blur_plane<DT, VEC, 3>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 4: blur_plane<DT, VEC, 4>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 5: blur_plane<DT, VEC, 5>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 6: blur_plane<DT, VEC, 6>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 7: blur_plane<DT, VEC, 7>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 8: blur_plane<DT, VEC, 8>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 9: blur_plane<DT, VEC, 9>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 10: blur_plane<DT, VEC, 10>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        default: blur_plane<DT, VEC, 11>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+      }
+    } else {                                   // no blur: normalise + store the (rotated) plane
+      for (int e = tid; e < Ho * pairs; e += nthr) {
+        const int oy = e / pairs, ox = 2 * (e - oy * pairs);
+        const bool has_b = ox + 1 < Wo;
+        const uint32_t a = src + (uint32_t)(oy * Wo + ox);
+        const float2 q = make_float2(u8f(ldsu8(a)), has_b ? u8f(ldsu8(a + 1)) : 0.f);
+        store_q<DT, VEC>(p, dests, nd, c, oy, ox, Wo, q, has_b);
+      }
+      __syncthreads();
+    }
+  }
+}
+
+}  // namespace sand

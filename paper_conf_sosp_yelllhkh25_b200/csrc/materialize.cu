@@ -170,6 +170,7 @@ __global__ void __launch_bounds__(512) k_stencil(const LaunchParams p) {
 
 #include "k_resample.cuh"
 #include "k_stream.cuh"
+#include "k_stencil.cuh"
 
 namespace sand {
 
@@ -254,6 +255,27 @@ int launch_resample_dt(const LaunchParams& p, const BatchShape& sh, cudaStream_t
   return SAND_OK;
 }
 
+// stencil kernel shape: Q2 band height R such that 3 planes + band/Q3 region fit 227 KB
+bool choose_stencil(const BatchShape& sh, sc::Shape* out, size_t* smem) {
+  const size_t plane = rs::a16((size_t)sh.st_max_wo * sh.st_max_ho);
+  const int gw = (int)rs::a16((size_t)sh.st_cols_bound) + 16;
+  const bool mild = sh.st_cols_bound <= 2 * sh.st_max_wo + 16 && sh.st_max_scy <= 2.0f;
+  if (!mild || sh.st_max_wo > 1024) return false;
+  static const int kCands[] = {64, 48, 32, 24, 16, 12, 8, 4};
+  for (int r : kCands) {
+    const int rows = (int)std::ceil((double)sh.st_max_scy * r) + 3;
+    const size_t band = sc::band_bytes(sh.st_max_wo, r, rows, gw);
+    const size_t u = std::max(plane, band);
+    const size_t total = 3 * plane + u;
+    if (total <= 227 * 1024) {
+      *out = sc::Shape{r, gw, rows, plane, u};
+      *smem = total;
+      return true;
+    }
+  }
+  return false;
+}
+
 template <typename K>
 cudaError_t allow_smem(K kernel) {
   cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
@@ -275,7 +297,9 @@ int configure_kernels(size_t stencil_smem) {
                           allow_smem(k_resample_gather<-1, false>), allow_smem(k_resample_gather<SAND_U8, true>),
                           allow_smem(k_resample_gather<SAND_BF16, true>), allow_smem(k_resample_gather<SAND_F32, true>),
                           allow_smem(k_stream<-1, false>), allow_smem(k_stream<SAND_U8, true>),
-                          allow_smem(k_stream<SAND_BF16, true>), allow_smem(k_stream<SAND_F32, true>)})
+                          allow_smem(k_stream<SAND_BF16, true>), allow_smem(k_stream<SAND_F32, true>),
+                          allow_smem(k_stencil2<-1, false>), allow_smem(k_stencil2<SAND_U8, true>),
+                          allow_smem(k_stencil2<SAND_BF16, true>), allow_smem(k_stencil2<SAND_F32, true>)})
       if (r != cudaSuccess) e = r;
     if (e != cudaSuccess) return cuda_error(e, "cudaFuncSetAttribute(k_resample)");
   }
@@ -305,6 +329,19 @@ int launch_materialize(const LaunchParams& p, const BatchShape& shape, size_t st
     ++*n_launched;
   }
   if (shape.has_stencil) {
+    sc::Shape scs;
+    size_t smem2;
+    if (getenv("SAND_STENCIL_V1") == nullptr && choose_stencil(shape, &scs, &smem2)) {
+      const int dt = shape.even_wo ? shape.dtype : -1;
+      if (dt == SAND_U8) k_stencil2<SAND_U8, true><<<p.n_items, 512, smem2, stream>>>(p, scs, shape.st_max_wo);
+      else if (dt == SAND_BF16) k_stencil2<SAND_BF16, true><<<p.n_items, 512, smem2, stream>>>(p, scs, shape.st_max_wo);
+      else if (dt == SAND_F32) k_stencil2<SAND_F32, true><<<p.n_items, 512, smem2, stream>>>(p, scs, shape.st_max_wo);
+      else k_stencil2<-1, false><<<p.n_items, 512, smem2, stream>>>(p, scs, shape.st_max_wo);
+      cudaError_t e = cudaGetLastError();
+      if (e != cudaSuccess) return cuda_error(e, "k_stencil2 launch");
+      ++*n_launched;
+      return SAND_OK;
+    }
     k_stencil<<<p.n_items, 512, stencil_smem, stream>>>(p);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_error(e, "k_stencil launch");

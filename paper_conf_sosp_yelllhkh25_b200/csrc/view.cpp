@@ -142,6 +142,11 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
           w.flags = (g.rot_on || g.blur_on) ? 1u : 0u;
           if (w.flags) {
             shape.has_stencil = 1;
+            shape.st_max_wo = std::max(shape.st_max_wo, g.out_w);
+            shape.st_max_ho = std::max(shape.st_max_ho, g.out_h);
+            const int cols = std::min(2 * g.out_w, static_cast<int>(std::ceil(static_cast<double>(g.sc_x) * g.out_w)) + 3);
+            shape.st_cols_bound = std::max(shape.st_cols_bound, cols);
+            shape.st_max_scy = std::max(shape.st_max_scy, g.sc_y);
           } else {
             shape.has_direct = 1;
             shape.max_wo = std::max(shape.max_wo, g.out_w);
