@@ -69,44 +69,71 @@ __device__ __forceinline__ uint8_t* plane_ptr(const LaunchParams& p, uint32_t de
   return static_cast<uint8_t*>(p.out[k]) + (((size_t)b * 3 + c) * vc.T + t) * plane * es;
 }
 
-// normalise + store the quantised pair q (columns ox, ox+1 of row oy, channel c) to every
-// destination of the item (R#17)
+// one destination plane (view, clip, t, channel) with its normalisation constants (R#17)
+struct ChDest {
+  uint8_t* base;     // element (0, 0) of the plane
+  float a, b;
+  int dt, es;
+};
+
+__device__ __forceinline__ ChDest ch_dest(const LaunchParams& p, uint32_t dest, int c) {
+  const ViewConst& vc = p.views[dest >> 24];
+  size_t es;
+  ChDest d;
+  d.base = plane_ptr(p, dest, c, es);
+  d.es = (int)es;
+  d.dt = vc.dtype;
+  d.a = vc.a[c];
+  d.b = vc.b[c];
+  return d;
+}
+
 template <int DT, bool VEC>
-__device__ __forceinline__ void store_q(const LaunchParams& p, const uint32_t* dests, int nd, int c, int oy, int ox,
-                                        int Wo, float2 q, bool has_b) {
+__device__ __forceinline__ void put_q(const ChDest& d, int oy, int ox, int Wo, float2 q, bool has_b) {
   const bool vec = VEC || (has_b && !(Wo & 1));
-  for (int d = 0; d < nd; ++d) {
-    const uint32_t dest = dests[d];
-    const ViewConst& vc = p.views[dest >> 24];
-    const int dt = DT >= 0 ? DT : vc.dtype;
-    size_t es;
-    uint8_t* base = plane_ptr(p, dest, c, es);
-    uint8_t* o = base + ((size_t)oy * Wo + ox) * es;
-    if (dt == SAND_BF16) {
-      const float2 y = __ffma2_rn(q, make_float2(vc.a[c], vc.a[c]), make_float2(vc.b[c], vc.b[c]));
-      if (vec) {
-        *reinterpret_cast<__nv_bfloat162*>(o) = __floats2bfloat162_rn(y.x, y.y);
-      } else {
-        reinterpret_cast<__nv_bfloat16*>(o)[0] = __float2bfloat16_rn(y.x);
-        if (has_b) reinterpret_cast<__nv_bfloat16*>(o)[1] = __float2bfloat16_rn(y.y);
-      }
-    } else if (dt == SAND_F32) {
-      const float2 y = __ffma2_rn(q, make_float2(vc.a[c], vc.a[c]), make_float2(vc.b[c], vc.b[c]));
-      if (vec) {
-        *reinterpret_cast<float2*>(o) = y;
-      } else {
-        reinterpret_cast<float*>(o)[0] = y.x;
-        if (has_b) reinterpret_cast<float*>(o)[1] = y.y;
-      }
+  const int dt = DT >= 0 ? DT : d.dt;
+  const int es = DT >= 0 ? (DT == SAND_U8 ? 1 : (DT == SAND_BF16 ? 2 : 4)) : d.es;
+  uint8_t* o = d.base + (size_t)(oy * Wo + ox) * es;
+  if (dt == SAND_BF16) {
+    const float2 y = __ffma2_rn(q, make_float2(d.a, d.a), make_float2(d.b, d.b));
+    if (vec) {
+      *reinterpret_cast<__nv_bfloat162*>(o) = __floats2bfloat162_rn(y.x, y.y);
     } else {
-      if (vec) {
-        *reinterpret_cast<uint16_t*>(o) = (uint16_t)((uint32_t)q.x | ((uint32_t)q.y << 8));
-      } else {
-        o[0] = (uint8_t)q.x;
-        if (has_b) o[1] = (uint8_t)q.y;
-      }
+      reinterpret_cast<__nv_bfloat16*>(o)[0] = __float2bfloat16_rn(y.x);
+      if (has_b) reinterpret_cast<__nv_bfloat16*>(o)[1] = __float2bfloat16_rn(y.y);
+    }
+  } else if (dt == SAND_F32) {
+    const float2 y = __ffma2_rn(q, make_float2(d.a, d.a), make_float2(d.b, d.b));
+    if (vec) {
+      *reinterpret_cast<float2*>(o) = y;
+    } else {
+      reinterpret_cast<float*>(o)[0] = y.x;
+      if (has_b) reinterpret_cast<float*>(o)[1] = y.y;
+    }
+  } else {
+    if (vec) {
+      *reinterpret_cast<uint16_t*>(o) = (uint16_t)((uint32_t)q.x | ((uint32_t)q.y << 8));
+    } else {
+      o[0] = (uint8_t)q.x;
+      if (has_b) o[1] = (uint8_t)q.y;
     }
   }
+}
+
+// the destinations of one channel: two in registers, the rest recomputed (rare)
+struct ChDests {
+  ChDest d0, d1;
+  int nd;
+  const uint32_t* dests;
+  int c;
+};
+
+template <int DT, bool VEC>
+__device__ __forceinline__ void store_q(const LaunchParams& p, const ChDests& cd, int oy, int ox, int Wo, float2 q,
+                                        bool has_b) {
+  put_q<DT, VEC>(cd.d0, oy, ox, Wo, q, has_b);
+  if (cd.nd > 1) put_q<DT, VEC>(cd.d1, oy, ox, Wo, q, has_b);
+  for (int d = 2; d < cd.nd; ++d) put_q<DT, VEC>(ch_dest(p, cd.dests[d], cd.c), oy, ox, Wo, q, has_b);
 }
 
 __device__ __forceinline__ float2 rint2(float2 v) {
@@ -118,8 +145,8 @@ constexpr int kBX = 8;        // blur: outputs per thread along the blocked axis
 // Separable Gaussian blur of one channel plane with radius R (R#16): horizontal pass into
 // the fp32 scratch in row strips, vertical pass, rint (Q4), normalise and store.
 template <int DT, bool VEC, int R>
-__device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupParams& g, const uint32_t* dests, int nd,
-                                           int c, uint32_t src, uint32_t scratch, size_t plane, int Wo, int Ho,
+__device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupParams& g, const ChDests& cd,
+                                           uint32_t src, uint32_t scratch, size_t plane, int Wo, int Ho,
                                            int tid, int nthr) {
   const int pairs = (Wo + 1) >> 1;
   const int strip_rows = (int)(plane / ((size_t)Wo * 4));   // fp32 rows the scratch holds
@@ -192,7 +219,7 @@ __device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupPar
 #pragma unroll
       for (int o = 0; o < kBX; ++o) {
         if (y0 + o >= ns) break;
-        store_q<DT, VEC>(p, dests, nd, c, ys + y0 + o, ox, Wo, rint2(accs[o]), has_b);
+        store_q<DT, VEC>(p, cd, ys + y0 + o, ox, Wo, rint2(accs[o]), has_b);
       }
     }
     __syncthreads();
@@ -218,6 +245,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
   const uint32_t ureg = s_base + (uint32_t)(3 * sh.plane);     // band buffers / Q3 plane
   uint2* ctab = reinterpret_cast<uint2*>(smem_raw + 3 * sh.plane);
   uint4* rtab = reinterpret_cast<uint4*>(smem_raw + 3 * sh.plane + a16((size_t)maxWo * 8));
+  const uint32_t s_rtab = ureg + (uint32_t)a16((size_t)maxWo * 8);
   const uint32_t s_grid = ureg + (uint32_t)(a16((size_t)maxWo * 8) + a16((size_t)sh.R * 16));
   const uint32_t s_rawb = s_grid + (uint32_t)(sh.grid_rows * sh.gw * 4);
   const uint32_t* dests = p.dests + w.dest_begin;
@@ -274,37 +302,37 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
       int have0 = -1, have1 = -1;
       Row3 S0, S1;
       for (int rr = r_lo; rr < r_hi; ++rr) {
-        const uint4 rt = st::lds128((uint32_t)__cvta_generic_to_shared(rtab) + 16u * rr);
+        const uint4 rt = st::lds128(s_rtab + 16u * rr);
         const uint32_t o0 = s_grid + rt.x, o1 = s_grid + rt.y;
         const int y0 = (int)rt.z;
         const float2 ly = make_float2(__uint_as_float(rt.w), __uint_as_float(rt.w));
-        const Row3* top;
-        const Row3* bot;
+        const uint32_t pix = (uint32_t)((oy_lo + rr) * Wo + ox);
+        auto put3 = [&](const Row3& top, const Row3& bot) {   // vertical lerp + rint -> Q2 planes
+#pragma unroll
+          for (int c = 0; c < 3; ++c) {
+            const float2 dv = __ffma2_rn(top.h[c], make_float2(-1.f, -1.f), bot.h[c]);
+            const float2 q = rint2(__ffma2_rn(ly, dv, top.h[c]));
+            const uint32_t plane = q2 + (uint32_t)(c * sh.plane) + pix;
+            if (has_b) stsu16(plane, (uint32_t)q.x | ((uint32_t)q.y << 8));
+            else stsu8(plane, (uint32_t)q.x);
+          }
+        };
         if (y0 & 1) {
           if (have1 != y0) { st::hrow_s(S1, o0, ca0, ca1, cb0, cb1, lx); have1 = y0; }
-          top = &S1;
-          bot = &S1;
           if (o1 != o0) {
             if (have0 != y0 + 1) { st::hrow_s(S0, o1, ca0, ca1, cb0, cb1, lx); have0 = y0 + 1; }
-            bot = &S0;
+            put3(S1, S0);
+          } else {
+            put3(S1, S1);
           }
         } else {
           if (have0 != y0) { st::hrow_s(S0, o0, ca0, ca1, cb0, cb1, lx); have0 = y0; }
-          top = &S0;
-          bot = &S0;
           if (o1 != o0) {
             if (have1 != y0 + 1) { st::hrow_s(S1, o1, ca0, ca1, cb0, cb1, lx); have1 = y0 + 1; }
-            bot = &S1;
+            put3(S0, S1);
+          } else {
+            put3(S0, S0);
           }
-        }
-        const uint32_t pix = (uint32_t)((oy_lo + rr) * Wo + ox);
-#pragma unroll
-        for (int c = 0; c < 3; ++c) {
-          const float2 dv = __ffma2_rn(top->h[c], make_float2(-1.f, -1.f), bot->h[c]);
-          const float2 q = rint2(__ffma2_rn(ly, dv, top->h[c]));
-          const uint32_t plane = q2 + (uint32_t)(c * sh.plane) + pix;
-          if (has_b) stsu16(plane, (uint32_t)q.x | ((uint32_t)q.y << 8));
-          else stsu8(plane, (uint32_t)q.x);
         }
       }
     }
@@ -316,45 +344,51 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
   const int r = g.blur_on ? g.blur_r : 0;
   const float cxo = (float)(Wo - 1) * 0.5f, cyo = (float)(Ho - 1) * 0.5f;
   for (int c = 0; c < 3; ++c) {
+    ChDests cd;
+    cd.nd = nd;
+    cd.dests = dests;
+    cd.c = c;
+    cd.d0 = ch_dest(p, dests[0], c);
+    if (nd > 1) cd.d1 = ch_dest(p, dests[1], c);
     uint32_t src = q2 + (uint32_t)(c * sh.plane);
     uint32_t scratch = ureg;
     if (g.rot_on) {                            // a8: Q3 = rotate(Q2) (R#15)
       const uint32_t q3 = ureg;
-      for (int e = tid; e < (n + 1) / 2; e += nthr) {
-        const int pix = 2 * e;
-        const int oy = pix / Wo, ox = pix - oy * Wo;
-        // two horizontally adjacent outputs (the second may wrap to the next row)
-        const int oy2 = ox + 1 < Wo ? oy : oy + 1, ox2 = ox + 1 < Wo ? ox + 1 : 0;
-        const float2 xc = make_float2(__fsub_rn((float)ox, cxo), __fsub_rn((float)ox2, cxo));
-        const float2 yc = make_float2(__fsub_rn((float)oy, cyo), __fsub_rn((float)oy2, cyo));
-        const float2 sx = __fadd2_rn(__fadd2_rn(__fmul2_rn(make_float2(g.rot_c, g.rot_c), xc),
-                                                __fmul2_rn(make_float2(-g.rot_s, -g.rot_s), yc)),
-                                     make_float2(cxo, cxo));
-        const float2 sy = __fadd2_rn(__fadd2_rn(__fmul2_rn(make_float2(g.rot_s, g.rot_s), xc),
-                                                __fmul2_rn(make_float2(g.rot_c, g.rot_c), yc)),
-                                     make_float2(cyo, cyo));
-        float2 v;
-        float* vv = &v.x;
-#pragma unroll
-        for (int h = 0; h < 2; ++h) {
-          const float fx = floorf(h ? sx.y : sx.x), fy = floorf(h ? sy.y : sy.x);
-          const float lxr = __fsub_rn(h ? sx.y : sx.x, fx), lyr = __fsub_rn(h ? sy.y : sy.x, fy);
+      const float rc = g.rot_c, rsn = g.rot_s, nrs = -g.rot_s;
+      for (int oy = warp; oy < Ho; oy += nwarps) {
+        const float yc = __fsub_rn((float)oy, cyo);
+        const float tx = __fmul_rn(nrs, yc), ty = __fmul_rn(rc, yc);   // row terms of R#15
+        const uint32_t orow = q3 + (uint32_t)(oy * Wo);
+        float xc = __fsub_rn((float)lane, cxo);
+        for (int ox = lane; ox < Wo; ox += 32, xc = __fadd_rn(xc, 32.f)) {
+          // sx = (c*xc + (-s)*yc) + cx, sy = (s*xc + c*yc) + cy, every op rounded (scalar IEEE)
+          const float sx = __fadd_rn(__fadd_rn(__fmul_rn(rc, xc), tx), cxo);
+          const float sy = __fadd_rn(__fadd_rn(__fmul_rn(rsn, xc), ty), cyo);
+          const float fx = floorf(sx), fy = floorf(sy);
+          const float lxr = __fsub_rn(sx, fx), lyr = __fsub_rn(sy, fy);
           const int x0 = (int)fx, y0 = (int)fy;
-          float t[2][2];
-#pragma unroll
-          for (int dy = 0; dy < 2; ++dy)
-#pragma unroll
-            for (int dx = 0; dx < 2; ++dx) {
-              const int xx = x0 + dx, yy = y0 + dy;
-              t[dy][dx] = (xx >= 0 && xx < Wo && yy >= 0 && yy < Ho) ? u8f(ldsu8(src + (uint32_t)(yy * Wo + xx))) : 0.f;
-            }
-          const float h0 = __fmaf_rn(lxr, __fsub_rn(t[0][1], t[0][0]), t[0][0]);
-          const float h1 = __fmaf_rn(lxr, __fsub_rn(t[1][1], t[1][0]), t[1][0]);
-          vv[h] = __fmaf_rn(lyr, __fsub_rn(h1, h0), h0);
+          float t00, t01, t10, t11;
+          if ((unsigned)x0 < (unsigned)(Wo - 1) && (unsigned)y0 < (unsigned)(Ho - 1)) {
+            const uint32_t a0 = src + (uint32_t)(y0 * Wo + x0);
+            t00 = u8f(ldsu8(a0));
+            t01 = u8f(ldsu8(a0 + 1));
+            t10 = u8f(ldsu8(a0 + (uint32_t)Wo));
+            t11 = u8f(ldsu8(a0 + (uint32_t)Wo + 1));
+          } else {                               // taps outside the image read 0 (fill=None)
+            auto tapv = [&](int xx, int yy) {
+              return (xx >= 0 && xx < Wo && yy >= 0 && yy < Ho) ? u8f(ldsu8(src + (uint32_t)(yy * Wo + xx))) : 0.f;
+            };
+            t00 = tapv(x0, y0);
+            t01 = tapv(x0 + 1, y0);
+            t10 = tapv(x0, y0 + 1);
+            t11 = tapv(x0 + 1, y0 + 1);
+          }
+          const float h0 = __fmaf_rn(lxr, __fsub_rn(t01, t00), t00);
+          const float h1 = __fmaf_rn(lxr, __fsub_rn(t11, t10), t10);
+          // rint via +1.5*2^23: the integer lands in the low mantissa bits (0..255)
+          const float tq = __fadd_rn(__fmaf_rn(lyr, __fsub_rn(h1, h0), h0), rs::kRound);
+          stsu8(orow + (uint32_t)ox, __float_as_uint(tq) & 0xffu);
         }
-        const float2 q = rint2(v);
-        stsu8(q3 + (uint32_t)pix, (uint32_t)q.x);
-        if (pix + 1 < n) stsu8(q3 + (uint32_t)pix + 1, (uint32_t)q.y);
       }
       __syncthreads();
       src = q3;
@@ -362,26 +396,27 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
     }
     if (g.blur_on) {                           // a9: separable Gaussian in strips (R#16)
       switch (r) {
-        case 0: blur_plane<DT, VEC, 0>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 1: blur_plane<DT, VEC, 1>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 2: blur_plane<DT, VEC, 2>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 3: blur_plane<DT, VEC, 3>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 4: blur_plane<DT, VEC, 4>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 5: blur_plane<DT, VEC, 5>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 6: blur_plane<DT, VEC, 6>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 7: blur_plane<DT, VEC, 7>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 8: blur_plane<DT, VEC, 8>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 9: blur_plane<DT, VEC, 9>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 10: blur_plane<DT, VEC, 10>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        default: blur_plane<DT, VEC, 11>(p, g, dests, nd, c, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 0: blur_plane<DT, VEC, 0>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 1: blur_plane<DT, VEC, 1>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 2: blur_plane<DT, VEC, 2>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 3: blur_plane<DT, VEC, 3>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 4: blur_plane<DT, VEC, 4>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 5: blur_plane<DT, VEC, 5>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 6: blur_plane<DT, VEC, 6>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 7: blur_plane<DT, VEC, 7>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 8: blur_plane<DT, VEC, 8>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 9: blur_plane<DT, VEC, 9>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 10: blur_plane<DT, VEC, 10>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        default: blur_plane<DT, VEC, 11>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
       }
     } else {                                   // no blur: normalise + store the (rotated) plane
-      for (int e = tid; e < Ho * pairs; e += nthr) {
-        const int oy = e / pairs, ox = 2 * (e - oy * pairs);
-        const bool has_b = ox + 1 < Wo;
-        const uint32_t a = src + (uint32_t)(oy * Wo + ox);
-        const float2 q = make_float2(u8f(ldsu8(a)), has_b ? u8f(ldsu8(a + 1)) : 0.f);
-        store_q<DT, VEC>(p, dests, nd, c, oy, ox, Wo, q, has_b);
+      for (int oy = warp; oy < Ho; oy += nwarps) {
+        const uint32_t row = src + (uint32_t)(oy * Wo);
+        for (int ox = 2 * lane; ox < Wo; ox += 64) {
+          const bool has_b = ox + 1 < Wo;
+          const float2 q = make_float2(u8f(ldsu8(row + ox)), has_b ? u8f(ldsu8(row + ox + 1)) : 0.f);
+          store_q<DT, VEC>(p, cd, oy, ox, Wo, q, has_b);
+        }
       }
       __syncthreads();
     }
