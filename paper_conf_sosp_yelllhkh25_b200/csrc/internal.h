@@ -76,8 +76,21 @@ struct EpochPlan {
 
 }  // namespace sand
 
+namespace sand {
+// A device + pinned-host buffer pair holding one uploaded epoch plan. Buffers of evicted plans
+// are recycled instead of freed: cudaFree / cudaFreeHost synchronise the device and would stall
+// the stream of read_batch calls at every epoch boundary.
+struct PlanBuffer {
+  void* d = nullptr;
+  void* h = nullptr;
+  size_t bytes = 0;
+  cudaEvent_t done = nullptr;   // recorded after the last kernel that read the buffer
+};
+}  // namespace sand
+
 struct sand_view {
   sand_store* store = nullptr;
+  std::vector<sand::PlanBuffer> pool;   // recycled plan buffers (guarded by mu)
   sand::SpecInfo info;
   sand::ViewConst vconst[sand::kMaxViews];
   std::vector<uint32_t> video_slot;   // dataset index -> unused (dims live in info)

@@ -340,7 +340,6 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
   __syncthreads();
 
   // ------------------------------------------------------------- phase 2: per channel
-  const int n = Ho * Wo;
   const int r = g.blur_on ? g.blur_r : 0;
   const float cxo = (float)(Wo - 1) * 0.5f, cyo = (float)(Ho - 1) * 0.5f;
   for (int c = 0; c < 3; ++c) {

@@ -179,42 +179,78 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
 
 namespace {
 
-void free_plan_device(EpochPlan& p) {
-  if (p.last_use) {
-    cudaEventSynchronize(p.last_use);
+// return a plan's buffers to the view's pool (its kernels finish before the pool hands the
+// buffer out again: the pool waits on the buffer's event, which is long done by then)
+void release_plan_device(sand_view* v, EpochPlan& p) {
+  if (p.d_buf) {
+    PlanBuffer b;
+    b.d = p.d_buf;
+    b.h = p.h_stage;
+    b.bytes = p.d_bytes;
+    b.done = p.last_use;
+    v->pool.push_back(b);
+  } else if (p.last_use) {
     cudaEventDestroy(p.last_use);
-    p.last_use = nullptr;
   }
-  if (p.d_buf) cudaFree(p.d_buf);
-  if (p.h_stage) cudaFreeHost(p.h_stage);
   p.d_buf = p.h_stage = nullptr;
+  p.last_use = nullptr;
   p.uploaded = false;
 }
 
-int upload_plan(EpochPlan& p, cudaStream_t stream) {
+void free_pool(sand_view* v) {
+  for (auto& b : v->pool) {
+    if (b.done) {
+      cudaEventSynchronize(b.done);
+      cudaEventDestroy(b.done);
+    }
+    cudaFree(b.d);
+    cudaFreeHost(b.h);
+  }
+  v->pool.clear();
+}
+
+int upload_plan(sand_view* v, EpochPlan& p, cudaStream_t stream) {
   const size_t gb = p.groups.size() * sizeof(GroupParams);
   const size_t ib = p.items.size() * sizeof(WorkItem);
   const size_t db = p.dests.size() * sizeof(uint32_t);
   const size_t off_i = (gb + 255) / 256 * 256;
   const size_t off_d = off_i + (ib + 255) / 256 * 256;
   const size_t total = std::max<size_t>(off_d + db, 256);
-  cudaError_t e = cudaMalloc(&p.d_buf, total);
-  if (e != cudaSuccess) return cuda_error(e, "cudaMalloc(plan)");
-  e = cudaMallocHost(&p.h_stage, total);
-  if (e != cudaSuccess) return cuda_error(e, "cudaMallocHost(plan)");
-  auto* h = static_cast<uint8_t*>(p.h_stage);
+  // smallest pooled buffer that fits, else a new one with headroom
+  int best = -1;
+  for (size_t i = 0; i < v->pool.size(); ++i)
+    if (v->pool[i].bytes >= total && (best < 0 || v->pool[i].bytes < v->pool[best].bytes)) best = (int)i;
+  PlanBuffer buf;
+  if (best >= 0) {
+    buf = v->pool[best];
+    v->pool.erase(v->pool.begin() + best);
+    if (buf.done) cudaEventSynchronize(buf.done);   // the previous owner's kernels are done
+  } else {
+    buf.bytes = total + total / 4;
+    cudaError_t e = cudaMalloc(&buf.d, buf.bytes);
+    if (e != cudaSuccess) return cuda_error(e, "cudaMalloc(plan)");
+    e = cudaMallocHost(&buf.h, buf.bytes);
+    if (e != cudaSuccess) {
+      cudaFree(buf.d);
+      return cuda_error(e, "cudaMallocHost(plan)");
+    }
+    e = cudaEventCreateWithFlags(&buf.done, cudaEventDisableTiming);
+    if (e != cudaSuccess) return cuda_error(e, "cudaEventCreate");
+  }
+  auto* h = static_cast<uint8_t*>(buf.h);
   if (gb) std::memcpy(h, p.groups.data(), gb);
   if (ib) std::memcpy(h + off_i, p.items.data(), ib);
   if (db) std::memcpy(h + off_d, p.dests.data(), db);
-  e = cudaMemcpyAsync(p.d_buf, p.h_stage, total, cudaMemcpyHostToDevice, stream);
+  cudaError_t e = cudaMemcpyAsync(buf.d, buf.h, total, cudaMemcpyHostToDevice, stream);
   if (e != cudaSuccess) return cuda_error(e, "cudaMemcpyAsync(plan)");
-  e = cudaEventCreateWithFlags(&p.last_use, cudaEventDisableTiming);
-  if (e != cudaSuccess) return cuda_error(e, "cudaEventCreate");
-  auto* d = static_cast<uint8_t*>(p.d_buf);
+  auto* d = static_cast<uint8_t*>(buf.d);
+  p.d_buf = buf.d;
+  p.h_stage = buf.h;
+  p.d_bytes = buf.bytes;
+  p.last_use = buf.done;
   p.d_groups = reinterpret_cast<GroupParams*>(d);
   p.d_items = reinterpret_cast<WorkItem*>(d + off_i);
   p.d_dests = reinterpret_cast<uint32_t*>(d + off_d);
-  p.d_bytes = total;
   p.uploaded = true;
   return SAND_OK;
 }
@@ -247,7 +283,7 @@ std::shared_ptr<EpochPlan> get_plan(sand_view* v, std::unique_lock<std::mutex>& 
     for (auto i = v->plans.begin(); i != v->plans.end(); ++i)
       if (i->second->last_touch < victim->second->last_touch) victim = i;
     if (victim->first == key) break;
-    free_plan_device(*victim->second);
+    release_plan_device(v, *victim->second);
     v->plans.erase(victim);
   }
   v->cv.notify_all();
@@ -392,7 +428,7 @@ extern "C" int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank,
   cudaError_t e = cudaSetDevice(v->store->device);
   if (e != cudaSuccess) return sand::cuda_error(e, "cudaSetDevice");
   if (!plan->uploaded) {
-    int rc = sand::upload_plan(*plan, stream);
+    int rc = sand::upload_plan(v, *plan, stream);
     if (rc != SAND_OK) return rc;
   }
   const uint64_t it = out->iteration;
@@ -544,7 +580,8 @@ extern "C" int sand_view_destroy(sand_view* v) {
   }
   if (v->worker.joinable()) v->worker.join();
   cudaSetDevice(v->store->device);
-  for (auto& kv : v->plans) sand::free_plan_device(*kv.second);
+  for (auto& kv : v->plans) sand::release_plan_device(v, *kv.second);
+  sand::free_pool(v);
   v->store->live_views--;
   delete v;
   return SAND_OK;

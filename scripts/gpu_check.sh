@@ -12,7 +12,7 @@ if [[ " $* " == *" bench "* ]]; then
 fi
 if [[ " $* " == *" ncu "* ]]; then
   for c in ${NCU_CONFIGS:-k400}; do
-    timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 60 --csv --log-file gpurun_out/launches_$c.csv \
+    timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"k_(stream|stencil|resample)" -c 40 --csv --log-file gpurun_out/launches_$c.csv \
       python bench.py --config $c --steps 20 --warmup 3 --no-e2e --no-cpu > /dev/null 2> gpurun_out/ncu_launch_$c.err
     timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_ -s 10 -c 2 -o gpurun_out/prof_$c -f \
       python bench.py --config $c --steps 20 --warmup 3 --no-e2e --no-cpu > /dev/null 2> gpurun_out/ncu_full_$c.err
