@@ -14,5 +14,10 @@ for c in ${NCU_CONFIGS:-k400 slowfast twoview ray}; do
     python bench.py --config $c --steps 30 --warmup 3 --no-e2e --no-cpu > /dev/null 2> gpurun_out/ncu_launch_$c.err
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_(stream|stencil|resample)" -s 6 -c 2 -o gpurun_out/prof_$c -f \
     python bench.py --config $c --steps 12 --warmup 3 --no-e2e --no-cpu > /dev/null 2> gpurun_out/ncu_full_$c.err
+  ncu -i gpurun_out/prof_$c.ncu-rep --page raw --csv > gpurun_out/ncu_raw_$c.csv 2>/dev/null
+  ncu -i gpurun_out/prof_$c.ncu-rep --page details --csv > gpurun_out/ncu_details_$c.csv 2>/dev/null
+  ncu -i gpurun_out/prof_$c.ncu-rep --page source --csv --print-source sass > gpurun_out/ncu_sass_$c.csv 2>/dev/null
+  gzip -f gpurun_out/ncu_sass_$c.csv
+  [ "$c" = "k400" ] || rm -f gpurun_out/prof_$c.ncu-rep
 done
-ls gpurun_out
+du -sh gpurun_out; ls gpurun_out
