@@ -172,6 +172,28 @@ def _oracle_spec(spec):
                                             views=views))
 
 
+def max_over_ranks(values, world, device):
+    """Element-wise max over ranks of a list of floats (the timed region's slowest rank)."""
+    import torch
+    t = torch.tensor(values, dtype=torch.float64, device=device)
+    if world > 1:
+        import torch.distributed as dist
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return [float(x) for x in t.tolist()]
+
+
+def gather_counters(counts, world, device):
+    """All-gather per-rank integer counters and sum them (the only collective of the run)."""
+    import torch
+    mine = torch.tensor(counts, dtype=torch.int64, device=device)
+    if world > 1:
+        import torch.distributed as dist
+        gathered = [torch.zeros_like(mine) for _ in range(world)]
+        dist.all_gather(gathered, mine)
+        return [int(x) for x in torch.stack(gathered).sum(0).tolist()], [g.tolist() for g in gathered]
+    return [int(x) for x in mine.tolist()], [mine.tolist()]
+
+
 def frames_per_step(spec):
     return spec.batch_size * sum(v.clip_len for v in spec.views)
 
@@ -298,22 +320,13 @@ def run_sand(args):
     launches = view.stats().kernel_launches - launches0
     elapsed_ms = start.elapsed_time(end)
     kernel_ms = sum(a.elapsed_time(b) for a, b in zip(kstart, kend)) / args.steps
-    t = torch.tensor([elapsed_ms, kernel_ms], dtype=torch.float64, device=f"cuda:{local}")
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    elapsed_ms, kernel_ms_max = float(t[0]), float(t[1])
+    elapsed_ms, kernel_ms_max = max_over_ranks([elapsed_ms, kernel_ms], world, f"cuda:{local}")
     ms_per_step = elapsed_ms / args.steps
     value = fps * args.steps * world / (elapsed_ms / 1000.0)
 
     # reuse counters: the only collective (NCCL all_gather of a few integers)
     c = store.counters()
-    mine = torch.tensor([c.fetches, c.uses, c.batches], dtype=torch.int64, device=f"cuda:{local}")
-    if world > 1:
-        gathered = [torch.zeros_like(mine) for _ in range(world)]
-        dist.all_gather(gathered, mine)
-        totals = torch.stack(gathered).sum(0).tolist()
-    else:
-        totals = mine.tolist()
+    totals, _ = gather_counters([c.fetches, c.uses, c.batches], world, f"cuda:{local}")
 
     # ---- e2e through the C-ABI with HOST buffers
     e2e = None
@@ -392,12 +405,7 @@ def run_e2e(args, w, spec, view, store, stream, rank, iters, s0, world):
                 ho.copy_(o, non_blocking=True)
     end.record(stream)
     torch.cuda.synchronize()
-    ms = start.elapsed_time(end)
-    import torch.distributed as dist
-    t = torch.tensor([ms], dtype=torch.float64, device=f"cuda:{torch.cuda.current_device()}")
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms = float(t[0])
+    ms = max_over_ranks([start.elapsed_time(end)], world, f"cuda:{torch.cuda.current_device()}")[0]
     return {"value": frames_per_step(spec) * n * world / (ms / 1000.0), "unit": "frames/s",
             "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h), "steps": n,
             "ms_per_step": ms / n}

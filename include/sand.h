@@ -204,6 +204,16 @@ typedef struct {
 int sand_view_batch_bytes(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration,
                           sand_batch_bytes* out);
 
+/* Host-only planning (no store, no device): the same planner read_batch uses.
+ * sand_plan_rank_clips writes the global clip ids of (epoch, rank) in DistributedSampler
+ * order (R#2, R#3) to out[0..*n) (cap entries available); sand_plan_clip plans one clip
+ * (temporal indices, spatial draws; R#4-R#18) given per-dataset-video frame counts and frame
+ * sizes (arrays of spec->n_videos entries). Errors: EINVAL (spec), ERANGE (cap / clip). */
+int sand_plan_rank_clips(const sand_view_spec* spec, uint64_t epoch, uint32_t rank, uint32_t* out, uint32_t cap,
+                         uint32_t* n);
+int sand_plan_clip(const sand_view_spec* spec, const uint32_t* n_frames, const uint32_t* widths,
+                   const uint32_t* heights, uint64_t epoch, uint32_t clip, sand_clip_meta* out);
+
 /* Launch statistics of a view group: kernels launched and batches read so far. */
 typedef struct {
   uint64_t batches, kernel_launches, plans_built, work_items;

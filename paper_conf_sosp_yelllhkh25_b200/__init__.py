@@ -22,7 +22,7 @@ from ._abi import (BF16, F32, GEOM_RRC, GEOM_SHORTSIDE_CROP, MAX_GROUPS, MAX_T, 
                    check, lib)
 from .configs import Spec, ViewSpec, Workload
 
-__all__ = ["Store", "View", "Spec", "ViewSpec", "Workload", "SandError", "lib", "make_spec",
+__all__ = ["Store", "View", "plan_rank_clips", "plan_clip", "Spec", "ViewSpec", "Workload", "SandError", "lib", "make_spec",
            "U8", "BF16", "F32", "GEOM_RRC", "GEOM_SHORTSIDE_CROP"]
 
 _TORCH_DTYPE = None
@@ -61,6 +61,31 @@ def make_spec(spec: Spec, videos) -> tuple[_abi.sand_view_spec, object]:
             o.std[c] = v.std[c]
         o.out_dtype = v.out_dtype
     return s, arr
+
+
+def plan_rank_clips(spec: Spec, videos, epoch: int, rank: int) -> list[int]:
+    """Global clip ids of (epoch, rank) in DistributedSampler order (host-only planner)."""
+    s, keep = make_spec(spec, list(videos))
+    cap = len(videos) * spec.samples_per_video + spec.world_size
+    out = (ctypes.c_uint32 * cap)()
+    n = ctypes.c_uint32()
+    check(lib().sand_plan_rank_clips(ctypes.byref(s), epoch, rank, out, cap, ctypes.byref(n)),
+          "sand_plan_rank_clips")
+    return list(out[: n.value])
+
+
+def plan_clip(spec: Spec, videos, epoch: int, clip: int) -> _abi.sand_clip_meta:
+    """Plan of one clip (frame indices, crop boxes, augmentation draws), host-only.
+
+    videos: list of (video_id, n_frames, width, height) in dataset order."""
+    s, keep = make_spec(spec, [v[0] for v in videos])
+    n = len(videos)
+    F = (ctypes.c_uint32 * n)(*[v[1] for v in videos])
+    W = (ctypes.c_uint32 * n)(*[v[2] for v in videos])
+    H = (ctypes.c_uint32 * n)(*[v[3] for v in videos])
+    out = _abi.sand_clip_meta()
+    check(lib().sand_plan_clip(ctypes.byref(s), F, W, H, epoch, clip, ctypes.byref(out)), "sand_plan_clip")
+    return out
 
 
 class Store:

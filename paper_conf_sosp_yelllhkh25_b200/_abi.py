@@ -102,6 +102,8 @@ SIGNATURES = {
     "sand_last_error": (ctypes.c_char_p, []),
     "sand_version": (ctypes.c_char_p, []),
     "sand_abi_sizes": (ctypes.c_int, [P(u64)]),
+    "sand_plan_rank_clips": (ctypes.c_int, [P(sand_view_spec), u64, u32, P(u32), u32, P(u32)]),
+    "sand_plan_clip": (ctypes.c_int, [P(sand_view_spec), P(u32), P(u32), P(u32), u64, u32, P(sand_clip_meta)]),
 }
 
 STRUCTS = [sand_frame_layout, sand_counters, sand_view_desc, sand_view_spec, sand_tensor_desc,

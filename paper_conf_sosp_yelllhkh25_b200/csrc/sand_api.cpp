@@ -1,6 +1,7 @@
 // sand_api.cpp — error reporting and version of the C-ABI (include/sand.h).
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <string>
 
 #include "internal.h"
@@ -38,4 +39,48 @@ extern "C" int sand_abi_sizes(uint64_t sizes[8]) {
   sizes[6] = sizeof(sand_clip_meta);
   sizes[7] = sizeof(sand_batch_bytes);
   return 8;
+}
+
+namespace {
+int host_spec(const sand_view_spec* spec, const uint32_t* n_frames, const uint32_t* widths, const uint32_t* heights,
+              sand::SpecInfo* info) {
+  if (!spec) return sand::set_error(SAND_EINVAL, "null spec");
+  std::string why;
+  const int rc = sand::validate_spec(*spec, &why);
+  if (rc != SAND_OK) return sand::set_error(rc, why);
+  info->spec = *spec;
+  info->videos.assign(spec->videos, spec->videos + spec->n_videos);
+  info->spec.videos = info->videos.data();
+  for (uint32_t i = 0; i < spec->n_videos; ++i)
+    info->dims.push_back({spec->videos[i], n_frames ? n_frames[i] : 1u, widths ? widths[i] : 2u,
+                          heights ? heights[i] : 2u});
+  sand::derive_spec(info);
+  return SAND_OK;
+}
+}  // namespace
+
+extern "C" int sand_plan_rank_clips(const sand_view_spec* spec, uint64_t epoch, uint32_t rank, uint32_t* out,
+                                    uint32_t cap, uint32_t* n) {
+  if (!out || !n) return sand::set_error(SAND_EINVAL, "null argument");
+  sand::SpecInfo info;
+  const int rc = host_spec(spec, nullptr, nullptr, nullptr, &info);
+  if (rc != SAND_OK) return rc;
+  if (rank >= spec->world_size) return sand::set_error(SAND_EINVAL, "rank >= world_size");
+  const std::vector<uint32_t> clips = sand::rank_clips(info, epoch, rank);
+  if (clips.size() > cap) return sand::set_error(SAND_ERANGE, "output capacity too small");
+  std::copy(clips.begin(), clips.end(), out);
+  *n = static_cast<uint32_t>(clips.size());
+  return SAND_OK;
+}
+
+extern "C" int sand_plan_clip(const sand_view_spec* spec, const uint32_t* n_frames, const uint32_t* widths,
+                              const uint32_t* heights, uint64_t epoch, uint32_t clip, sand_clip_meta* out) {
+  if (!out || !n_frames || !widths || !heights) return sand::set_error(SAND_EINVAL, "null argument");
+  sand::SpecInfo info;
+  const int rc = host_spec(spec, n_frames, widths, heights, &info);
+  if (rc != SAND_OK) return rc;
+  if (static_cast<uint64_t>(clip) >= static_cast<uint64_t>(spec->n_videos) * spec->samples_per_video)
+    return sand::set_error(SAND_ERANGE, "clip id out of range");
+  sand::plan_clip(info, epoch, clip, out);
+  return SAND_OK;
 }

@@ -1,0 +1,75 @@
+"""CPU parity of the product's host planner (libsand.so, no device) against the oracle.
+
+The plan (clip order per rank, frame indices, crop boxes, flip/rotation/blur draws) is the
+integer/double part of the path (§8(a) rows a1-a3); it must be BIT-EXACT (north_star). These
+tests call the host-only C-ABI entry points sand_plan_rank_clips / sand_plan_clip, which share
+the planner read_batch uses; the GPU tests check the same through sand_view_get_meta.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_sosp_yelllhkh25_b200 as sand
+from paper_conf_sosp_yelllhkh25_b200 import configs
+
+from helpers import meta_fields, to_oracle, videos_of
+
+
+@pytest.mark.parametrize("name", ["tiny", "k400", "slowfast", "twoview", "ray"])
+def test_host_plan_matches_oracle_bit_exact(name):
+    w = configs.get(name)
+    vids = videos_of(w, min(w.n_videos, 64))
+    ospec = to_oracle(w.spec)
+    ods = oracle.make_dataset(vids)
+    rng = np.random.default_rng(3)
+    n = len(vids) * w.spec.samples_per_video
+    for epoch in (0, 1, 7, 2**33 + 5):
+        for clip in rng.choice(n, size=min(n, 24), replace=False):
+            got = sand.plan_clip(w.spec, vids, epoch, int(clip))
+            ref = oracle.ClipMeta()
+            oracle.lib().oracle_plan_clip(oracle.ctypes.byref(ospec), ods, epoch, int(clip), oracle.ctypes.byref(ref))
+            assert meta_fields(w.spec, got) == meta_fields(w.spec, ref), (name, epoch, clip)
+
+
+@pytest.mark.parametrize("n_videos,world,drop_last,S", [(64, 1, False, 1), (64, 8, False, 1), (70, 8, False, 1),
+                                                       (70, 8, True, 1), (5, 8, False, 1), (33, 4, False, 2)])
+def test_rank_clips_match_oracle_partition(n_videos, world, drop_last, S):
+    spec = configs.k400().spec
+    spec.world_size, spec.drop_last, spec.samples_per_video = world, drop_last, S
+    vids = [1000 + i for i in range(n_videos)]
+    for epoch in (0, 3):
+        perm = oracle.permutation(n_videos * S, spec.seed, epoch)
+        for r in range(world):
+            assert sand.plan_rank_clips(spec, vids, epoch, r) == oracle.partition(perm, world, r, drop_last).tolist()
+
+
+def test_samples_per_video_and_shared_window_plans():
+    w = configs.ray()
+    w.spec.samples_per_video = 2
+    vids = videos_of(w, 8)
+    ospec = to_oracle(w.spec)
+    ods = oracle.make_dataset(vids)
+    for clip in range(16):
+        got = sand.plan_clip(w.spec, vids, 4, clip)
+        ref = oracle.ClipMeta()
+        oracle.lib().oracle_plan_clip(oracle.ctypes.byref(ospec), ods, 4, clip, oracle.ctypes.byref(ref))
+        assert meta_fields(w.spec, got) == meta_fields(w.spec, ref)
+        assert got.sample == clip % 2
+
+
+def test_invalid_specs_rejected_on_host():
+    w = configs.tiny()
+    vids = videos_of(w)
+    bad = configs.tiny().spec
+    bad.views[0].blur_ksize = 22
+    with pytest.raises(sand.SandError):
+        sand.plan_clip(bad, vids, 0, 0)
+    bad = configs.tiny().spec
+    bad.views[0].clip_len = 0
+    with pytest.raises(sand.SandError):
+        sand.plan_rank_clips(bad, [1000], 0, 0)
+    two = configs.twoview().spec
+    two.views[1].rot_max_deg = 3.0
+    two.views[1].spatial_group = 0           # same group, different augmentation -> invalid
+    with pytest.raises(sand.SandError):
+        sand.plan_clip(two, videos_of(configs.twoview(), 4), 0, 0)
