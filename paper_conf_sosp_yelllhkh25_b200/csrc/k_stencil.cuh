@@ -276,7 +276,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
     int y_hi;
     tap(g.sc_y, g.off_y, oy_lo + nr - 1, g.lim_y, g.org_y, dmy, y_hi, fl);
     __syncthreads();                          // previous band's walkers are done with the grid
-    st::stage_rows(s_rawb, Yp, UVp, w.pitch, x16, gw, y_lo, y_hi, tid, nthr);
+    st::stage_rows(s_rawb, Yp + x16, UVp + x16, w.pitch, gw, y_lo, y_hi, warp, nwarps, lane);
     for (int r = tid; r < nr; r += nthr) {
       int y0, y1;
       float ly;

@@ -55,15 +55,17 @@ __device__ __forceinline__ void cp_async16s(uint32_t s, const void* gmem) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
 }
 
-// Y rows [ya, yb] then UV rows [ya>>1, yb>>1] -> raw (shared address), gw bytes from column x16
-__device__ __forceinline__ void stage_rows(uint32_t raw, const uint8_t* Yp, const uint8_t* UVp, uint32_t pitch,
-                                           int x16, int gw, int ya, int yb, int tid, int nthr) {
+// Y rows [ya, yb] then UV rows [ya>>1, yb>>1] -> raw (shared address), gw bytes per row.
+// y0/uv0: global addresses of column x16 of Y row 0 / UV row 0 (loop-invariant, computed once
+// per CTA). Warps take rows, lanes take 16 B chunks (gw <= 512 B: one request per lane).
+__device__ __forceinline__ void stage_rows(uint32_t raw, const uint8_t* y0, const uint8_t* uv0, uint32_t pitch,
+                                           int gw, int ya, int yb, int warp, int nwarps, int lane) {
   const int ny = yb - ya + 1, u0 = ya >> 1, nuv = (yb >> 1) - u0 + 1;
   const int chunks = gw >> 4;
-  const int warp = tid >> 5, lane = tid & 31, nwarps = nthr >> 5;
-  for (int r = warp; r < ny + nuv; r += nwarps) {   // warps over rows, lanes over 16 B chunks
-    const uint8_t* src = (r < ny ? Yp + (size_t)(ya + r) * pitch : UVp + (size_t)(u0 + r - ny) * pitch) + x16;
+  for (int r = warp; r < ny + nuv; r += nwarps) {
+    const uint8_t* src = r < ny ? y0 + (size_t)(ya + r) * pitch : uv0 + (size_t)(u0 + r - ny) * pitch;
     const uint32_t dst = raw + (uint32_t)(r * gw);
+#pragma unroll 1
     for (int k = lane; k < chunks; k += 32) cp_async16s(dst + 16u * k, src + 16 * k);
   }
   asm volatile("cp.async.commit_group;\n" ::: "memory");
@@ -85,11 +87,12 @@ __device__ __forceinline__ Chroma3 chroma_at(uint32_t uv) {
 // PRMT gathers the three bytes and the exponent byte 0x4B tops the word (see rs::biased).
 __device__ __forceinline__ uint32_t rgbx_dpx(uint32_t Y, const Chroma3& c) {
   const int yy = (int)max(Y, 16u) * 1220542 + ((1 << 19) - 16 * 1220542);
-  const int mr = min(__viaddmax_s32(yy, c.r, 0), 0x0FFFFFFF) >> 4;
-  const int mg = min(__viaddmax_s32(yy, c.g, 0), 0x0FFFFFFF) >> 4;
-  const int mb = min(__viaddmax_s32(yy, c.b, 0), 0x0FFFFFFF) >> 4;
-  const uint32_t rg = __byte_perm((uint32_t)mr, (uint32_t)mg, 0x0062);
-  return __byte_perm(rg, (uint32_t)mb, 0x7610) | 0x4B000000u;
+  // x >> 4 of the clamped (non-negative) sums as IMAD.HI (FMA pipe) to relieve the ALU pipe
+  const uint32_t mr = __umulhi((uint32_t)min(__viaddmax_s32(yy, c.r, 0), 0x0FFFFFFF), 1u << 28);
+  const uint32_t mg = __umulhi((uint32_t)min(__viaddmax_s32(yy, c.g, 0), 0x0FFFFFFF), 1u << 28);
+  const uint32_t mb = __umulhi((uint32_t)min(__viaddmax_s32(yy, c.b, 0), 0x0FFFFFFF), 1u << 28);
+  const uint32_t rg = __byte_perm(mr, mg, 0x0062);
+  return __byte_perm(rg, mb, 0x7610) + 0x4B000000u;   // byte 3 is zero: add == or
 }
 
 // convert staged rows [ya, yb] into the ring (slot = (y - y_first) % ring_rows)
@@ -172,8 +175,9 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
   const int gw = ((x_hi + 16) & ~15) - x16;
   const uint32_t rowbytes = (uint32_t)gw * 4u;
   const int y_first = tap0(g.sc_y, g.off_y, Y0, g.org_y);
-  const uint8_t* Yp = p.slab + w.y_off;
-  const uint8_t* UVp = Yp + (size_t)w.pitch * w.src_h;
+  const uint8_t* Yx = p.slab + w.y_off + x16;                // column x16 of Y row 0
+  const uint8_t* UVx = Yx + (size_t)w.pitch * w.src_h;       // column x16 of UV row 0
+  const uint32_t pitch = w.pitch;
 
   // sub-band k covers output rows [k*S, min((k+1)*S, nr)); it adds source rows
   // (y1(last row of k-1), y1(last row of k)]
@@ -185,7 +189,7 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
   };
   const int nsub = (nr + sh.S - 1) / sh.S;
   int ya = y_first, yb = last_src(0);
-  st::stage_rows(s_raw, Yp, UVp, w.pitch, x16, gw, ya, yb, tid, nthr);
+  st::stage_rows(s_raw, Yx, UVx, pitch, gw, ya, yb, warp, nwarps, lane);
 
   // tap tables (overlap the first copy): columns (x0, x1, lambda); rows (byte offsets of
   // the two ring rows, y0, lambda)
@@ -225,7 +229,7 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
     if (k + 1 < nsub) {                              // stage the next sub-band's new rows
       const int na = yb + 1, nb = last_src(k + 1);
       if (nb >= na)
-        st::stage_rows(s_raw + (uint32_t)((k + 1) & 1) * rawcap, Yp, UVp, w.pitch, x16, gw, na, nb, tid, nthr);
+        st::stage_rows(s_raw + (uint32_t)((k + 1) & 1) * rawcap, Yx, UVx, pitch, gw, na, nb, warp, nwarps, lane);
       ya = na;
       yb = max(nb, yb);
     }
