@@ -139,6 +139,11 @@ __device__ __forceinline__ void hrow_s(rs::Row3& r, uint32_t rowaddr, uint32_t c
   r.h[2] = rs::hlerp<2>(a0, a1, b0, b1, lx);
 }
 
+// row actions of the walker (computed once per row by the table builder)
+constexpr uint32_t kActShift = 1;   // y0 = previous y0 + 1: the old bottom row is the new top
+constexpr uint32_t kActJump = 2;    // new y0 (first row or a step > 1): compute both rows
+constexpr uint32_t kActClamp = 4;   // y1 == y0 (bottom edge): bottom = top
+
 }  // namespace st
 
 template <int DT, bool VEC>
@@ -204,13 +209,21 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
     float ly;
     tap(g.sc_y, g.off_y, Y0 + r, g.lim_y, g.org_y, y0, y1, ly);
     const uint32_t s0 = (uint32_t)((y0 - y_first) % sh.ring), s1 = (uint32_t)((y1 - y_first) % sh.ring);
-    rtab[r] = make_uint4(s0 * rowbytes, s1 * rowbytes, (uint32_t)y0, __float_as_uint(ly));
+    // action relative to the previous output row of the super-band
+    uint32_t act = st::kActJump;
+    if (r > 0) {
+      const int yp = tap0(g.sc_y, g.off_y, Y0 + r - 1, g.org_y);
+      act = y0 == yp ? 0u : (y0 == yp + 1 ? st::kActShift : st::kActJump);
+    }
+    if (y1 == y0) act |= st::kActClamp;
+    rtab[r] = make_uint4(s0 * rowbytes, s1 * rowbytes, act, __float_as_uint(ly));
   }
 
-  // per-thread walker state: output columns (ox, ox+1) for the whole super-band
+  // per-thread walker state: output columns (ox, ox+1) for the whole super-band. Every lane
+  // walks (lanes past the last pair repeat it without storing), so warps stay converged.
   const int pairs = (Wo + 1) >> 1;
-  const bool walker = tid < pairs;
-  const int ox = 2 * tid;
+  const bool valid = tid < pairs;
+  const int ox = 2 * min(tid, pairs - 1);
   const bool has_b = ox + 1 < Wo;
   const bool vec = has_b && !(Wo & 1);
   uint32_t ca0 = 0, ca1 = 0, cb0 = 0, cb1 = 0;
@@ -219,8 +232,11 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
   const uint32_t* dests = p.dests + w.dest_begin;
   Dest dl[kInlineDests];
   int dt[kInlineDests];
-  int have0 = -1, have1 = -1;
-  Row3 S0, S1;
+  // Two register sets X, Y hold the horizontal lerps of source rows y0 and y0 + 1; `top`
+  // says which one is y0. A shift by one source row flips `top` and recomputes only the other
+  // set, so no register copies are needed between rows.
+  Row3 X, Y;
+  int top = 0;
 
   for (int k = 0; k < nsub; ++k) {
     asm volatile("cp.async.wait_group 0;\n" ::: "memory");
@@ -234,7 +250,6 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
       yb = max(nb, yb);
     }
     __syncthreads();                                 // ring holds every row of sub-band k
-    if (!walker) continue;
     if (k == 0) {                                    // tables are visible now
       const int ja = g.flip ? Wo - 1 - ox : ox;
       const int jb = has_b ? (g.flip ? Wo - 2 - ox : ox + 1) : ja;
@@ -254,27 +269,32 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
     const int r_lo = k * sh.S, r_hi = min(r_lo + sh.S, nr);
     for (int rr = r_lo; rr < r_hi; ++rr) {
       const uint4 rt = st::lds128(s_rtab + 16u * rr);
-      const uint32_t o0 = s_ring + rt.x, o1 = s_ring + rt.y;
-      const int y0 = (int)rt.z;
+      const uint32_t act = rt.z;
       const float l = __uint_as_float(rt.w);
-      const int oy = Y0 + rr;
-      // parity slots: rows y0 and y0+1 are held in different register sets (R#12 taps)
-      if (y0 & 1) {
-        if (have1 != y0) { st::hrow_s(S1, o0, ca0, ca1, cb0, cb1, lx); have1 = y0; }
-        if (o1 != o0) {
-          if (have0 != y0 + 1) { st::hrow_s(S0, o1, ca0, ca1, cb0, cb1, lx); have0 = y0 + 1; }
-          emit<DT, kInlineDests, VEC>(S1, S0, l, dl, dt, p, dests, nd, oy, ox, vec, has_b);
-        } else {
-          emit<DT, kInlineDests, VEC>(S1, S1, l, dl, dt, p, dests, nd, oy, ox, vec, has_b);
+      if (top == 0) {
+        if (act & st::kActJump) {
+          st::hrow_s(X, s_ring + rt.x, ca0, ca1, cb0, cb1, lx);
+          if (act & st::kActClamp) Y = X;                // bottom edge: y1 == y0 (rare)
+          else st::hrow_s(Y, s_ring + rt.y, ca0, ca1, cb0, cb1, lx);
+        } else if (act & st::kActShift) {
+          top = 1;                                      // Y is the new top; X the new bottom
+          if (act & st::kActClamp) X = Y;
+          else st::hrow_s(X, s_ring + rt.y, ca0, ca1, cb0, cb1, lx);
         }
       } else {
-        if (have0 != y0) { st::hrow_s(S0, o0, ca0, ca1, cb0, cb1, lx); have0 = y0; }
-        if (o1 != o0) {
-          if (have1 != y0 + 1) { st::hrow_s(S1, o1, ca0, ca1, cb0, cb1, lx); have1 = y0 + 1; }
-          emit<DT, kInlineDests, VEC>(S0, S1, l, dl, dt, p, dests, nd, oy, ox, vec, has_b);
-        } else {
-          emit<DT, kInlineDests, VEC>(S0, S0, l, dl, dt, p, dests, nd, oy, ox, vec, has_b);
+        if (act & st::kActJump) {
+          st::hrow_s(Y, s_ring + rt.x, ca0, ca1, cb0, cb1, lx);
+          if (act & st::kActClamp) X = Y;
+          else st::hrow_s(X, s_ring + rt.y, ca0, ca1, cb0, cb1, lx);
+        } else if (act & st::kActShift) {
+          top = 0;
+          if (act & st::kActClamp) Y = X;
+          else st::hrow_s(Y, s_ring + rt.y, ca0, ca1, cb0, cb1, lx);
         }
+      }
+      if (valid) {
+        if (top == 0) emit<DT, kInlineDests, VEC>(X, Y, l, dl, dt, p, dests, nd, Y0 + rr, ox, vec, has_b);
+        else emit<DT, kInlineDests, VEC>(Y, X, l, dl, dt, p, dests, nd, Y0 + rr, ox, vec, has_b);
       }
     }
   }
