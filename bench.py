@@ -298,7 +298,8 @@ def run_sand(args):
     kend = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
     start = torch.cuda.Event(enable_timing=True)
     end = torch.cuda.Event(enable_timing=True)
-    launches0 = view.stats().kernel_launches
+    st0 = view.stats()
+    launches0 = st0.kernel_launches
     clocks = ClockSampler(local)
     clocks.start()
     time.sleep(0.2)
@@ -317,7 +318,13 @@ def run_sand(args):
     if world > 1:
         dist.barrier()
     clk = clocks.stop()
-    launches = view.stats().kernel_launches - launches0
+    st1 = view.stats()
+    launches = st1.kernel_launches - launches0
+    host = {"read_batch_us": (st1.read_ns - st0.read_ns) / 1e3 / args.steps,
+            "plan_wait_us": (st1.plan_wait_ns - st0.plan_wait_ns) / 1e3 / args.steps,
+            "plans_built": int(st1.plans_built - st0.plans_built),
+            "plan_build_ms_each": ((st1.plan_build_ns - st0.plan_build_ns) / 1e6 /
+                                   max(1, st1.plans_built - st0.plans_built))}
     elapsed_ms = start.elapsed_time(end)
     kernel_ms = sum(a.elapsed_time(b) for a, b in zip(kstart, kend)) / args.steps
     elapsed_ms, kernel_ms_max = max_over_ranks([elapsed_ms, kernel_ms], world, f"cuda:{local}")
@@ -348,6 +355,7 @@ def run_sand(args):
                      "kernel_ms_per_step": kernel_ms, "peak_source": peak_src,
                      "frac_of_8tbs_spec": achieved / 8000.0},
         "gpu_launches": int(launches),
+        "host": host,
         "clocks": clk,
         "reuse": {"fetches": totals[0], "uses": totals[1], "batches": totals[2]},
     }

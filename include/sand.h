@@ -214,9 +214,12 @@ int sand_plan_rank_clips(const sand_view_spec* spec, uint64_t epoch, uint32_t ra
 int sand_plan_clip(const sand_view_spec* spec, const uint32_t* n_frames, const uint32_t* widths,
                    const uint32_t* heights, uint64_t epoch, uint32_t clip, sand_clip_meta* out);
 
-/* Launch statistics of a view group: kernels launched and batches read so far. */
+/* Statistics of a view group: batches read, kernels launched, epoch plans built and work
+ * items launched so far; host time spent building plans (all builder threads), blocked in
+ * read_batch waiting for a plan, and inside read_batch in total (nanoseconds). */
 typedef struct {
   uint64_t batches, kernel_launches, plans_built, work_items;
+  uint64_t plan_build_ns, plan_wait_ns, read_ns;
 } sand_view_stats;
 int sand_view_get_stats(const sand_view* v, sand_view_stats* out);
 

@@ -145,6 +145,9 @@ class View:
         self._h = ctypes.c_void_p()
         check(lib().sand_view_create(store.handle, ctypes.byref(self._spec_c), ctypes.byref(self._h)),
               "sand_view_create")
+        self._out = _abi.sand_batch_out()   # reused by read_batch: one View per Python thread
+        self._out_ref = ctypes.byref(self._out)
+        self._read = lib().sand_view_read_batch
 
     def output_desc(self, k: int) -> _abi.sand_tensor_desc:
         d = _abi.sand_tensor_desc()
@@ -166,7 +169,7 @@ class View:
         return n.value
 
     def read_batch(self, epoch: int, rank: int, iteration: int, outs, stream: int | None = None) -> None:
-        o = _abi.sand_batch_out()
+        o = self._out
         o.iteration = iteration
         if stream is None:
             import torch
@@ -174,7 +177,9 @@ class View:
         o.stream = stream
         for k, t in enumerate(outs):
             o.data[k] = t.data_ptr() if hasattr(t, "data_ptr") else int(t)
-        check(lib().sand_view_read_batch(self._h, epoch, rank, ctypes.byref(o)), "sand_view_read_batch")
+        rc = self._read(self._h, epoch, rank, self._out_ref)
+        if rc:
+            check(rc, "sand_view_read_batch")
 
     def prefetch_epoch(self, epoch: int, rank: int = 0) -> None:
         check(lib().sand_view_prefetch_epoch(self._h, epoch, rank), "sand_view_prefetch_epoch")

@@ -77,7 +77,8 @@ class sand_batch_bytes(ctypes.Structure):
 
 
 class sand_view_stats(ctypes.Structure):
-    _fields_ = [("batches", u64), ("kernel_launches", u64), ("plans_built", u64), ("work_items", u64)]
+    _fields_ = [("batches", u64), ("kernel_launches", u64), ("plans_built", u64), ("work_items", u64),
+                ("plan_build_ns", u64), ("plan_wait_ns", u64), ("read_ns", u64)]
 
 
 P = ctypes.POINTER

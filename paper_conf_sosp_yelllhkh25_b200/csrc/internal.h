@@ -62,6 +62,7 @@ struct EpochPlan {
   std::vector<uint32_t> fetch_begin;          // iterations + 1
   std::vector<std::pair<uint32_t, uint32_t>> fetch_keys;   // (video, frame)
   std::vector<uint32_t> fetch_uses;
+  std::vector<VideoEntry*> fetch_entry;       // store entry of each fetch key (stable: never erased)
   // device copy
   void* d_buf = nullptr;
   void* h_stage = nullptr;
@@ -70,7 +71,9 @@ struct EpochPlan {
   WorkItem* d_items = nullptr;
   uint32_t* d_dests = nullptr;
   bool uploaded = false;
-  cudaEvent_t last_use = nullptr;
+  cudaEvent_t last_use = nullptr;              // recorded after every kernel that reads the buffer
+  cudaEvent_t ready = nullptr;                 // upload complete (recorded on the view's upload stream)
+  cudaStream_t ready_waited = nullptr;         // last caller stream made to wait on `ready`
   uint64_t last_touch = 0;
 };
 
@@ -84,7 +87,8 @@ struct PlanBuffer {
   void* d = nullptr;
   void* h = nullptr;
   size_t bytes = 0;
-  cudaEvent_t done = nullptr;   // recorded after the last kernel that read the buffer
+  cudaEvent_t done = nullptr;    // recorded after the last kernel that read the buffer
+  cudaEvent_t ready = nullptr;   // recorded after the upload that wrote it
 };
 }  // namespace sand
 
@@ -100,17 +104,24 @@ struct sand_view {
   std::map<std::pair<uint64_t, uint32_t>, std::shared_ptr<sand::EpochPlan>> plans;
   std::map<std::pair<uint64_t, uint32_t>, bool> pending;   // being built by the worker
   std::deque<std::pair<uint64_t, uint32_t>> queue;
-  std::thread worker;
+  std::vector<std::thread> workers;     // plan builders (pre-materialisation threads)
+  cudaStream_t upload_stream = nullptr;  // plan uploads (H2D), ordered before use by events
+  std::vector<sand::VideoEntry*> entries;   // dataset index -> store entry (immutable geometry)
+  std::vector<std::shared_ptr<sand::EpochPlan>> spare_plans;   // evicted plans, recycled by builders
   bool stop = false;
   uint64_t touch = 0;
   // stats
   uint64_t batches = 0, launches = 0, plans_built = 0, work_items = 0;
+  uint64_t plan_build_ns = 0, plan_wait_ns = 0, read_ns = 0;
   size_t stencil_smem = 0;   // dynamic smem of the stencil path (0 if no view rotates/blurs)
 };
 
 namespace sand {
 
-std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32_t rank);
+// Build the epoch plan of (epoch, rank) into `reuse` (a recycled plan whose device copy was
+// released) or a new plan.
+std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32_t rank,
+                                      std::shared_ptr<EpochPlan> reuse = nullptr);
 
 // kernels (materialize.cu)
 size_t stencil_smem_bytes(int max_h, int max_w, int max_r);

@@ -102,21 +102,52 @@ __device__ __forceinline__ float biased(uint32_t w) {
   return __uint_as_float(r);
 }
 
+// Packed fp32 pairs as 64-bit values (PTX f32x2 ops, sm_100a FFMA2/FADD2): the 64-bit type
+// keeps each pair in an aligned register pair, so no MOVs are needed to feed the packed units.
+// .rn ops are never contracted, so every op rounds exactly as the scalar R#12 sequence.
+namespace f2 {
+__device__ __forceinline__ uint64_t fma(uint64_t a, uint64_t b, uint64_t c) {
+  uint64_t d;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
+  return d;
+}
+__device__ __forceinline__ uint64_t add(uint64_t a, uint64_t b) {
+  uint64_t d;
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+__device__ __forceinline__ uint64_t pack(uint32_t lo, uint32_t hi) {
+  uint64_t d;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(d) : "r"(lo), "r"(hi));
+  return d;
+}
+__device__ __forceinline__ uint64_t pack(float lo, float hi) { return pack(__float_as_uint(lo), __float_as_uint(hi)); }
+__device__ __forceinline__ uint64_t splat(float x) { return pack(x, x); }
+__device__ __forceinline__ uint32_t lo(uint64_t v) { return (uint32_t)v; }
+__device__ __forceinline__ uint32_t hi(uint64_t v) { return (uint32_t)(v >> 32); }
+__device__ __forceinline__ float lof(uint64_t v) { return __uint_as_float(lo(v)); }
+__device__ __forceinline__ float hif(uint64_t v) { return __uint_as_float(hi(v)); }
+}  // namespace f2
+
 struct Row3 {
-  float2 h[3];   // horizontal lerps of (column a, column b) per channel
+  uint64_t h[3];   // horizontal lerps of (column a, column b) per channel, packed fp32 pairs
 };
 
 template <int C>
-__device__ __forceinline__ float2 hlerp(uint32_t a0, uint32_t a1, uint32_t b0, uint32_t b1, float2 lx) {
-  const float2 P0 = make_float2(biased<C>(a0), biased<C>(b0));
-  const float2 P1 = make_float2(biased<C>(a1), biased<C>(b1));
-  const float2 d = __ffma2_rn(P0, make_float2(-1.f, -1.f), P1);          // p1 - p0 (exact)
-  const float2 p0 = __fadd2_rn(P0, make_float2(-kBias, -kBias));          // p0 (exact)
-  return __ffma2_rn(lx, d, p0);                                           // fmaf(l, p1 - p0, p0)
+__device__ __forceinline__ uint64_t hlerp(uint32_t a0, uint32_t a1, uint32_t b0, uint32_t b1, uint64_t lx) {
+  const uint64_t P0 = f2::pack(__float_as_uint(biased<C>(a0)), __float_as_uint(biased<C>(b0)));
+  const uint64_t P1 = f2::pack(__float_as_uint(biased<C>(a1)), __float_as_uint(biased<C>(b1)));
+  const uint64_t d = f2::fma(P0, f2::splat(-1.f), P1);     // p1 - p0 (exact)
+  const uint64_t p0 = f2::add(P0, f2::splat(-kBias));      // p0 (exact)
+  return f2::fma(lx, d, p0);                               // fmaf(l, p1 - p0, p0)
 }
 
+// rint of a packed pair of values in [0, 256) as 1.5*2^23 + q (RNE); the low byte of each
+// word is q
+__device__ __forceinline__ uint64_t rint_biased(uint64_t v) { return f2::add(v, f2::splat(kRound)); }
+
 __device__ __forceinline__ void hrow(Row3& r, const uint32_t* __restrict__ grow, uint32_t ca, uint32_t cb,
-                                     float2 lx) {
+                                     uint64_t lx) {
   const uint32_t a0 = grow[ca & 0xffffu], a1 = grow[ca >> 16];
   const uint32_t b0 = grow[cb & 0xffffu], b1 = grow[cb >> 16];
   r.h[0] = hlerp<0>(a0, a1, b0, b1, lx);
@@ -157,35 +188,38 @@ __device__ __forceinline__ Dest make_dest(const LaunchParams& p, uint32_t dest, 
   return d;
 }
 
-// store quantised pair q of channel c; DT < 0: dtype read at run time
+// store quantised pair of channel c: q holds the integers 0..255 as floats, tq the same as
+// 1.5*2^23 + q (low byte = q); DT < 0: dtype read at run time
 template <int DT, bool VEC>
-__device__ __forceinline__ void put(const Dest& d, int dtype, int c, float2 q, bool vec_rt, bool has_b) {
+__device__ __forceinline__ void put(const Dest& d, int dtype, int c, uint64_t q, uint64_t tq, bool vec_rt, bool has_b) {
   const bool vec = VEC || vec_rt;
-  // q holds integers 0..255; y = fmaf(q, a_c, b_c) per element (R#17)
   const int dt = DT >= 0 ? DT : dtype;
   uint8_t* o = d.row + (size_t)c * d.cstride;
-  if (dt == SAND_BF16) {
-    const float2 y = __ffma2_rn(q, make_float2(d.a[c], d.a[c]), make_float2(d.b[c], d.b[c]));
+  if (dt == SAND_U8) {
+    const uint32_t pair = __byte_perm(f2::lo(tq), f2::hi(tq), 0x0040);
     if (vec) {
-      *reinterpret_cast<__nv_bfloat162*>(o) = __floats2bfloat162_rn(y.x, y.y);
+      *reinterpret_cast<uint16_t*>(o) = (uint16_t)pair;
     } else {
-      reinterpret_cast<__nv_bfloat16*>(o)[0] = __float2bfloat16_rn(y.x);
-      if (has_b) reinterpret_cast<__nv_bfloat16*>(o)[1] = __float2bfloat16_rn(y.y);
+      o[0] = (uint8_t)pair;
+      if (has_b) o[1] = (uint8_t)(pair >> 8);
     }
-  } else if (dt == SAND_F32) {
-    const float2 y = __ffma2_rn(q, make_float2(d.a[c], d.a[c]), make_float2(d.b[c], d.b[c]));
+    return;
+  }
+  // y = fmaf(q, a_c, b_c) per element (R#17)
+  const uint64_t y = f2::fma(q, f2::splat(d.a[c]), f2::splat(d.b[c]));
+  if (dt == SAND_BF16) {
     if (vec) {
-      *reinterpret_cast<float2*>(o) = y;
+      *reinterpret_cast<__nv_bfloat162*>(o) = __floats2bfloat162_rn(f2::lof(y), f2::hif(y));
     } else {
-      reinterpret_cast<float*>(o)[0] = y.x;
-      if (has_b) reinterpret_cast<float*>(o)[1] = y.y;
+      reinterpret_cast<__nv_bfloat16*>(o)[0] = __float2bfloat16_rn(f2::lof(y));
+      if (has_b) reinterpret_cast<__nv_bfloat16*>(o)[1] = __float2bfloat16_rn(f2::hif(y));
     }
   } else {
     if (vec) {
-      *reinterpret_cast<uint16_t*>(o) = (uint16_t)((uint32_t)q.x | ((uint32_t)q.y << 8));
+      *reinterpret_cast<uint64_t*>(o) = y;
     } else {
-      o[0] = (uint8_t)q.x;
-      if (has_b) o[1] = (uint8_t)q.y;
+      reinterpret_cast<float*>(o)[0] = f2::lof(y);
+      if (has_b) reinterpret_cast<float*>(o)[1] = f2::hif(y);
     }
   }
 }
@@ -196,20 +230,19 @@ template <int DT, int ND, bool VEC>
 __device__ __forceinline__ void emit(const Row3& top, const Row3& bot, float l, Dest (&dl)[ND], const int (&dt)[ND],
                                      const LaunchParams& p, const uint32_t* __restrict__ dests, int nd, int oy,
                                      int ox, bool vec, bool has_b) {
-  const float2 ly = make_float2(l, l);
-  float2 q[3];
+  const uint64_t ly = f2::splat(l);
+  uint64_t q[3], tq[3];
 #pragma unroll
   for (int c = 0; c < 3; ++c) {
-    const float2 dv = __ffma2_rn(top.h[c], make_float2(-1.f, -1.f), bot.h[c]);   // h1 - h0
-    const float2 v = __ffma2_rn(ly, dv, top.h[c]);                               // fmaf(ly, h1-h0, h0)
-    const float2 tq = __fadd2_rn(v, make_float2(kRound, kRound));                // rint (RNE)
-    q[c] = __fadd2_rn(tq, make_float2(-kRound, -kRound));
+    const uint64_t dv = f2::fma(top.h[c], f2::splat(-1.f), bot.h[c]);   // h1 - h0
+    tq[c] = rint_biased(f2::fma(ly, dv, top.h[c]));                     // rint(fmaf(ly, h1-h0, h0))
+    q[c] = DT == SAND_U8 ? tq[c] : f2::add(tq[c], f2::splat(-kRound));
   }
 #pragma unroll
   for (int d = 0; d < ND; ++d) {
     if (d == 0 || d < nd) {
 #pragma unroll
-      for (int c = 0; c < 3; ++c) put<DT, VEC>(dl[d], dt[d], c, q[c], vec, has_b);
+      for (int c = 0; c < 3; ++c) put<DT, VEC>(dl[d], dt[d], c, q[c], tq[c], vec, has_b);
       dl[d].row += dl[d].rstride;
     }
   }
@@ -217,7 +250,7 @@ __device__ __forceinline__ void emit(const Row3& top, const Row3& bot, float l, 
     const Dest e = make_dest(p, dests[d], oy, ox);
     const int et = DT >= 0 ? DT : p.views[dests[d] >> 24].dtype;
 #pragma unroll
-    for (int c = 0; c < 3; ++c) put<DT, VEC>(e, et, c, q[c], vec, has_b);
+    for (int c = 0; c < 3; ++c) put<DT, VEC>(e, et, c, q[c], tq[c], vec, has_b);
   }
 }
 
@@ -230,7 +263,7 @@ template <int DT, int ND, bool VEC>
 __device__ __forceinline__ void walk_rows(const LaunchParams& p, const uint32_t* __restrict__ dests, int nd,
                                           const uint2* __restrict__ rtab, const uint32_t* __restrict__ grid,
                                           int gw, int oy0, int rr_lo, int rr_hi, int ox, uint32_t ca, uint32_t cb,
-                                          float2 lx, bool vec, bool has_b) {
+                                          uint64_t lx, bool vec, bool has_b) {
   Dest dl[ND];
   int dt[ND];
 #pragma unroll
@@ -285,7 +318,7 @@ __device__ __forceinline__ void walk(const LaunchParams& p, const WorkItem& w, c
     const int ja = g.flip ? Wo - 1 - ox : ox;
     const int jb = has_b ? (g.flip ? Wo - 2 - ox : ox + 1) : ja;
     const uint2 ta = t.ctab[ja], tb = t.ctab[jb];
-    const float2 lx = make_float2(__uint_as_float(ta.y), __uint_as_float(tb.y));
+    const uint64_t lx = f2::pack(ta.y, tb.y);
     if (nd == 1)
       walk_rows<DT, 1, VEC>(p, dests, nd, rtab, grid, gw, oy_lo, rr_lo, rr_hi, ox, ta.x, tb.x, lx, vec, has_b);
     else

@@ -276,7 +276,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
     int y_hi;
     tap(g.sc_y, g.off_y, oy_lo + nr - 1, g.lim_y, g.org_y, dmy, y_hi, fl);
     __syncthreads();                          // previous band's walkers are done with the grid
-    st::stage_rows(s_rawb, Yp + x16, UVp + x16, w.pitch, gw, y_lo, y_hi, warp, nwarps, lane);
+    st::stage_rows_cp(s_rawb, Yp + x16, UVp + x16, w.pitch, gw, y_lo, y_hi, warp, nwarps, lane);
     for (int r = tid; r < nr; r += nthr) {
       int y0, y1;
       float ly;
@@ -296,7 +296,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
       const uint2 ta = ctab[ja], tb = ctab[jb];
       const uint32_t ca0 = 4u * (ta.x & 0xffffu), ca1 = 4u * (ta.x >> 16);
       const uint32_t cb0 = 4u * (tb.x & 0xffffu), cb1 = 4u * (tb.x >> 16);
-      const float2 lx = make_float2(__uint_as_float(ta.y), __uint_as_float(tb.y));
+      const uint64_t lx = f2::pack(ta.y, tb.y);
       const int per = (nr + groups - 1) / groups;
       const int r_lo = grp * per, r_hi = min(nr, r_lo + per);
       int have0 = -1, have1 = -1;
@@ -305,16 +305,17 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
         const uint4 rt = st::lds128(s_rtab + 16u * rr);
         const uint32_t o0 = s_grid + rt.x, o1 = s_grid + rt.y;
         const int y0 = (int)rt.z;
-        const float2 ly = make_float2(__uint_as_float(rt.w), __uint_as_float(rt.w));
+        const uint64_t ly = f2::splat(__uint_as_float(rt.w));
         const uint32_t pix = (uint32_t)((oy_lo + rr) * Wo + ox);
         auto put3 = [&](const Row3& top, const Row3& bot) {   // vertical lerp + rint -> Q2 planes
 #pragma unroll
           for (int c = 0; c < 3; ++c) {
-            const float2 dv = __ffma2_rn(top.h[c], make_float2(-1.f, -1.f), bot.h[c]);
-            const float2 q = rint2(__ffma2_rn(ly, dv, top.h[c]));
+            const uint64_t dv = f2::fma(top.h[c], f2::splat(-1.f), bot.h[c]);
+            const uint64_t tq = rint_biased(f2::fma(ly, dv, top.h[c]));   // low bytes = q
+            const uint32_t pair = __byte_perm(f2::lo(tq), f2::hi(tq), 0x0040);
             const uint32_t plane = q2 + (uint32_t)(c * sh.plane) + pix;
-            if (has_b) stsu16(plane, (uint32_t)q.x | ((uint32_t)q.y << 8));
-            else stsu8(plane, (uint32_t)q.x);
+            if (has_b) stsu16(plane, pair);
+            else stsu8(plane, pair);
           }
         };
         if (y0 & 1) {

@@ -34,7 +34,7 @@ struct Shape {      // host-chosen launch shape
 
 __host__ __device__ inline size_t smem_bytes(const Shape& s, int maxWo) {
   return a16((size_t)maxWo * 8) + a16((size_t)s.SB * 16) + (size_t)s.ring * s.gw * 4 +
-         2 * a16((size_t)s.raw_rows * s.gw);
+         2 * a16((size_t)s.raw_rows * s.gw) + 16;   // + two mbarriers
 }
 
 __device__ __forceinline__ uint32_t lds32(uint32_t a) {
@@ -55,11 +55,45 @@ __device__ __forceinline__ void cp_async16s(uint32_t s, const void* gmem) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
 }
 
-// Y rows [ya, yb] then UV rows [ya>>1, yb>>1] -> raw (shared address), gw bytes per row.
-// y0/uv0: global addresses of column x16 of Y row 0 / UV row 0 (loop-invariant, computed once
-// per CTA). Warps take rows, lanes take 16 B chunks (gw <= 512 B: one request per lane).
-__device__ __forceinline__ void stage_rows(uint32_t raw, const uint8_t* y0, const uint8_t* uv0, uint32_t pitch,
-                                           int gw, int ya, int yb, int warp, int nwarps, int lane) {
+// mbarrier / bulk-copy primitives (32-bit shared-window addresses)
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n"
+      "SAND_WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra SAND_WAIT_%=;\n}\n" ::"r"(bar),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+               "l"(src), "r"(bytes), "r"(bar)
+               : "memory");
+}
+
+// Y rows [ya, yb] then UV rows [ya>>1, yb>>1] -> raw (shared address), gw bytes per row, as
+// one bulk copy (TMA engine) per row issued by thread `row`; completion is counted in bytes
+// on the buffer's mbarrier. y0/uv0: global addresses of column x16 of Y row 0 / UV row 0
+// (16 B aligned: store rows are 64 B aligned, x16 is a multiple of 16, gw of 16).
+__device__ __forceinline__ void stage_rows(uint32_t raw, uint32_t bar, const uint8_t* y0, const uint8_t* uv0,
+                                           uint32_t pitch, int gw, int ya, int yb, int tid, int nthr) {
+  const int ny = yb - ya + 1, u0 = ya >> 1, nuv = (yb >> 1) - u0 + 1;
+  if (tid == 0) mbar_arrive_expect_tx(bar, (uint32_t)((ny + nuv) * gw));
+  for (int r = tid; r < ny + nuv; r += nthr) {
+    const uint8_t* src = r < ny ? y0 + (size_t)(ya + r) * pitch : uv0 + (size_t)(u0 + r - ny) * pitch;
+    bulk_g2s(raw + (uint32_t)(r * gw), src, (uint32_t)gw, bar);
+  }
+}
+
+// cp.async variant (k_stencil): warps take rows, lanes take 16 B chunks
+__device__ __forceinline__ void stage_rows_cp(uint32_t raw, const uint8_t* y0, const uint8_t* uv0, uint32_t pitch,
+                                              int gw, int ya, int yb, int warp, int nwarps, int lane) {
   const int ny = yb - ya + 1, u0 = ya >> 1, nuv = (yb >> 1) - u0 + 1;
   const int chunks = gw >> 4;
   for (int r = warp; r < ny + nuv; r += nwarps) {
@@ -83,16 +117,22 @@ __device__ __forceinline__ Chroma3 chroma_at(uint32_t uv) {
 }
 
 // RGBx word of luma Y with chroma c: sat((yy + term) >> 20) per channel (OpenCV integer
-// BT.601), computed as min(max(yy + term, 0), 2^28 - 1) >> 4, whose byte 2 is the channel;
-// PRMT gathers the three bytes and the exponent byte 0x4B tops the word (see rs::biased).
+// BT.601), computed as relu(min(yy + term, 2^28 - 1)) >> 4 (one DPX VIADDMNMX.RELU), whose
+// byte 2 is the channel; PRMT gathers the three bytes and the exponent byte 0x4B tops the word
+// (see rs::biased).
 __device__ __forceinline__ uint32_t rgbx_dpx(uint32_t Y, const Chroma3& c) {
   const int yy = (int)max(Y, 16u) * 1220542 + ((1 << 19) - 16 * 1220542);
-  // x >> 4 of the clamped (non-negative) sums as IMAD.HI (FMA pipe) to relieve the ALU pipe
-  const uint32_t mr = __umulhi((uint32_t)min(__viaddmax_s32(yy, c.r, 0), 0x0FFFFFFF), 1u << 28);
-  const uint32_t mg = __umulhi((uint32_t)min(__viaddmax_s32(yy, c.g, 0), 0x0FFFFFFF), 1u << 28);
-  const uint32_t mb = __umulhi((uint32_t)min(__viaddmax_s32(yy, c.b, 0), 0x0FFFFFFF), 1u << 28);
-  const uint32_t rg = __byte_perm(mr, mg, 0x0062);
-  return __byte_perm(rg, mb, 0x7610) + 0x4B000000u;   // byte 3 is zero: add == or
+  // x >> 4 of the clamped sums as IMAD.HI (FMA pipe) to relieve the ALU pipe
+  const uint32_t mr = __umulhi((uint32_t)__viaddmin_s32_relu(yy, c.r, 0x0FFFFFFF), 1u << 28);
+  const uint32_t mg = __umulhi((uint32_t)__viaddmin_s32_relu(yy, c.g, 0x0FFFFFFF), 1u << 28);
+  const uint32_t mb = __umulhi((uint32_t)__viaddmin_s32_relu(yy, c.b, 0x0FFFFFFF), 1u << 28) + 0x4B000000u;
+  return __byte_perm(__byte_perm(mr, mg, 0x0062), mb, 0x7610);
+}
+
+// byte I of w, zero-extended (one PRMT)
+template <int I>
+__device__ __forceinline__ uint32_t byte_of(uint32_t w) {
+  return __byte_perm(w, 0u, 0x4440 | I);
 }
 
 // convert staged rows [ya, yb] into the ring (slot = (y - y_first) % ring_rows)
@@ -117,13 +157,13 @@ __device__ __forceinline__ void convert_rows(uint32_t ring, uint32_t raw, int gw
       const Chroma3 c0 = chroma_at<0>(uv), c1 = chroma_at<16>(uv);
       if (top) {
         const uint32_t yw = lds32(yrow_t + 4 * q);
-        sts128(out_t + 16 * q, make_uint4(rgbx_dpx(yw & 0xffu, c0), rgbx_dpx((yw >> 8) & 0xffu, c0),
-                                          rgbx_dpx((yw >> 16) & 0xffu, c1), rgbx_dpx(yw >> 24, c1)));
+        sts128(out_t + 16 * q, make_uint4(rgbx_dpx(byte_of<0>(yw), c0), rgbx_dpx(byte_of<1>(yw), c0),
+                                          rgbx_dpx(byte_of<2>(yw), c1), rgbx_dpx(byte_of<3>(yw), c1)));
       }
       if (bot) {
         const uint32_t yw = lds32(yrow_b + 4 * q);
-        sts128(out_b + 16 * q, make_uint4(rgbx_dpx(yw & 0xffu, c0), rgbx_dpx((yw >> 8) & 0xffu, c0),
-                                          rgbx_dpx((yw >> 16) & 0xffu, c1), rgbx_dpx(yw >> 24, c1)));
+        sts128(out_b + 16 * q, make_uint4(rgbx_dpx(byte_of<0>(yw), c0), rgbx_dpx(byte_of<1>(yw), c0),
+                                          rgbx_dpx(byte_of<2>(yw), c1), rgbx_dpx(byte_of<3>(yw), c1)));
       }
     }
   }
@@ -131,7 +171,7 @@ __device__ __forceinline__ void convert_rows(uint32_t ring, uint32_t raw, int gw
 
 // horizontal lerps of one ring row for the thread's column pair (R#12); col*: byte offsets
 __device__ __forceinline__ void hrow_s(rs::Row3& r, uint32_t rowaddr, uint32_t ca0, uint32_t ca1, uint32_t cb0,
-                                       uint32_t cb1, float2 lx) {
+                                       uint32_t cb1, uint64_t lx) {
   const uint32_t a0 = lds32(rowaddr + ca0), a1 = lds32(rowaddr + ca1);
   const uint32_t b0 = lds32(rowaddr + cb0), b1 = lds32(rowaddr + cb1);
   r.h[0] = rs::hlerp<0>(a0, a1, b0, b1, lx);
@@ -139,10 +179,13 @@ __device__ __forceinline__ void hrow_s(rs::Row3& r, uint32_t rowaddr, uint32_t c
   r.h[2] = rs::hlerp<2>(a0, a1, b0, b1, lx);
 }
 
-// row actions of the walker (computed once per row by the table builder)
-constexpr uint32_t kActShift = 1;   // y0 = previous y0 + 1: the old bottom row is the new top
-constexpr uint32_t kActJump = 2;    // new y0 (first row or a step > 1): compute both rows
-constexpr uint32_t kActClamp = 4;   // y1 == y0 (bottom edge): bottom = top
+// row actions of the walker (computed once per row by the table builder). Register sets hold
+// the horizontal lerps of the output row's top (y0) and bottom (y1) source rows.
+constexpr uint32_t kActTop = 1;    // (re)compute the top set from ring row y0
+constexpr uint32_t kActBot = 2;    // (re)compute the bottom set from ring row y1
+constexpr uint32_t kActFlip = 4;   // y0 = previous y0 + 1: the old bottom set becomes the top
+// At the bottom edge (y1 == y0) the bottom set is not computed and lambda_y is stored as 0:
+// fmaf(0, b - h0, h0) == h0 == fmaf(lambda, h0 - h0, h0) for any finite b (R#12 unchanged).
 
 }  // namespace st
 
@@ -170,6 +213,13 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
   const uint32_t s_ring = s_rtab + (uint32_t)a16((size_t)sh.SB * 16);
   const uint32_t s_raw = s_ring + (uint32_t)(sh.ring * sh.gw * 4);
   const uint32_t rawcap = (uint32_t)a16((size_t)sh.raw_rows * sh.gw);
+  const uint32_t s_bar = s_raw + 2u * rawcap;            // mbarriers of raw buffers 0 and 1
+  if (tid == 0) {
+    st::mbar_init(s_bar, 1);
+    st::mbar_init(s_bar + 8, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
 
   // footprint of the super-band (monotone taps)
   const int x_lo = tap0(g.sc_x, g.off_x, 0, g.org_x);
@@ -194,7 +244,9 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
   };
   const int nsub = (nr + sh.S - 1) / sh.S;
   int ya = y_first, yb = last_src(0);
-  st::stage_rows(s_raw, Yx, UVx, pitch, gw, ya, yb, warp, nwarps, lane);
+  st::stage_rows(s_raw, s_bar, Yx, UVx, pitch, gw, ya, yb, tid, nthr);
+  uint32_t phase = 0;          // bit b: parity of the next completion of buffer b's barrier
+  bool staged = true;          // sub-band k's rows were staged (k = 0 always adds rows)
 
   // tap tables (overlap the first copy): columns (x0, x1, lambda); rows (byte offsets of
   // the two ring rows, y0, lambda)
@@ -210,24 +262,28 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
     tap(g.sc_y, g.off_y, Y0 + r, g.lim_y, g.org_y, y0, y1, ly);
     const uint32_t s0 = (uint32_t)((y0 - y_first) % sh.ring), s1 = (uint32_t)((y1 - y_first) % sh.ring);
     // action relative to the previous output row of the super-band
-    uint32_t act = st::kActJump;
+    uint32_t act = st::kActTop | st::kActBot;      // first row or a step > 1
     if (r > 0) {
       const int yp = tap0(g.sc_y, g.off_y, Y0 + r - 1, g.org_y);
-      act = y0 == yp ? 0u : (y0 == yp + 1 ? st::kActShift : st::kActJump);
+      act = y0 == yp ? 0u : (y0 == yp + 1 ? st::kActFlip | st::kActBot : act);
     }
-    if (y1 == y0) act |= st::kActClamp;
+    if (y1 == y0) {
+      act &= ~st::kActBot;
+      ly = 0.f;
+    }
     rtab[r] = make_uint4(s0 * rowbytes, s1 * rowbytes, act, __float_as_uint(ly));
   }
 
   // per-thread walker state: output columns (ox, ox+1) for the whole super-band. Every lane
   // walks (lanes past the last pair repeat it without storing), so warps stay converged.
   const int pairs = (Wo + 1) >> 1;
-  const bool valid = tid < pairs;
+  int valid = tid < pairs ? 1 : 0;
+  asm volatile("" : "+r"(valid));   // keep it in a register: no TID re-read per row
   const int ox = 2 * min(tid, pairs - 1);
   const bool has_b = ox + 1 < Wo;
   const bool vec = has_b && !(Wo & 1);
   uint32_t ca0 = 0, ca1 = 0, cb0 = 0, cb1 = 0;
-  float2 lx = make_float2(0.f, 0.f);
+  uint64_t lx = 0ull;
   const int nd = (int)w.n_dest;
   const uint32_t* dests = p.dests + w.dest_begin;
   Dest dl[kInlineDests];
@@ -236,16 +292,26 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
   // says which one is y0. A shift by one source row flips `top` and recomputes only the other
   // set, so no register copies are needed between rows.
   Row3 X, Y;
+#pragma unroll
+  for (int c = 0; c < 3; ++c) X.h[c] = Y.h[c] = 0ull;   // finite (+0) before first use
   int top = 0;
 
   for (int k = 0; k < nsub; ++k) {
-    asm volatile("cp.async.wait_group 0;\n" ::: "memory");
-    __syncthreads();                                 // raw[k&1] landed; walk(k-1) finished
-    st::convert_rows(s_ring, s_raw + (uint32_t)(k & 1) * rawcap, gw, ya, yb, y_first, sh.ring, warp, nwarps, lane);
+    const uint32_t buf = (uint32_t)(k & 1);
+    if (staged) {                                    // raw[buf] landed
+      st::mbar_wait(s_bar + 8u * buf, (phase >> buf) & 1u);
+      phase ^= 1u << buf;
+    }
+    __syncthreads();                                 // walk(k-1) finished
+    if (staged)
+      st::convert_rows(s_ring, s_raw + buf * rawcap, gw, ya, yb, y_first, sh.ring, warp, nwarps, lane);
+    staged = false;
     if (k + 1 < nsub) {                              // stage the next sub-band's new rows
       const int na = yb + 1, nb = last_src(k + 1);
-      if (nb >= na)
-        st::stage_rows(s_raw + (uint32_t)((k + 1) & 1) * rawcap, Yx, UVx, pitch, gw, na, nb, warp, nwarps, lane);
+      if (nb >= na) {
+        st::stage_rows(s_raw + (buf ^ 1u) * rawcap, s_bar + 8u * (buf ^ 1u), Yx, UVx, pitch, gw, na, nb, tid, nthr);
+        staged = true;
+      }
       ya = na;
       yb = max(nb, yb);
     }
@@ -258,7 +324,7 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
       ca1 = 4u * (ta.x >> 16);
       cb0 = 4u * (tb.x & 0xffffu);
       cb1 = 4u * (tb.x >> 16);
-      lx = make_float2(__uint_as_float(ta.y), __uint_as_float(tb.y));
+      lx = f2::pack(ta.y, tb.y);
 #pragma unroll
       for (int d = 0; d < kInlineDests; ++d)
         if (d < nd) {
@@ -271,26 +337,13 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
       const uint4 rt = st::lds128(s_rtab + 16u * rr);
       const uint32_t act = rt.z;
       const float l = __uint_as_float(rt.w);
+      top ^= (act & st::kActFlip) ? 1 : 0;
       if (top == 0) {
-        if (act & st::kActJump) {
-          st::hrow_s(X, s_ring + rt.x, ca0, ca1, cb0, cb1, lx);
-          if (act & st::kActClamp) Y = X;                // bottom edge: y1 == y0 (rare)
-          else st::hrow_s(Y, s_ring + rt.y, ca0, ca1, cb0, cb1, lx);
-        } else if (act & st::kActShift) {
-          top = 1;                                      // Y is the new top; X the new bottom
-          if (act & st::kActClamp) X = Y;
-          else st::hrow_s(X, s_ring + rt.y, ca0, ca1, cb0, cb1, lx);
-        }
+        if (act & st::kActTop) st::hrow_s(X, s_ring + rt.x, ca0, ca1, cb0, cb1, lx);
+        if (act & st::kActBot) st::hrow_s(Y, s_ring + rt.y, ca0, ca1, cb0, cb1, lx);
       } else {
-        if (act & st::kActJump) {
-          st::hrow_s(Y, s_ring + rt.x, ca0, ca1, cb0, cb1, lx);
-          if (act & st::kActClamp) X = Y;
-          else st::hrow_s(X, s_ring + rt.y, ca0, ca1, cb0, cb1, lx);
-        } else if (act & st::kActShift) {
-          top = 0;
-          if (act & st::kActClamp) Y = X;
-          else st::hrow_s(Y, s_ring + rt.y, ca0, ca1, cb0, cb1, lx);
-        }
+        if (act & st::kActTop) st::hrow_s(Y, s_ring + rt.x, ca0, ca1, cb0, cb1, lx);
+        if (act & st::kActBot) st::hrow_s(X, s_ring + rt.y, ca0, ca1, cb0, cb1, lx);
       }
       if (valid) {
         if (top == 0) emit<DT, kInlineDests, VEC>(X, Y, l, dl, dt, p, dests, nd, Y0 + rr, ox, vec, has_b);

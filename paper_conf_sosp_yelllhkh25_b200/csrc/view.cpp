@@ -2,13 +2,17 @@
 // (SAND view abstraction §5.1; POSIX API Table 2).
 //
 // Plans are built per (epoch, rank) on the host — synchronously on first use or
-// ahead of time on a worker thread (sand_view_prefetch_epoch; the plan analogue of
-// the paper's pre-materialisation threads) — and uploaded once, so a read
-// is a presence check plus one kernel launch on the caller's stream.
+// ahead of time by builder threads (read_batch queues the next epochs at iteration 0,
+// sand_view_prefetch_epoch queues any; the plan analogue of the paper's
+// pre-materialisation threads) — and uploaded once by the builder on the view's
+// upload stream, so a read is a presence check, one event wait and one kernel launch on
+// the caller's stream.
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 
 #include "internal.h"
@@ -16,17 +20,21 @@
 namespace sand {
 namespace {
 
-constexpr size_t kPlanCache = 4;
+constexpr size_t kPlanCache = 4;   // current epoch, kPlanAhead ahead, and the previous one
+}  // namespace
+constexpr uint64_t kPlanAhead = 2;
+namespace {
 constexpr double kPi = 3.14159265358979323846;
 
-struct FrameBase {
-  uint64_t offset, frame_stride;
-  uint32_t pitch;
-};
+uint64_t now_ns() {
+  return static_cast<uint64_t>(
+      std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now().time_since_epoch()).count());
+}
 
-FrameBase frame_base(const sand_store* s, uint32_t video) {
-  const VideoEntry& v = s->videos.at(video);
-  return {v.offset, v.frame_stride, v.pitch};
+int env_int(const char* name, int dflt, int lo, int hi) {
+  const char* e = std::getenv(name);
+  const int x = e ? std::atoi(e) : dflt;
+  return std::min(hi, std::max(lo, x));
 }
 
 GroupParams group_params(const sand_view_desc& d, const sand_clip_meta& m, uint32_t q, uint32_t W, uint32_t H) {
@@ -75,21 +83,42 @@ GroupParams group_params(const sand_view_desc& d, const sand_clip_meta& m, uint3
 
 }  // namespace
 
-std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32_t rank) {
+std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32_t rank,
+                                      std::shared_ptr<EpochPlan> plan) {
   const SpecInfo& info = v.info;
   const sand_view_spec& s = info.spec;
   const uint32_t B = s.batch_size;
   const uint32_t nG = static_cast<uint32_t>(info.groups.size());
-  auto plan = std::make_shared<EpochPlan>();
+  // a recycled plan keeps its vectors' capacity: no allocation or page faults per epoch
+  if (!plan) plan = std::make_shared<EpochPlan>();
   plan->epoch = epoch;
   plan->rank = rank;
+  plan->last_touch = 0;
+  plan->items.clear();
+  plan->dests.clear();
+  plan->item_begin.clear();
+  plan->shapes.clear();
+  plan->fetch_begin.clear();
+  plan->fetch_keys.clear();
+  plan->fetch_uses.clear();
+  plan->fetch_entry.clear();
   const std::vector<uint32_t> clips = rank_clips(info, epoch, rank);
   plan->iterations = clips.size() / B;
   const uint64_t n_clips = plan->iterations * B;
-  plan->metas.resize(n_clips);
-  plan->groups.resize(n_clips * nG);
+  plan->metas.resize(n_clips);            // every entry is overwritten by plan_clip
+  plan->groups.resize(n_clips * nG);      // ... and by group_params
+  uint32_t frames_per_clip = 0;
+  for (uint32_t k = 0; k < s.n_views; ++k) frames_per_clip += s.views[k].clip_len;
+  plan->items.reserve(n_clips * frames_per_clip * nG);
+  plan->dests.reserve(n_clips * frames_per_clip);
+  plan->item_begin.reserve(plan->iterations + 1);
+  plan->fetch_begin.reserve(plan->iterations + 1);
+  plan->shapes.reserve(plan->iterations);
   plan->item_begin.push_back(0);
   plan->fetch_begin.push_back(0);
+  std::vector<uint64_t> uses_of;   // (frame << 32) | (view << 16) | t
+  uses_of.reserve(frames_per_clip);
+  std::vector<uint32_t> batch_videos(B);
   int32_t common_dtype = s.views[0].out_dtype;
   int32_t even_wo = 1;
   for (uint32_t k = 0; k < s.n_views; ++k) {
@@ -100,74 +129,96 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
     BatchShape shape{};
     shape.dtype = common_dtype;
     shape.even_wo = even_wo;
-    std::vector<std::pair<uint64_t, uint32_t>> fetch;   // ((video<<32)|frame, uses)
+    struct Fetch {
+      uint64_t key;   // (video << 32) | frame
+      uint32_t uses;
+      VideoEntry* entry;
+      bool operator<(const Fetch& o) const { return key < o.key; }
+    };
+    std::vector<Fetch> fetch;
+    fetch.reserve(B * frames_per_clip);
     for (uint32_t b = 0; b < B; ++b) {
       const uint64_t slot = it * B + b;
       sand_clip_meta& m = plan->metas[slot];
       const uint32_t clip = clips[slot];
       plan_clip(info, epoch, clip, &m);
       const VideoDims& dim = info.dims[clip / s.samples_per_video];
-      const FrameBase fb = frame_base(v.store, dim.id);
+      VideoEntry* ent = v.entries[clip / s.samples_per_video];
       for (uint32_t gi = 0; gi < nG; ++gi) {
         const uint32_t q = info.groups[gi];
         plan->groups[slot * nG + gi] = group_params(s.views[info.leader[q]], m, q, dim.width, dim.height);
       }
-      // unique source frames of the clip, in order of first use
-      std::vector<uint32_t> uniq;
+      // launch-shape contribution and stencil flag of each group (independent of the frame)
+      uint32_t gflags[SAND_MAX_GROUPS];
+      for (uint32_t gi = 0; gi < nG; ++gi) {
+        const GroupParams& g = plan->groups[slot * nG + gi];
+        gflags[gi] = (g.rot_on || g.blur_on) ? 1u : 0u;
+        const int cols = std::min(2 * g.out_w, static_cast<int>(std::ceil(static_cast<double>(g.sc_x) * g.out_w)) + 3);
+        if (gflags[gi]) {
+          shape.has_stencil = 1;
+          shape.st_max_wo = std::max(shape.st_max_wo, g.out_w);
+          shape.st_max_ho = std::max(shape.st_max_ho, g.out_h);
+          shape.st_cols_bound = std::max(shape.st_cols_bound, cols);
+          shape.st_max_scy = std::max(shape.st_max_scy, g.sc_y);
+        } else {
+          shape.has_direct = 1;
+          shape.max_wo = std::max(shape.max_wo, g.out_w);
+          shape.max_ho = std::max(shape.max_ho, g.out_h);
+          shape.cols_bound = std::max(shape.cols_bound, cols);
+          shape.max_scy = std::max(shape.max_scy, g.sc_y);
+        }
+      }
+      // (frame, view, t) uses of the clip sorted by frame: one pass groups the destinations of
+      // each unique source frame (view-major, t ascending within a frame)
+      uses_of.clear();
       for (uint32_t k = 0; k < s.n_views; ++k)
         for (uint32_t t = 0; t < s.views[k].clip_len; ++t)
-          if (std::find(uniq.begin(), uniq.end(), m.frames[k][t]) == uniq.end()) uniq.push_back(m.frames[k][t]);
-      for (uint32_t f : uniq) {
+          uses_of.push_back((static_cast<uint64_t>(m.frames[k][t]) << 32) | (k << 16) | t);
+      std::sort(uses_of.begin(), uses_of.end());
+      for (size_t i = 0; i < uses_of.size();) {
+        const uint32_t f = static_cast<uint32_t>(uses_of[i] >> 32);
+        size_t j = i;
+        while (j < uses_of.size() && static_cast<uint32_t>(uses_of[j] >> 32) == f) ++j;
         uint32_t uses = 0;
         for (uint32_t gi = 0; gi < nG; ++gi) {
           const uint32_t q = info.groups[gi];
           WorkItem w{};
           w.dest_begin = static_cast<uint32_t>(plan->dests.size());
-          for (uint32_t k = 0; k < s.n_views; ++k) {
-            if (s.views[k].spatial_group != q) continue;
-            for (uint32_t t = 0; t < s.views[k].clip_len; ++t)
-              if (m.frames[k][t] == f) plan->dests.push_back(pack_dest(k, t, b));
+          for (size_t x = i; x < j; ++x) {
+            const uint32_t k = static_cast<uint32_t>(uses_of[x] >> 16) & 0xffffu;
+            if (s.views[k].spatial_group == q)
+              plan->dests.push_back(pack_dest(k, static_cast<uint32_t>(uses_of[x]) & 0xffffu, b));
           }
           w.n_dest = static_cast<uint32_t>(plan->dests.size()) - w.dest_begin;
           if (w.n_dest == 0) continue;
           uses += w.n_dest;
-          w.y_off = fb.offset + fb.frame_stride * f;
-          w.pitch = fb.pitch;
+          w.y_off = ent->offset + ent->frame_stride * f;
+          w.pitch = ent->pitch;
           w.src_w = dim.width;
           w.src_h = dim.height;
           w.gp = static_cast<uint32_t>(slot * nG + gi);
           w.clip_slot = b;
           w.group = q;
-          const GroupParams& g = plan->groups[w.gp];
-          w.flags = (g.rot_on || g.blur_on) ? 1u : 0u;
-          if (w.flags) {
-            shape.has_stencil = 1;
-            shape.st_max_wo = std::max(shape.st_max_wo, g.out_w);
-            shape.st_max_ho = std::max(shape.st_max_ho, g.out_h);
-            const int cols = std::min(2 * g.out_w, static_cast<int>(std::ceil(static_cast<double>(g.sc_x) * g.out_w)) + 3);
-            shape.st_cols_bound = std::max(shape.st_cols_bound, cols);
-            shape.st_max_scy = std::max(shape.st_max_scy, g.sc_y);
-          } else {
-            shape.has_direct = 1;
-            shape.max_wo = std::max(shape.max_wo, g.out_w);
-            shape.max_ho = std::max(shape.max_ho, g.out_h);
-            const int cols = std::min(2 * g.out_w, static_cast<int>(std::ceil(static_cast<double>(g.sc_x) * g.out_w)) + 3);
-            shape.cols_bound = std::max(shape.cols_bound, cols);
-            shape.max_scy = std::max(shape.max_scy, g.sc_y);
-          }
+          w.flags = gflags[gi];
           plan->items.push_back(w);
         }
-        fetch.push_back({(static_cast<uint64_t>(dim.id) << 32) | f, uses});
+        fetch.push_back({(static_cast<uint64_t>(dim.id) << 32) | f, uses, ent});
+        i = j;
       }
+      batch_videos[b] = dim.id;
     }
-    // batch-unique (video, frame): merge clips that share a source frame
-    std::sort(fetch.begin(), fetch.end());
+    // batch-unique (video, frame): clips of different videos never share a frame, so merging
+    // (sort + run-length) is only needed when a video occurs twice in the batch
+    std::sort(batch_videos.begin(), batch_videos.begin() + B);
+    const bool shared = std::adjacent_find(batch_videos.begin(), batch_videos.begin() + B) != batch_videos.begin() + B;
+    if (shared) std::sort(fetch.begin(), fetch.end());
     for (size_t i = 0; i < fetch.size();) {
       size_t j = i;
       uint32_t uses = 0;
-      while (j < fetch.size() && fetch[j].first == fetch[i].first) uses += fetch[j++].second;
-      plan->fetch_keys.push_back({static_cast<uint32_t>(fetch[i].first >> 32), static_cast<uint32_t>(fetch[i].first)});
+      while (j < fetch.size() && fetch[j].key == fetch[i].key) uses += fetch[j++].uses;
+      plan->fetch_keys.push_back({static_cast<uint32_t>(fetch[i].key >> 32), static_cast<uint32_t>(fetch[i].key)});
       plan->fetch_uses.push_back(uses);
+      plan->fetch_entry.push_back(fetch[i].entry);
       i = j;
     }
     plan->fetch_begin.push_back(static_cast<uint32_t>(plan->fetch_keys.size()));
@@ -179,8 +230,8 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
 
 namespace {
 
-// return a plan's buffers to the view's pool (its kernels finish before the pool hands the
-// buffer out again: the pool waits on the buffer's event, which is long done by then)
+// return a plan's buffers to the view's pool (caller holds v->mu). The next owner waits on
+// the buffer's events before overwriting it.
 void release_plan_device(sand_view* v, EpochPlan& p) {
   if (p.d_buf) {
     PlanBuffer b;
@@ -188,75 +239,108 @@ void release_plan_device(sand_view* v, EpochPlan& p) {
     b.h = p.h_stage;
     b.bytes = p.d_bytes;
     b.done = p.last_use;
+    b.ready = p.ready;
     v->pool.push_back(b);
-  } else if (p.last_use) {
-    cudaEventDestroy(p.last_use);
   }
   p.d_buf = p.h_stage = nullptr;
-  p.last_use = nullptr;
+  p.last_use = p.ready = nullptr;
   p.uploaded = false;
 }
 
-void free_pool(sand_view* v) {
-  for (auto& b : v->pool) {
-    if (b.done) {
-      cudaEventSynchronize(b.done);
-      cudaEventDestroy(b.done);
-    }
-    cudaFree(b.d);
-    cudaFreeHost(b.h);
+void destroy_buffer(PlanBuffer& b) {
+  if (b.done) {
+    cudaEventSynchronize(b.done);
+    cudaEventDestroy(b.done);
   }
+  if (b.ready) {
+    cudaEventSynchronize(b.ready);
+    cudaEventDestroy(b.ready);
+  }
+  cudaFree(b.d);
+  cudaFreeHost(b.h);
+}
+
+void free_pool(sand_view* v) {
+  for (auto& b : v->pool) destroy_buffer(b);
   v->pool.clear();
 }
 
-int upload_plan(sand_view* v, EpochPlan& p, cudaStream_t stream) {
-  const size_t gb = p.groups.size() * sizeof(GroupParams);
-  const size_t ib = p.items.size() * sizeof(WorkItem);
-  const size_t db = p.dests.size() * sizeof(uint32_t);
-  const size_t off_i = (gb + 255) / 256 * 256;
-  const size_t off_d = off_i + (ib + 255) / 256 * 256;
-  const size_t total = std::max<size_t>(off_d + db, 256);
-  // smallest pooled buffer that fits, else a new one with headroom
+struct PlanLayout {
+  size_t gb, ib, db, off_i, off_d, total;
+};
+
+PlanLayout plan_layout(const EpochPlan& p) {
+  PlanLayout L;
+  L.gb = p.groups.size() * sizeof(GroupParams);
+  L.ib = p.items.size() * sizeof(WorkItem);
+  L.db = p.dests.size() * sizeof(uint32_t);
+  L.off_i = (L.gb + 255) / 256 * 256;
+  L.off_d = L.off_i + (L.ib + 255) / 256 * 256;
+  L.total = std::max<size_t>(L.off_d + L.db, 256);
+  return L;
+}
+
+// Caller holds v->mu: the smallest pooled buffer of at least `bytes`, or an empty one.
+PlanBuffer take_buffer(sand_view* v, size_t bytes) {
   int best = -1;
   for (size_t i = 0; i < v->pool.size(); ++i)
-    if (v->pool[i].bytes >= total && (best < 0 || v->pool[i].bytes < v->pool[best].bytes)) best = (int)i;
+    if (v->pool[i].bytes >= bytes && (best < 0 || v->pool[i].bytes < v->pool[best].bytes)) best = (int)i;
   PlanBuffer buf;
   if (best >= 0) {
     buf = v->pool[best];
     v->pool.erase(v->pool.begin() + best);
-    if (buf.done) cudaEventSynchronize(buf.done);   // the previous owner's kernels are done
-  } else {
-    buf.bytes = total + total / 4;
-    cudaError_t e = cudaMalloc(&buf.d, buf.bytes);
-    if (e != cudaSuccess) return cuda_error(e, "cudaMalloc(plan)");
-    e = cudaMallocHost(&buf.h, buf.bytes);
-    if (e != cudaSuccess) {
-      cudaFree(buf.d);
-      return cuda_error(e, "cudaMallocHost(plan)");
-    }
-    e = cudaEventCreateWithFlags(&buf.done, cudaEventDisableTiming);
-    if (e != cudaSuccess) return cuda_error(e, "cudaEventCreate");
   }
-  auto* h = static_cast<uint8_t*>(buf.h);
-  if (gb) std::memcpy(h, p.groups.data(), gb);
-  if (ib) std::memcpy(h + off_i, p.items.data(), ib);
-  if (db) std::memcpy(h + off_d, p.dests.data(), db);
-  cudaError_t e = cudaMemcpyAsync(buf.d, buf.h, total, cudaMemcpyHostToDevice, stream);
+  return buf;
+}
+
+// Upload a built plan into buf (allocated here if empty) on the view's upload stream; runs on
+// the builder thread without v->mu. On failure the buffer is handed back through *buf.
+int upload_plan(sand_view* v, EpochPlan& p, PlanBuffer* buf) {
+  const PlanLayout L = plan_layout(p);
+  cudaError_t e = cudaSetDevice(v->store->device);
+  if (e != cudaSuccess) return cuda_error(e, "cudaSetDevice");
+  if (!buf->d) {
+    buf->bytes = L.total + L.total / 4;
+    const char* what = "cudaMalloc(plan)";
+    e = cudaMalloc(&buf->d, buf->bytes);
+    if (e == cudaSuccess) e = cudaMallocHost(&buf->h, buf->bytes), what = "cudaMallocHost(plan)";
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&buf->done, cudaEventDisableTiming), what = "cudaEventCreate";
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&buf->ready, cudaEventDisableTiming);
+    if (e != cudaSuccess) {
+      destroy_buffer(*buf);
+      *buf = PlanBuffer{};
+      return cuda_error(e, what);
+    }
+  } else {
+    cudaEventSynchronize(buf->done);    // kernels of the previous owner finished
+    cudaEventSynchronize(buf->ready);   // its upload no longer reads the staging copy
+  }
+  auto* h = static_cast<uint8_t*>(buf->h);
+  if (L.gb) std::memcpy(h, p.groups.data(), L.gb);
+  if (L.ib) std::memcpy(h + L.off_i, p.items.data(), L.ib);
+  if (L.db) std::memcpy(h + L.off_d, p.dests.data(), L.db);
+  e = cudaMemcpyAsync(buf->d, buf->h, L.total, cudaMemcpyHostToDevice, v->upload_stream);
   if (e != cudaSuccess) return cuda_error(e, "cudaMemcpyAsync(plan)");
-  auto* d = static_cast<uint8_t*>(buf.d);
-  p.d_buf = buf.d;
-  p.h_stage = buf.h;
-  p.d_bytes = buf.bytes;
-  p.last_use = buf.done;
+  e = cudaEventRecord(buf->ready, v->upload_stream);
+  if (e != cudaSuccess) return cuda_error(e, "cudaEventRecord(plan ready)");
+  auto* d = static_cast<uint8_t*>(buf->d);
+  p.d_buf = buf->d;
+  p.h_stage = buf->h;
+  p.d_bytes = buf->bytes;
+  p.last_use = buf->done;
+  p.ready = buf->ready;
+  p.ready_waited = nullptr;
   p.d_groups = reinterpret_cast<GroupParams*>(d);
-  p.d_items = reinterpret_cast<WorkItem*>(d + off_i);
-  p.d_dests = reinterpret_cast<uint32_t*>(d + off_d);
+  p.d_items = reinterpret_cast<WorkItem*>(d + L.off_i);
+  p.d_dests = reinterpret_cast<uint32_t*>(d + L.off_d);
   p.uploaded = true;
   return SAND_OK;
 }
 
-// Caller holds v->mu. Returns the cached plan, waiting for / building it as needed.
-std::shared_ptr<EpochPlan> get_plan(sand_view* v, std::unique_lock<std::mutex>& lk, uint64_t epoch, uint32_t rank) {
+// Caller holds v->mu. Returns the cached plan, waiting for / building (and uploading) it as
+// needed; *rc reports an upload failure (the plan is then returned without device copy).
+std::shared_ptr<EpochPlan> get_plan(sand_view* v, std::unique_lock<std::mutex>& lk, uint64_t epoch, uint32_t rank,
+                                    int* rc = nullptr) {
   const auto key = std::make_pair(epoch, rank);
   for (;;) {
     auto it = v->plans.find(key);
@@ -271,10 +355,30 @@ std::shared_ptr<EpochPlan> get_plan(sand_view* v, std::unique_lock<std::mutex>& 
     break;
   }
   v->pending[key] = true;
+  std::shared_ptr<EpochPlan> plan;
+  if (!v->spare_plans.empty()) {
+    plan = std::move(v->spare_plans.back());
+    v->spare_plans.pop_back();
+  }
   lk.unlock();
-  auto plan = build_plan(*v, epoch, rank);
+  const uint64_t t0 = now_ns();
+  plan = build_plan(*v, epoch, rank, std::move(plan));
+  const PlanLayout L = plan_layout(*plan);
   lk.lock();
+  PlanBuffer buf = take_buffer(v, L.total);
+  lk.unlock();
+  const int urc = upload_plan(v, *plan, &buf);
+  const uint64_t t1 = now_ns();
+  lk.lock();
+  v->plan_build_ns += t1 - t0;
   v->pending.erase(key);
+  if (rc) *rc = urc;
+  if (urc != SAND_OK) {   // not cached: the next call rebuilds; the buffer returns to the pool
+    if (buf.d) v->pool.push_back(buf);
+    plan->uploaded = false;
+    v->cv.notify_all();
+    return plan;
+  }
   v->plans_built++;
   plan->last_touch = ++v->touch;
   v->plans[key] = plan;
@@ -284,6 +388,7 @@ std::shared_ptr<EpochPlan> get_plan(sand_view* v, std::unique_lock<std::mutex>& 
       if (i->second->last_touch < victim->second->last_touch) victim = i;
     if (victim->first == key) break;
     release_plan_device(v, *victim->second);
+    if (victim->second.use_count() == 1) v->spare_plans.push_back(std::move(victim->second));
     v->plans.erase(victim);
   }
   v->cv.notify_all();
@@ -327,6 +432,7 @@ extern "C" int sand_view_create(sand_store* s, const sand_view_spec* spec, sand_
         return sand::set_error(SAND_ERANGE, "dataset video " + std::to_string(id) + " not in the store");
       }
       v->info.dims.push_back({id, it->second.n_frames, it->second.width, it->second.height});
+      v->entries.push_back(&it->second);
     }
   }
   sand::derive_spec(&v->info);
@@ -375,8 +481,14 @@ extern "C" int sand_view_create(sand_store* s, const sand_view_spec* spec, sand_
     delete v;
     return rc;
   }
+  e = cudaStreamCreateWithFlags(&v->upload_stream, cudaStreamNonBlocking);
+  if (e != cudaSuccess) {
+    delete v;
+    return sand::cuda_error(e, "cudaStreamCreate(upload)");
+  }
   s->live_views++;
-  v->worker = std::thread(sand::worker_loop, v);
+  const int n_workers = sand::env_int("SAND_PLAN_THREADS", 2, 1, 16);
+  for (int i = 0; i < n_workers; ++i) v->workers.emplace_back(sand::worker_loop, v);
   *out = v;
   return SAND_OK;
 }
@@ -422,34 +534,45 @@ extern "C" int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank,
     if (reinterpret_cast<uintptr_t>(out->data[k]) % 16 != 0) return sand::set_error(SAND_EINVAL, "output not 16 B aligned");
   }
   auto stream = static_cast<cudaStream_t>(out->stream);
+  const uint64_t t0 = sand::now_ns();
   std::unique_lock<std::mutex> lk(v->mu);
-  auto plan = sand::get_plan(v, lk, epoch, rank);
+  int urc = SAND_OK;
+  auto plan = sand::get_plan(v, lk, epoch, rank, &urc);
+  const uint64_t t1 = sand::now_ns();
+  v->plan_wait_ns += t1 - t0;
   if (out->iteration >= plan->iterations) return sand::set_error(SAND_ERANGE, "iteration out of range");
   cudaError_t e = cudaSetDevice(v->store->device);
   if (e != cudaSuccess) return sand::cuda_error(e, "cudaSetDevice");
-  if (!plan->uploaded) {
-    int rc = sand::upload_plan(v, *plan, stream);
-    if (rc != SAND_OK) return rc;
+  if (!plan->uploaded) return urc != SAND_OK ? urc : sand::set_error(SAND_ECUDA, "plan has no device copy");
+  if (plan->ready_waited != stream) {   // order the caller's stream after the plan upload
+    e = cudaStreamWaitEvent(stream, plan->ready, 0);
+    if (e != cudaSuccess) return sand::cuda_error(e, "cudaStreamWaitEvent(plan ready)");
+    plan->ready_waited = stream;
   }
   const uint64_t it = out->iteration;
   const uint32_t ib = plan->item_begin[it], ie = plan->item_begin[it + 1];
-  // plan the next epoch on the worker while this one is consumed (pre-materialisation of the
-  // plan, the analogue of the paper's pre-materialisation threads)
+  // plan the next epochs on the builder threads while this one is consumed
+  // (pre-materialisation of the plan, the analogue of the paper's pre-materialisation
+  // threads)
   if (it == 0) {
-    const auto next = std::make_pair(epoch + 1, rank);
-    if (!v->plans.count(next) && !v->pending.count(next)) {
-      v->queue.push_back(next);
-      v->cv.notify_all();
+    for (uint64_t ahead = 1; ahead <= sand::kPlanAhead; ++ahead) {
+      const auto next = std::make_pair(epoch + ahead, rank);
+      if (!v->plans.count(next) && !v->pending.count(next) &&
+          std::find(v->queue.begin(), v->queue.end(), next) == v->queue.end()) {
+        v->queue.push_back(next);
+        v->cv.notify_one();
+      }
     }
   }
   sand_store* st = v->store;
   {
     std::lock_guard<std::mutex> slk(st->mu);
     for (uint32_t i = plan->fetch_begin[it]; i < plan->fetch_begin[it + 1]; ++i) {
-      const auto& key = plan->fetch_keys[i];
-      if (!st->videos.at(key.first).present[key.second])
+      if (!plan->fetch_entry[i]->present[plan->fetch_keys[i].second]) {
+        const auto& key = plan->fetch_keys[i];
         return sand::set_error(SAND_ENOENT, "frame " + std::to_string(key.second) + " of video " +
                                                 std::to_string(key.first) + " is not in the store");
+      }
     }
   }
   sand::LaunchParams lp{};
@@ -472,15 +595,16 @@ extern "C" int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank,
   {
     std::lock_guard<std::mutex> slk(st->mu);
     for (uint32_t i = plan->fetch_begin[it]; i < plan->fetch_begin[it + 1]; ++i) {
-      auto& ve = st->videos.at(plan->fetch_keys[i].first);
-      ve.fetches[plan->fetch_keys[i].second] += 1;
-      ve.uses[plan->fetch_keys[i].second] += plan->fetch_uses[i];
+      sand::VideoEntry* ve = plan->fetch_entry[i];
+      ve->fetches[plan->fetch_keys[i].second] += 1;
+      ve->uses[plan->fetch_keys[i].second] += plan->fetch_uses[i];
     }
     st->batches++;
   }
   v->batches++;
   v->launches += static_cast<uint64_t>(launched);
   v->work_items += lp.n_items;
+  v->read_ns += sand::now_ns() - t0;
   return SAND_OK;
 }
 
@@ -568,6 +692,9 @@ extern "C" int sand_view_get_stats(const sand_view* v, sand_view_stats* out) {
   out->kernel_launches = v->launches;
   out->plans_built = v->plans_built;
   out->work_items = v->work_items;
+  out->plan_build_ns = v->plan_build_ns;
+  out->plan_wait_ns = v->plan_wait_ns;
+  out->read_ns = v->read_ns;
   return SAND_OK;
 }
 
@@ -578,10 +705,12 @@ extern "C" int sand_view_destroy(sand_view* v) {
     v->stop = true;
     v->cv.notify_all();
   }
-  if (v->worker.joinable()) v->worker.join();
+  for (auto& w : v->workers)
+    if (w.joinable()) w.join();
   cudaSetDevice(v->store->device);
   for (auto& kv : v->plans) sand::release_plan_device(v, *kv.second);
   sand::free_pool(v);
+  if (v->upload_stream) cudaStreamDestroy(v->upload_stream);
   v->store->live_views--;
   delete v;
   return SAND_OK;
