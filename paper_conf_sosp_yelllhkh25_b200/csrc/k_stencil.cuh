@@ -286,7 +286,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
     }
     asm volatile("cp.async.wait_group 0;\n" ::: "memory");
     __syncthreads();
-    st::convert_rows(s_grid, s_rawb, gw, y_lo, y_hi, y_lo, 1 << 30, warp, nwarps, lane);
+    st::convert_rows(s_grid, s_rawb, gw, y_lo, y_hi, y_lo, 1 << 30, 5u, warp, nwarps, lane);   // no wrap
     __syncthreads();
     if (grp < groups && pr < pairs) {
       const int ox = 2 * pr;

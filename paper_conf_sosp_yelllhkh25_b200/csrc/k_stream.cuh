@@ -27,14 +27,22 @@ struct Shape {      // host-chosen launch shape
   int SB;           // output rows per CTA
   int nsb;          // super-bands per item (ceil(maxHo / SB))
   int S;            // output rows per sub-band
-  int ring;         // ring capacity in source rows
-  int raw_rows;     // raw staging capacity in rows (Y + UV) per buffer
+  int ring;         // ring capacity in source rows (>= rows one sub-band spans)
+  int raw_rows;     // raw staging capacity in rows (Y + UV)
   int gw;           // max row width in bytes of Y (= words of RGBx), multiple of 16
+  uint32_t ring_magic;   // floor(2^32 / ring) + 1: x / ring == umulhi(x, ring_magic) for x < 2^16
 };
+
+__device__ __forceinline__ uint32_t ring_mod(uint32_t x, uint32_t ring, uint32_t magic) {
+  return x - __umulhi(x, magic) * ring;
+}
+__device__ __forceinline__ uint32_t ring_mod(uint32_t x, const Shape& s) {
+  return ring_mod(x, (uint32_t)s.ring, s.ring_magic);
+}
 
 __host__ __device__ inline size_t smem_bytes(const Shape& s, int maxWo) {
   return a16((size_t)maxWo * 8) + a16((size_t)s.SB * 16) + (size_t)s.ring * s.gw * 4 +
-         2 * a16((size_t)s.raw_rows * s.gw) + 16;   // + two mbarriers
+         a16((size_t)s.raw_rows * s.gw) + 16;   // + the staging mbarrier
 }
 
 __device__ __forceinline__ uint32_t lds32(uint32_t a) {
@@ -137,7 +145,7 @@ __device__ __forceinline__ uint32_t byte_of(uint32_t w) {
 
 // convert staged rows [ya, yb] into the ring (slot = (y - y_first) % ring_rows)
 __device__ __forceinline__ void convert_rows(uint32_t ring, uint32_t raw, int gw, int ya, int yb, int y_first,
-                                             int ring_rows, int warp, int nwarps, int lane) {
+                                             int ring_rows, uint32_t ring_magic, int warp, int nwarps, int lane) {
   const int ny = yb - ya + 1;
   if (ny <= 0) return;
   const int u0 = ya >> 1, nuv = (yb >> 1) - u0 + 1;
@@ -147,7 +155,7 @@ __device__ __forceinline__ void convert_rows(uint32_t ring, uint32_t raw, int gw
   for (int u = warp; u < nuv; u += nwarps) {
     const int yt = 2 * (u0 + u);
     const bool top = yt >= ya, bot = yt + 1 <= yb;
-    const int st = (yt - y_first + ring_rows) % ring_rows;   // yt may be y_first - 1
+    const int st = (int)ring_mod((uint32_t)(yt - y_first + ring_rows), (uint32_t)ring_rows, ring_magic);   // yt may be y_first - 1
     const int sb = st + 1 == ring_rows ? 0 : st + 1;
     const uint32_t yrow_t = raw + (uint32_t)((yt - ya) * gw), yrow_b = raw + (uint32_t)((yt + 1 - ya) * gw);
     const uint32_t out_t = ring + (uint32_t)st * rowbytes, out_b = ring + (uint32_t)sb * rowbytes;
@@ -187,10 +195,63 @@ constexpr uint32_t kActFlip = 4;   // y0 = previous y0 + 1: the old bottom set b
 // At the bottom edge (y1 == y0) the bottom set is not computed and lambda_y is stored as 0:
 // fmaf(0, b - h0, h0) == h0 == fmaf(lambda, h0 - h0, h0) for any finite b (R#12 unchanged).
 
+// Vertical lerp + rint + stores of one output row for NP column pairs (R#12, R#17), NP = 2:
+// four adjacent columns, one 8 B (bf16) / 16 B (f32) / 4 B (u8) store per channel and
+// destination. Requires out_w % 4 == 0 for every view (host-checked), so the stores are aligned.
+template <int DT, int ND, int NP>
+__device__ __forceinline__ void emit_np(const rs::Row3 (&top)[NP], const rs::Row3 (&bot)[NP], float l,
+                                        rs::Dest (&dl)[ND], const LaunchParams& p, const uint32_t* __restrict__ dests,
+                                        int nd, int oy, int ox) {
+  using namespace rs;
+  const uint64_t ly = f2::splat(l);
+  uint64_t q[NP][3], tq[NP][3];
+#pragma unroll
+  for (int j = 0; j < NP; ++j)
+#pragma unroll
+    for (int c = 0; c < 3; ++c) {
+      const uint64_t dv = f2::fma(top[j].h[c], f2::splat(-1.f), bot[j].h[c]);   // h1 - h0
+      tq[j][c] = rint_biased(f2::fma(ly, dv, top[j].h[c]));                     // rint(fmaf(ly, h1-h0, h0))
+      q[j][c] = DT == SAND_U8 ? tq[j][c] : f2::add(tq[j][c], f2::splat(-kRound));
+    }
+  auto store = [&](const Dest& d) {
+#pragma unroll
+    for (int c = 0; c < 3; ++c) {
+      uint8_t* o = d.row + (size_t)c * d.cstride;
+      if (DT == SAND_U8) {
+        const uint32_t p0 = __byte_perm(f2::lo(tq[0][c]), f2::hi(tq[0][c]), 0x0040);
+        const uint32_t p1 = __byte_perm(f2::lo(tq[1][c]), f2::hi(tq[1][c]), 0x0040);
+        *reinterpret_cast<uint32_t*>(o) = __byte_perm(p0, p1, 0x5410);
+      } else {
+        const uint64_t a = f2::splat(d.a[c]), b = f2::splat(d.b[c]);
+        const uint64_t y0 = f2::fma(q[0][c], a, b), y1 = f2::fma(q[1][c], a, b);   // fmaf(q, a_c, b_c)
+        if (DT == SAND_BF16) {
+          const __nv_bfloat162 v0 = __floats2bfloat162_rn(f2::lof(y0), f2::hif(y0));
+          const __nv_bfloat162 v1 = __floats2bfloat162_rn(f2::lof(y1), f2::hif(y1));
+          *reinterpret_cast<uint2*>(o) =
+              make_uint2(*reinterpret_cast<const uint32_t*>(&v0), *reinterpret_cast<const uint32_t*>(&v1));
+        } else {
+          *reinterpret_cast<uint4*>(o) = make_uint4(f2::lo(y0), f2::hi(y0), f2::lo(y1), f2::hi(y1));
+        }
+      }
+    }
+  };
+#pragma unroll
+  for (int d = 0; d < ND; ++d) {
+    if (d == 0 || d < nd) {
+      store(dl[d]);
+      dl[d].row += dl[d].rstride;
+    }
+  }
+  for (int d = ND; d < nd; ++d) store(make_dest(p, dests[d], oy, ox));   // rare: more destinations
+}
+
 }  // namespace st
 
-template <int DT, bool VEC>
-__global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Shape sh, int maxWo) {
+// NP column pairs per thread: NP = 1 (any width, any dtype) or NP = 2 (out_w % 4 == 0 and a
+// single specialised dtype; halves the per-row walker overhead per column)
+template <int DT, bool VEC, int NP>
+__global__ void __launch_bounds__(NP == 1 ? 256 : 128, NP == 1 ? 3 : 4) k_stream(const LaunchParams p, st::Shape sh, int maxWo) {
+  static_assert(NP == 1 || (NP == 2 && VEC && DT >= 0), "NP = 2 needs the specialised vector path");
   extern __shared__ __align__(16) uint8_t smem_raw[];
   using namespace rs;
   const int item_idx = blockIdx.x / sh.nsb;
@@ -212,11 +273,9 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
   const uint32_t s_rtab = s_base + (uint32_t)a16((size_t)maxWo * 8);
   const uint32_t s_ring = s_rtab + (uint32_t)a16((size_t)sh.SB * 16);
   const uint32_t s_raw = s_ring + (uint32_t)(sh.ring * sh.gw * 4);
-  const uint32_t rawcap = (uint32_t)a16((size_t)sh.raw_rows * sh.gw);
-  const uint32_t s_bar = s_raw + 2u * rawcap;            // mbarriers of raw buffers 0 and 1
+  const uint32_t s_bar = s_raw + (uint32_t)a16((size_t)sh.raw_rows * sh.gw);   // staging mbarrier
   if (tid == 0) {
     st::mbar_init(s_bar, 1);
-    st::mbar_init(s_bar + 8, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
@@ -244,8 +303,8 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
   };
   const int nsub = (nr + sh.S - 1) / sh.S;
   int ya = y_first, yb = last_src(0);
-  st::stage_rows(s_raw, s_bar, Yx, UVx, pitch, gw, ya, yb, tid, nthr);
-  uint32_t phase = 0;          // bit b: parity of the next completion of buffer b's barrier
+  if (warp == 0) st::stage_rows(s_raw, s_bar, Yx, UVx, pitch, gw, ya, yb, lane, 32);
+  uint32_t phase = 0;          // parity of the staging barrier's next completion
   bool staged = true;          // sub-band k's rows were staged (k = 0 always adds rows)
 
   // tap tables (overlap the first copy): columns (x0, x1, lambda); rows (byte offsets of
@@ -260,7 +319,7 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
     int y0, y1;
     float ly;
     tap(g.sc_y, g.off_y, Y0 + r, g.lim_y, g.org_y, y0, y1, ly);
-    const uint32_t s0 = (uint32_t)((y0 - y_first) % sh.ring), s1 = (uint32_t)((y1 - y_first) % sh.ring);
+    const uint32_t s0 = st::ring_mod((uint32_t)(y0 - y_first), sh), s1 = st::ring_mod((uint32_t)(y1 - y_first), sh);
     // action relative to the previous output row of the super-band
     uint32_t act = st::kActTop | st::kActBot;      // first row or a step > 1
     if (r > 0) {
@@ -274,16 +333,18 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
     rtab[r] = make_uint4(s0 * rowbytes, s1 * rowbytes, act, __float_as_uint(ly));
   }
 
-  // per-thread walker state: output columns (ox, ox+1) for the whole super-band. Every lane
-  // walks (lanes past the last pair repeat it without storing), so warps stay converged.
+  // per-thread walker state: output columns [ox, ox + 2 NP) for the whole super-band. Every
+  // lane walks (lanes past the last column group repeat it without storing), so warps stay
+  // converged.
   const int pairs = (Wo + 1) >> 1;
-  int valid = tid < pairs ? 1 : 0;
+  const int ngrp = (pairs + NP - 1) / NP;
+  int valid = tid < ngrp ? 1 : 0;
   asm volatile("" : "+r"(valid));   // keep it in a register: no TID re-read per row
-  const int ox = 2 * min(tid, pairs - 1);
+  const int ox = 2 * NP * min(tid, ngrp - 1);
   const bool has_b = ox + 1 < Wo;
   const bool vec = has_b && !(Wo & 1);
-  uint32_t ca0 = 0, ca1 = 0, cb0 = 0, cb1 = 0;
-  uint64_t lx = 0ull;
+  uint32_t ca0[NP], ca1[NP], cb0[NP], cb1[NP];
+  uint64_t lx[NP];
   const int nd = (int)w.n_dest;
   const uint32_t* dests = p.dests + w.dest_begin;
   Dest dl[kInlineDests];
@@ -291,40 +352,57 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
   // Two register sets X, Y hold the horizontal lerps of source rows y0 and y0 + 1; `top`
   // says which one is y0. A shift by one source row flips `top` and recomputes only the other
   // set, so no register copies are needed between rows.
-  Row3 X, Y;
+  Row3 X[NP], Y[NP];
 #pragma unroll
-  for (int c = 0; c < 3; ++c) X.h[c] = Y.h[c] = 0ull;   // finite (+0) before first use
+  for (int j = 0; j < NP; ++j) {
+    ca0[j] = ca1[j] = cb0[j] = cb1[j] = 0;
+    lx[j] = 0ull;
+#pragma unroll
+    for (int c = 0; c < 3; ++c) X[j].h[c] = Y[j].h[c] = 0ull;   // finite (+0) before first use
+  }
   int top = 0;
+  auto hrows = [&](Row3 (&R)[NP], uint32_t rowaddr) {
+#pragma unroll
+    for (int j = 0; j < NP; ++j) st::hrow_s(R[j], rowaddr, ca0[j], ca1[j], cb0[j], cb1[j], lx[j]);
+  };
 
+  // One staging buffer: sub-band k+1's rows are copied while sub-band k is walked (the
+  // copy is issued once the conversion of k has drained the buffer).
   for (int k = 0; k < nsub; ++k) {
-    const uint32_t buf = (uint32_t)(k & 1);
-    if (staged) {                                    // raw[buf] landed
-      st::mbar_wait(s_bar + 8u * buf, (phase >> buf) & 1u);
-      phase ^= 1u << buf;
+    if (staged) {                                    // raw landed
+      st::mbar_wait(s_bar, phase);
+      phase ^= 1u;
     }
-    __syncthreads();                                 // walk(k-1) finished
-    if (staged)
-      st::convert_rows(s_ring, s_raw + buf * rawcap, gw, ya, yb, y_first, sh.ring, warp, nwarps, lane);
+    __syncthreads();                                 // walk(k-1) finished: its ring rows are free
+    if (staged) st::convert_rows(s_ring, s_raw, gw, ya, yb, y_first, sh.ring, sh.ring_magic, warp, nwarps, lane);
     staged = false;
+    __syncthreads();                                 // ring holds every row of sub-band k; raw drained
     if (k + 1 < nsub) {                              // stage the next sub-band's new rows
       const int na = yb + 1, nb = last_src(k + 1);
       if (nb >= na) {
-        st::stage_rows(s_raw + (buf ^ 1u) * rawcap, s_bar + 8u * (buf ^ 1u), Yx, UVx, pitch, gw, na, nb, tid, nthr);
+        if (warp == 0) {
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic reads of raw before async writes
+          st::stage_rows(s_raw, s_bar, Yx, UVx, pitch, gw, na, nb, lane, 32);
+        }
         staged = true;
       }
       ya = na;
       yb = max(nb, yb);
     }
-    __syncthreads();                                 // ring holds every row of sub-band k
     if (k == 0) {                                    // tables are visible now
-      const int ja = g.flip ? Wo - 1 - ox : ox;
-      const int jb = has_b ? (g.flip ? Wo - 2 - ox : ox + 1) : ja;
-      const uint2 ta = ctab[ja], tb = ctab[jb];
-      ca0 = 4u * (ta.x & 0xffffu);
-      ca1 = 4u * (ta.x >> 16);
-      cb0 = 4u * (tb.x & 0xffffu);
-      cb1 = 4u * (tb.x >> 16);
-      lx = f2::pack(ta.y, tb.y);
+#pragma unroll
+      for (int j = 0; j < NP; ++j) {
+        const int oj = ox + 2 * j;                     // NP = 2: every pair is inside the row
+        const bool hb = NP == 1 ? has_b : true;
+        const int ja = g.flip ? Wo - 1 - oj : oj;
+        const int jb = hb ? (g.flip ? Wo - 2 - oj : oj + 1) : ja;
+        const uint2 ta = ctab[ja], tb = ctab[jb];
+        ca0[j] = 4u * (ta.x & 0xffffu);
+        ca1[j] = 4u * (ta.x >> 16);
+        cb0[j] = 4u * (tb.x & 0xffffu);
+        cb1[j] = 4u * (tb.x >> 16);
+        lx[j] = f2::pack(ta.y, tb.y);
+      }
 #pragma unroll
       for (int d = 0; d < kInlineDests; ++d)
         if (d < nd) {
@@ -339,15 +417,20 @@ __global__ void __launch_bounds__(256, 3) k_stream(const LaunchParams p, st::Sha
       const float l = __uint_as_float(rt.w);
       top ^= (act & st::kActFlip) ? 1 : 0;
       if (top == 0) {
-        if (act & st::kActTop) st::hrow_s(X, s_ring + rt.x, ca0, ca1, cb0, cb1, lx);
-        if (act & st::kActBot) st::hrow_s(Y, s_ring + rt.y, ca0, ca1, cb0, cb1, lx);
+        if (act & st::kActTop) hrows(X, s_ring + rt.x);
+        if (act & st::kActBot) hrows(Y, s_ring + rt.y);
       } else {
-        if (act & st::kActTop) st::hrow_s(Y, s_ring + rt.x, ca0, ca1, cb0, cb1, lx);
-        if (act & st::kActBot) st::hrow_s(X, s_ring + rt.y, ca0, ca1, cb0, cb1, lx);
+        if (act & st::kActTop) hrows(Y, s_ring + rt.x);
+        if (act & st::kActBot) hrows(X, s_ring + rt.y);
       }
       if (valid) {
-        if (top == 0) emit<DT, kInlineDests, VEC>(X, Y, l, dl, dt, p, dests, nd, Y0 + rr, ox, vec, has_b);
-        else emit<DT, kInlineDests, VEC>(Y, X, l, dl, dt, p, dests, nd, Y0 + rr, ox, vec, has_b);
+        if constexpr (NP == 1) {
+          if (top == 0) emit<DT, kInlineDests, VEC>(X[0], Y[0], l, dl, dt, p, dests, nd, Y0 + rr, ox, vec, has_b);
+          else emit<DT, kInlineDests, VEC>(Y[0], X[0], l, dl, dt, p, dests, nd, Y0 + rr, ox, vec, has_b);
+        } else {
+          if (top == 0) st::emit_np<DT, kInlineDests, NP>(X, Y, l, dl, p, dests, nd, Y0 + rr, ox);
+          else st::emit_np<DT, kInlineDests, NP>(Y, X, l, dl, p, dests, nd, Y0 + rr, ox);
+        }
       }
     }
   }

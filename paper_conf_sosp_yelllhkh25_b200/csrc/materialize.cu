@@ -207,8 +207,11 @@ ResampleCfg choose_resample(const BatchShape& sh) {
     s.S = env_int("SAND_STREAM_S", 8);
     s.SB = env_int("SAND_STREAM_SB", 56);
     s.nsb = (sh.max_ho + s.SB - 1) / s.SB;
-    s.ring = (int)std::ceil((double)sh.max_scy * s.S) + 3;
+    // rows one sub-band spans: y0 of its S output rows moves by <= ceil((S-1) * scy), plus
+    // the first y0 and the last y1; the raw buffer holds a sub-band's new Y rows and their UV rows
+    s.ring = (int)std::ceil((double)sh.max_scy * (s.S - 1)) + 2;
     s.raw_rows = s.ring + s.ring / 2 + 2;
+    s.ring_magic = (uint32_t)((1ull << 32) / (uint64_t)s.ring + 1);
     s.gw = (int)gwb;
     ResampleCfg c{2, 0, st::smem_bytes(s, sh.max_wo), s};
     if (s.ring <= 255 && c.smem <= 200 * 1024) return c;
@@ -236,9 +239,19 @@ int launch_resample_dt(const LaunchParams& p, const BatchShape& sh, cudaStream_t
   if (cfg.smem > 227 * 1024) return set_error(SAND_EINVAL, "resample tile exceeds shared memory (source crop too large)");
   const int pairs = (sh.max_wo + 1) / 2;
   if (cfg.mode == 2) {
-    const int threads = ((pairs + 31) / 32) * 32;
     const unsigned blocks = (unsigned)((uint64_t)p.n_items * cfg.st.nsb);
-    k_stream<DT, VEC><<<blocks, threads, cfg.smem, stream>>>(p, cfg.st, sh.max_wo);
+    static const int np_env = env_int("SAND_STREAM_NP", 2);
+    if constexpr (VEC && DT >= 0) {
+      if (sh.wo_mod4 && np_env == 2) {   // four columns per thread
+        const int threads = (((pairs + 1) / 2 + 31) / 32) * 32;
+        k_stream<DT, VEC, 2><<<blocks, threads, cfg.smem, stream>>>(p, cfg.st, sh.max_wo);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return cuda_error(e, "k_stream launch");
+        return SAND_OK;
+      }
+    }
+    const int threads = ((pairs + 31) / 32) * 32;
+    k_stream<DT, VEC, 1><<<blocks, threads, cfg.smem, stream>>>(p, cfg.st, sh.max_wo);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_error(e, "k_stream launch");
     return SAND_OK;
@@ -296,8 +309,10 @@ int configure_kernels(size_t stencil_smem) {
                           allow_smem(k_resample_raw<SAND_BF16, true>), allow_smem(k_resample_raw<SAND_F32, true>),
                           allow_smem(k_resample_gather<-1, false>), allow_smem(k_resample_gather<SAND_U8, true>),
                           allow_smem(k_resample_gather<SAND_BF16, true>), allow_smem(k_resample_gather<SAND_F32, true>),
-                          allow_smem(k_stream<-1, false>), allow_smem(k_stream<SAND_U8, true>),
-                          allow_smem(k_stream<SAND_BF16, true>), allow_smem(k_stream<SAND_F32, true>),
+                          allow_smem(k_stream<-1, false, 1>), allow_smem(k_stream<SAND_U8, true, 1>),
+                          allow_smem(k_stream<SAND_BF16, true, 1>), allow_smem(k_stream<SAND_F32, true, 1>),
+                          allow_smem(k_stream<SAND_U8, true, 2>), allow_smem(k_stream<SAND_BF16, true, 2>),
+                          allow_smem(k_stream<SAND_F32, true, 2>),
                           allow_smem(k_stencil2<-1, false>), allow_smem(k_stencil2<SAND_U8, true>),
                           allow_smem(k_stencil2<SAND_BF16, true>), allow_smem(k_stencil2<SAND_F32, true>)})
       if (r != cudaSuccess) e = r;

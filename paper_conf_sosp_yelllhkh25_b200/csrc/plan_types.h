@@ -68,6 +68,7 @@ struct BatchShape {
   float max_scy;          // largest vertical source step (rows per output row)
   int32_t dtype;          // output dtype shared by every view, or -1 if mixed
   int32_t even_wo;        // every view's out_w is even
+  int32_t wo_mod4;        // every view's out_w is a multiple of 4
   // stencil (rotation/blur) items
   int32_t st_max_wo, st_max_ho, st_cols_bound;
   float st_max_scy;

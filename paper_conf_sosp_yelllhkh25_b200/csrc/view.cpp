@@ -120,15 +120,17 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
   uses_of.reserve(frames_per_clip);
   std::vector<uint32_t> batch_videos(B);
   int32_t common_dtype = s.views[0].out_dtype;
-  int32_t even_wo = 1;
+  int32_t even_wo = 1, wo_mod4 = 1;
   for (uint32_t k = 0; k < s.n_views; ++k) {
     if (s.views[k].out_dtype != common_dtype) common_dtype = -1;
     if (s.views[k].out_w & 1u) even_wo = 0;
+    if (s.views[k].out_w & 3u) wo_mod4 = 0;
   }
   for (uint64_t it = 0; it < plan->iterations; ++it) {
     BatchShape shape{};
     shape.dtype = common_dtype;
     shape.even_wo = even_wo;
+    shape.wo_mod4 = wo_mod4;
     struct Fetch {
       uint64_t key;   // (video << 32) | frame
       uint32_t uses;
