@@ -323,10 +323,20 @@ def run_sand(args):
     host = {"read_batch_us": (st1.read_ns - st0.read_ns) / 1e3 / args.steps,
             "plan_wait_us": (st1.plan_wait_ns - st0.plan_wait_ns) / 1e3 / args.steps,
             "plans_built": int(st1.plans_built - st0.plans_built),
+            "plan_cpu_ms_each": (st1.plan_cpu_ns - st0.plan_cpu_ns) / 1e6 / max(1, st1.plans_built - st0.plans_built),
+            "plan_buffer_wait_ms": (st1.plan_buffer_wait_ns - st0.plan_buffer_wait_ns) / 1e6,
+            "lock_wait_us": (st1.lock_wait_ns - st0.lock_wait_ns) / 1e3 / args.steps,
+            "pending_waits": int(st1.pending_waits - st0.pending_waits),
             "plan_build_ms_each": ((st1.plan_build_ns - st0.plan_build_ns) / 1e6 /
                                    max(1, st1.plans_built - st0.plans_built))}
     elapsed_ms = start.elapsed_time(end)
-    kernel_ms = sum(a.elapsed_time(b) for a, b in zip(kstart, kend)) / args.steps
+    kraw = [a.elapsed_time(b) for a, b in zip(kstart, kend)]
+    kt = sorted(kraw)
+    kernel_ms = sum(kt) / args.steps
+    host["kernel_ms_p10_p50_p90"] = [kt[len(kt) // 10], kt[len(kt) // 2], kt[(9 * len(kt)) // 10]]
+    slow = [(i, round(x, 3)) for i, x in enumerate(kraw) if x > 2 * kt[len(kt) // 2]]
+    host["slow_steps"] = {"n": len(slow), "ms_total": round(sum(x for _, x in slow), 3),
+                          "first": [(first_timed + i, x) for i, x in slow[:8]], "iters_per_epoch": iters}
     elapsed_ms, kernel_ms_max = max_over_ranks([elapsed_ms, kernel_ms], world, f"cuda:{local}")
     ms_per_step = elapsed_ms / args.steps
     value = fps * args.steps * world / (elapsed_ms / 1000.0)

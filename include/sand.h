@@ -216,10 +216,13 @@ int sand_plan_clip(const sand_view_spec* spec, const uint32_t* n_frames, const u
 
 /* Statistics of a view group: batches read, kernels launched, epoch plans built and work
  * items launched so far; host time spent building plans (all builder threads), blocked in
- * read_batch waiting for a plan, and inside read_batch in total (nanoseconds). */
+ * read_batch waiting for a plan, and inside read_batch in total (nanoseconds); the planner's
+ * CPU time alone, its waits for recycled plan buffers, read_batch's wait for the view lock,
+ * and how many reads found their epoch plan still being built. */
 typedef struct {
   uint64_t batches, kernel_launches, plans_built, work_items;
   uint64_t plan_build_ns, plan_wait_ns, read_ns;
+  uint64_t plan_cpu_ns, plan_buffer_wait_ns, lock_wait_ns, pending_waits;
 } sand_view_stats;
 int sand_view_get_stats(const sand_view* v, sand_view_stats* out);
 

@@ -60,7 +60,24 @@ PRODUCT_CU = ["materialize.cu"]
 PRODUCT_HDR = ["internal.h", "plan_types.h", "planner.h", "k_resample.cuh", "k_stream.cuh", "k_stencil.cuh"]
 
 
-def build_product(force=False):
+def build_product(force=False, variant=None, defines=()):
+    """libsand.so, or libsand_<variant>.so compiled with extra -D defines (A/B experiments)."""
+    if variant:
+        import shutil
+        bdir = os.path.join(PKG, "build_" + variant)
+        os.makedirs(bdir, exist_ok=True)
+        objs = []
+        inc = ["-I", os.path.join(ROOT, "include"), "-I", CSRC]
+        for s in PRODUCT_CPP:
+            objs.append(os.path.join(PKG, "build", s + ".o"))
+        for s in PRODUCT_CU:
+            obj = os.path.join(bdir, s + ".o")
+            objs.append(obj)
+            _run([NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xptxas", "-v",
+                  "--expt-relaxed-constexpr", *["-D" + d for d in defines], *inc, "-c", os.path.join(CSRC, s), "-o", obj])
+        _run([NVCC, *ARCH, "-shared", "-Xcompiler", "-fPIC", *objs, "-o", os.path.join(PKG, f"libsand_{variant}.so"),
+              "-lcudart", "-lpthread"])
+        return
     os.makedirs(os.path.join(PKG, "build"), exist_ok=True)
     inc = ["-I", os.path.join(ROOT, "include"), "-I", CSRC]
     hdrs = [os.path.join(ROOT, "include", "sand.h")] + [os.path.join(CSRC, h) for h in PRODUCT_HDR]
@@ -95,5 +112,8 @@ if __name__ == "__main__":
     what = sys.argv[1:] or ["all"]
     force = "--force" in what
     what = [w for w in what if w != "--force"] or ["all"]
+    if what and what[0] == "variant":   # python native_build.py variant <name> DEF=1 ...
+        build_product(variant=what[1], defines=what[2:])
+        sys.exit(0)
     for w in what:
         {"all": build_all, "synth": build_synth, "oracle": build_oracle, "product": build_product}[w](force)

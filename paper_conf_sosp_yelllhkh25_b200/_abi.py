@@ -11,7 +11,8 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libsand.so")
+# SAND_LIB selects another in-tree build of the same library (A/B experiments: libsand_*.so)
+LIB_PATH = os.path.join(_HERE, os.environ.get("SAND_LIB", "libsand.so"))
 
 MAX_VIEWS = 8
 MAX_GROUPS = 8
@@ -78,7 +79,8 @@ class sand_batch_bytes(ctypes.Structure):
 
 class sand_view_stats(ctypes.Structure):
     _fields_ = [("batches", u64), ("kernel_launches", u64), ("plans_built", u64), ("work_items", u64),
-                ("plan_build_ns", u64), ("plan_wait_ns", u64), ("read_ns", u64)]
+                ("plan_build_ns", u64), ("plan_wait_ns", u64), ("read_ns", u64),
+                ("plan_cpu_ns", u64), ("plan_buffer_wait_ns", u64), ("lock_wait_ns", u64), ("pending_waits", u64)]
 
 
 P = ctypes.POINTER

@@ -113,7 +113,11 @@ struct sand_view {
   // stats
   uint64_t batches = 0, launches = 0, plans_built = 0, work_items = 0;
   uint64_t plan_build_ns = 0, plan_wait_ns = 0, read_ns = 0;
+  uint64_t plan_cpu_ns = 0, plan_buffer_wait_ns = 0, lock_wait_ns = 0, pending_waits = 0;
   size_t stencil_smem = 0;   // dynamic smem of the stencil path (0 if no view rotates/blurs)
+  uint32_t* d_sched = nullptr;   // kSchedSlots pairs of ticket counters (persistent kernels)
+  uint32_t sched_seq = 0;        // next slot pair
+  size_t n_buffers = 0;          // plan buffers allocated so far
 };
 
 namespace sand {

@@ -31,6 +31,7 @@ struct Shape {      // host-chosen launch shape
   int raw_rows;     // raw staging capacity in rows (Y + UV)
   int gw;           // max row width in bytes of Y (= words of RGBx), multiple of 16
   uint32_t ring_magic;   // floor(2^32 / ring) + 1: x / ring == umulhi(x, ring_magic) for x < 2^16
+  int opts;         // bit0: warp-row conversion units instead of flattened units (A/B switch)
 };
 
 __device__ __forceinline__ uint32_t ring_mod(uint32_t x, uint32_t ring, uint32_t magic) {
@@ -177,6 +178,48 @@ __device__ __forceinline__ void convert_rows(uint32_t ring, uint32_t raw, int gw
   }
 }
 
+// convert_rows with the (UV row, 4-pixel group) units flattened over all threads of the CTA,
+// so a row width that is not a multiple of 32 groups leaves no lane idle
+__device__ __forceinline__ void convert_rows_flat(uint32_t ring, uint32_t raw, int gw, int ya, int yb, int y_first,
+                                                  int ring_rows, uint32_t ring_magic, int tid, int nthr) {
+  const int ny = yb - ya + 1;
+  if (ny <= 0) return;
+  const int u0 = ya >> 1, nuv = (yb >> 1) - u0 + 1;
+  const int q4 = gw >> 2;                      // 4-pixel groups per row
+  const int total = nuv * q4;
+  if (tid >= total) return;
+  const uint32_t rawUV = raw + (uint32_t)(ny * gw);
+  const uint32_t rowbytes = (uint32_t)gw * 4u;
+  int u = tid / q4, q = tid - u * q4;          // unit -> (u, q), advanced incrementally
+  const int du = nthr / q4, dq = nthr - du * q4;
+  for (int i = tid; i < total; i += nthr) {
+    const int yt = 2 * (u0 + u);
+    const int st = (int)ring_mod((uint32_t)(yt - y_first + ring_rows), (uint32_t)ring_rows, ring_magic);
+    const int sb = st + 1 == ring_rows ? 0 : st + 1;
+    const uint32_t yrow_t = raw + (uint32_t)((yt - ya) * gw + 4 * q);
+    const uint32_t uv = lds32(rawUV + (uint32_t)(u * gw + 4 * q));
+    const Chroma3 c0 = chroma_at<0>(uv), c1 = chroma_at<16>(uv);
+    if (yt >= ya) {
+      const uint32_t yw = lds32(yrow_t);
+      sts128(ring + (uint32_t)st * rowbytes + 16u * q,
+             make_uint4(rgbx_dpx(byte_of<0>(yw), c0), rgbx_dpx(byte_of<1>(yw), c0), rgbx_dpx(byte_of<2>(yw), c1),
+                        rgbx_dpx(byte_of<3>(yw), c1)));
+    }
+    if (yt + 1 <= yb) {
+      const uint32_t yw = lds32(yrow_t + (uint32_t)gw);
+      sts128(ring + (uint32_t)sb * rowbytes + 16u * q,
+             make_uint4(rgbx_dpx(byte_of<0>(yw), c0), rgbx_dpx(byte_of<1>(yw), c0), rgbx_dpx(byte_of<2>(yw), c1),
+                        rgbx_dpx(byte_of<3>(yw), c1)));
+    }
+    q += dq;
+    u += du;
+    if (q >= q4) {
+      q -= q4;
+      ++u;
+    }
+  }
+}
+
 // horizontal lerps of one ring row for the thread's column pair (R#12); col*: byte offsets
 __device__ __forceinline__ void hrow_s(rs::Row3& r, uint32_t rowaddr, uint32_t ca0, uint32_t ca1, uint32_t cb0,
                                        uint32_t cb1, uint64_t lx) {
@@ -249,22 +292,16 @@ __device__ __forceinline__ void emit_np(const rs::Row3 (&top)[NP], const rs::Row
 
 // NP column pairs per thread: NP = 1 (any width, any dtype) or NP = 2 (out_w % 4 == 0 and a
 // single specialised dtype; halves the per-row walker overhead per column)
+#ifndef SAND_NP2_MINB
+#define SAND_NP2_MINB 4   // resident 128-thread CTAs per SM the NP = 2 walker is compiled for
+#endif
 template <int DT, bool VEC, int NP>
-__global__ void __launch_bounds__(NP == 1 ? 256 : 128, NP == 1 ? 3 : 4) k_stream(const LaunchParams p, st::Shape sh, int maxWo) {
+__global__ void __launch_bounds__(NP == 1 ? 256 : 128, NP == 1 ? 3 : SAND_NP2_MINB) k_stream(const LaunchParams p, st::Shape sh, int maxWo) {
   static_assert(NP == 1 || (NP == 2 && VEC && DT >= 0), "NP = 2 needs the specialised vector path");
   extern __shared__ __align__(16) uint8_t smem_raw[];
   using namespace rs;
-  const int item_idx = blockIdx.x / sh.nsb;
-  const int sb = blockIdx.x - item_idx * sh.nsb;
-  const WorkItem w = p.items[item_idx];
-  if (w.flags & 1u) return;
-  const GroupParams& g = p.groups[w.gp];
-  const int Wo = g.out_w, Ho = g.out_h;
-  const int Y0 = sb * sh.SB;
-  if (Y0 >= Ho) return;
-  const int nr = min(sh.SB, Ho - Y0);
   const int tid = threadIdx.x, nthr = blockDim.x;
-  const int warp = tid >> 5, lane = tid & 31, nwarps = nthr >> 5;
+  const int warp = tid >> 5, lane = tid & 31;
 
   uint2* ctab = reinterpret_cast<uint2*>(smem_raw);
   uint4* rtab = reinterpret_cast<uint4*>(smem_raw + a16((size_t)maxWo * 8));
@@ -274,11 +311,27 @@ __global__ void __launch_bounds__(NP == 1 ? 256 : 128, NP == 1 ? 3 : 4) k_stream
   const uint32_t s_ring = s_rtab + (uint32_t)a16((size_t)sh.SB * 16);
   const uint32_t s_raw = s_ring + (uint32_t)(sh.ring * sh.gw * 4);
   const uint32_t s_bar = s_raw + (uint32_t)a16((size_t)sh.raw_rows * sh.gw);   // staging mbarrier
+  // persistent CTAs: task (item, super-band) indices blockIdx.x + i * gridDim.x (uniform
+  // across the CTA, so item/group fields stay in uniform registers)
+  const uint32_t n_tasks = p.n_items * (uint32_t)sh.nsb;
   if (tid == 0) {
     st::mbar_init(s_bar, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
+  uint32_t phase = 0;          // parity of the staging barrier's next completion
+
+  for (uint32_t task = blockIdx.x; task < n_tasks; task += gridDim.x) {
+  [&]() {
+  const int item_idx = (int)(task / (uint32_t)sh.nsb);
+  const int sb = (int)task - item_idx * sh.nsb;
+  const WorkItem w = p.items[item_idx];
+  if (w.flags & 1u) return;
+  const GroupParams& g = p.groups[w.gp];
+  const int Wo = g.out_w, Ho = g.out_h;
+  const int Y0 = sb * sh.SB;
+  if (Y0 >= Ho) return;
+  const int nr = min(sh.SB, Ho - Y0);
 
   // footprint of the super-band (monotone taps)
   const int x_lo = tap0(g.sc_x, g.off_x, 0, g.org_x);
@@ -303,8 +356,10 @@ __global__ void __launch_bounds__(NP == 1 ? 256 : 128, NP == 1 ? 3 : 4) k_stream
   };
   const int nsub = (nr + sh.S - 1) / sh.S;
   int ya = y_first, yb = last_src(0);
-  if (warp == 0) st::stage_rows(s_raw, s_bar, Yx, UVx, pitch, gw, ya, yb, lane, 32);
-  uint32_t phase = 0;          // parity of the staging barrier's next completion
+  if (warp == 0) {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // the previous task's generic reads of raw
+    st::stage_rows(s_raw, s_bar, Yx, UVx, pitch, gw, ya, yb, lane, 32);
+  }
   bool staged = true;          // sub-band k's rows were staged (k = 0 always adds rows)
 
   // tap tables (overlap the first copy): columns (x0, x1, lambda); rows (byte offsets of
@@ -374,7 +429,10 @@ __global__ void __launch_bounds__(NP == 1 ? 256 : 128, NP == 1 ? 3 : 4) k_stream
       phase ^= 1u;
     }
     __syncthreads();                                 // walk(k-1) finished: its ring rows are free
-    if (staged) st::convert_rows(s_ring, s_raw, gw, ya, yb, y_first, sh.ring, sh.ring_magic, warp, nwarps, lane);
+    if (staged) {
+      if (sh.opts & 1) st::convert_rows(s_ring, s_raw, gw, ya, yb, y_first, sh.ring, sh.ring_magic, warp, nthr >> 5, lane);
+      else st::convert_rows_flat(s_ring, s_raw, gw, ya, yb, y_first, sh.ring, sh.ring_magic, tid, nthr);
+    }
     staged = false;
     __syncthreads();                                 // ring holds every row of sub-band k; raw drained
     if (k + 1 < nsub) {                              // stage the next sub-band's new rows
@@ -433,6 +491,9 @@ __global__ void __launch_bounds__(NP == 1 ? 256 : 128, NP == 1 ? 3 : 4) k_stream
         }
       }
     }
+  }
+  }();
+  __syncthreads();             // task done: shared memory free for the next one
   }
 }
 

@@ -13,6 +13,9 @@
 
 #include <algorithm>
 #include <cmath>
+#include <map>
+#include <mutex>
+#include <tuple>
 #include <cstdlib>
 #include <string>
 
@@ -205,13 +208,14 @@ ResampleCfg choose_resample(const BatchShape& sh) {
   if (mild && sh.max_wo <= 512 && forced != 1 && forced != 0) {
     st::Shape s;
     s.S = env_int("SAND_STREAM_S", 8);
-    s.SB = env_int("SAND_STREAM_SB", 56);
+    s.SB = env_int("SAND_STREAM_SB", 32);
     s.nsb = (sh.max_ho + s.SB - 1) / s.SB;
     // rows one sub-band spans: y0 of its S output rows moves by <= ceil((S-1) * scy), plus
     // the first y0 and the last y1; the raw buffer holds a sub-band's new Y rows and their UV rows
     s.ring = (int)std::ceil((double)sh.max_scy * (s.S - 1)) + 2;
     s.raw_rows = s.ring + s.ring / 2 + 2;
     s.ring_magic = (uint32_t)((1ull << 32) / (uint64_t)s.ring + 1);
+    s.opts = env_int("SAND_STREAM_OPTS", 0);
     s.gw = (int)gwb;
     ResampleCfg c{2, 0, st::smem_bytes(s, sh.max_wo), s};
     if (s.ring <= 255 && c.smem <= 200 * 1024) return c;
@@ -233,17 +237,46 @@ ResampleCfg choose_resample(const BatchShape& sh) {
   return {0, 1, 0, {}};
 }
 
+// Grid of a persistent kernel: every resident CTA slot of the device (occupancy at this block
+// size and shared memory), capped by the task count. Cached per (kernel, threads, smem).
+template <typename K>
+unsigned persistent_grid(K kernel, int threads, size_t smem, uint64_t tasks) {
+  static std::mutex mu;
+  static std::map<std::tuple<const void*, int, size_t>, unsigned> cache;
+  const auto key = std::make_tuple(reinterpret_cast<const void*>(kernel), threads, smem);
+  unsigned slots = 0;
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = cache.find(key);
+    if (it != cache.end()) slots = it->second;
+  }
+  if (slots == 0) {
+    int dev = 0, nsm = 0, nb = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kernel, threads, smem);
+    const int cap = env_int("SAND_CTAS_PER_SM", 0);
+    if (cap > 0) nb = std::min(nb, cap);
+    slots = (unsigned)std::max(1, nsm) * (unsigned)std::max(1, nb);
+    if (env_int("SAND_PERSIST", 1) == 0) slots = ~0u;   // one CTA per task (A/B switch)
+    std::lock_guard<std::mutex> lk(mu);
+    cache[key] = slots;
+  }
+  return (unsigned)std::min<uint64_t>(tasks, slots);
+}
+
 template <int DT, bool VEC>
 int launch_resample_dt(const LaunchParams& p, const BatchShape& sh, cudaStream_t stream) {
   const ResampleCfg cfg = choose_resample(sh);
   if (cfg.smem > 227 * 1024) return set_error(SAND_EINVAL, "resample tile exceeds shared memory (source crop too large)");
   const int pairs = (sh.max_wo + 1) / 2;
   if (cfg.mode == 2) {
-    const unsigned blocks = (unsigned)((uint64_t)p.n_items * cfg.st.nsb);
+    const uint64_t tasks = (uint64_t)p.n_items * cfg.st.nsb;
     static const int np_env = env_int("SAND_STREAM_NP", 2);
     if constexpr (VEC && DT >= 0) {
       if (sh.wo_mod4 && np_env == 2) {   // four columns per thread
         const int threads = (((pairs + 1) / 2 + 31) / 32) * 32;
+        const unsigned blocks = persistent_grid(k_stream<DT, VEC, 2>, threads, cfg.smem, tasks);
         k_stream<DT, VEC, 2><<<blocks, threads, cfg.smem, stream>>>(p, cfg.st, sh.max_wo);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return cuda_error(e, "k_stream launch");
@@ -251,6 +284,7 @@ int launch_resample_dt(const LaunchParams& p, const BatchShape& sh, cudaStream_t
       }
     }
     const int threads = ((pairs + 31) / 32) * 32;
+    const unsigned blocks = persistent_grid(k_stream<DT, VEC, 1>, threads, cfg.smem, tasks);
     k_stream<DT, VEC, 1><<<blocks, threads, cfg.smem, stream>>>(p, cfg.st, sh.max_wo);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_error(e, "k_stream launch");
@@ -291,7 +325,10 @@ bool choose_stencil(const BatchShape& sh, sc::Shape* out, size_t* smem) {
 
 template <typename K>
 cudaError_t allow_smem(K kernel) {
-  cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+  cudaFuncAttributes fa;
+  cudaError_t e = cudaFuncGetAttributes(&fa, kernel);
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024 - (int)fa.sharedSizeBytes);
   if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(kernel, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
 }

@@ -84,6 +84,10 @@ struct LaunchParams {
   ViewConst views[kMaxViews];
   uint32_t n_views;
   uint32_t batch;          // B
+  uint32_t* sched;         // ticket counters of persistent kernels: [2 * slot] next task, [2 * slot + 1] CTAs done
+  uint32_t sched_slot;     // slot of this launch (counters are zero between launches)
 };
+
+constexpr int kSchedSlots = 64;
 
 }  // namespace sand

@@ -21,6 +21,8 @@ namespace sand {
 namespace {
 
 constexpr size_t kPlanCache = 4;   // current epoch, kPlanAhead ahead, and the previous one
+constexpr size_t kMaxPooled = 8;   // idle plan buffers kept for reuse
+constexpr size_t kPrealloc = 6;    // spare plan buffers allocated with the first one
 }  // namespace
 constexpr uint64_t kPlanAhead = 2;
 namespace {
@@ -282,17 +284,48 @@ PlanLayout plan_layout(const EpochPlan& p) {
   return L;
 }
 
-// Caller holds v->mu: the smallest pooled buffer of at least `bytes`, or an empty one.
+// Caller holds v->mu: the smallest pooled buffer of at least `bytes` whose previous owner's
+// kernels and upload have completed, or an empty one (the builder then allocates a new buffer).
+// Evicted plans may still have batches queued on the GPU when the host runs ahead; taking
+// such a buffer would make the builder wait for the GPU and leave the next epoch's plan late.
 PlanBuffer take_buffer(sand_view* v, size_t bytes) {
   int best = -1;
-  for (size_t i = 0; i < v->pool.size(); ++i)
-    if (v->pool[i].bytes >= bytes && (best < 0 || v->pool[i].bytes < v->pool[best].bytes)) best = (int)i;
+  for (size_t i = 0; i < v->pool.size(); ++i) {
+    const PlanBuffer& b = v->pool[i];
+    if (b.bytes < bytes || (best >= 0 && b.bytes >= v->pool[best].bytes)) continue;
+    if ((b.done && cudaEventQuery(b.done) != cudaSuccess) || (b.ready && cudaEventQuery(b.ready) != cudaSuccess))
+      continue;
+    best = (int)i;
+  }
   PlanBuffer buf;
   if (best >= 0) {
     buf = v->pool[best];
     v->pool.erase(v->pool.begin() + best);
+  } else if (v->pool.size() >= kMaxPooled) {   // bound the pool: wait for the oldest instead
+    buf = v->pool.front();
+    v->pool.erase(v->pool.begin());
+    if (buf.bytes < bytes) {
+      destroy_buffer(buf);
+      buf = PlanBuffer{};
+    }
   }
   return buf;
+}
+
+// Allocate a plan buffer of `bytes` (device copy, pinned staging copy, events).
+int alloc_buffer(size_t bytes, PlanBuffer* buf) {
+  buf->bytes = bytes;
+  const char* what = "cudaMalloc(plan)";
+  cudaError_t e = cudaMalloc(&buf->d, buf->bytes);
+  if (e == cudaSuccess) e = cudaMallocHost(&buf->h, buf->bytes), what = "cudaMallocHost(plan)";
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&buf->done, cudaEventDisableTiming), what = "cudaEventCreate";
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&buf->ready, cudaEventDisableTiming);
+  if (e != cudaSuccess) {
+    destroy_buffer(*buf);
+    *buf = PlanBuffer{};
+    return cuda_error(e, what);
+  }
+  return SAND_OK;
 }
 
 // Upload a built plan into buf (allocated here if empty) on the view's upload stream; runs on
@@ -302,20 +335,28 @@ int upload_plan(sand_view* v, EpochPlan& p, PlanBuffer* buf) {
   cudaError_t e = cudaSetDevice(v->store->device);
   if (e != cudaSuccess) return cuda_error(e, "cudaSetDevice");
   if (!buf->d) {
-    buf->bytes = L.total + L.total / 4;
-    const char* what = "cudaMalloc(plan)";
-    e = cudaMalloc(&buf->d, buf->bytes);
-    if (e == cudaSuccess) e = cudaMallocHost(&buf->h, buf->bytes), what = "cudaMallocHost(plan)";
-    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&buf->done, cudaEventDisableTiming), what = "cudaEventCreate";
-    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&buf->ready, cudaEventDisableTiming);
-    if (e != cudaSuccess) {
-      destroy_buffer(*buf);
-      *buf = PlanBuffer{};
-      return cuda_error(e, what);
+    // the first allocation also fills the pool with spares of the same size (+25 %): pinned and
+    // device allocations take driver locks and can stall the launching thread, so none happen
+    // once batches are being read
+    const size_t bytes = L.total + L.total / 4;
+    const int rc = alloc_buffer(bytes, buf);
+    if (rc != SAND_OK) return rc;
+    std::vector<PlanBuffer> spares;
+    {
+      std::lock_guard<std::mutex> lk(v->mu);
+      if (v->n_buffers == 0) spares.resize(kPrealloc);
+      v->n_buffers += 1 + spares.size();
     }
+    for (auto& b : spares)
+      if (alloc_buffer(bytes, &b) != SAND_OK) b = PlanBuffer{};
+    std::lock_guard<std::mutex> lk(v->mu);
+    for (auto& b : spares)
+      if (b.d) v->pool.push_back(b);
   } else {
+    const uint64_t w0 = now_ns();
     cudaEventSynchronize(buf->done);    // kernels of the previous owner finished
     cudaEventSynchronize(buf->ready);   // its upload no longer reads the staging copy
+    v->plan_buffer_wait_ns += now_ns() - w0;   // builder-side statistic (benign race)
   }
   auto* h = static_cast<uint8_t*>(buf->h);
   if (L.gb) std::memcpy(h, p.groups.data(), L.gb);
@@ -351,6 +392,7 @@ std::shared_ptr<EpochPlan> get_plan(sand_view* v, std::unique_lock<std::mutex>& 
       return it->second;
     }
     if (v->pending.count(key)) {
+      if (rc) v->pending_waits++;
       v->cv.wait(lk);
       continue;
     }
@@ -365,8 +407,10 @@ std::shared_ptr<EpochPlan> get_plan(sand_view* v, std::unique_lock<std::mutex>& 
   lk.unlock();
   const uint64_t t0 = now_ns();
   plan = build_plan(*v, epoch, rank, std::move(plan));
+  const uint64_t tb = now_ns();
   const PlanLayout L = plan_layout(*plan);
   lk.lock();
+  v->plan_cpu_ns += tb - t0;
   PlanBuffer buf = take_buffer(v, L.total);
   lk.unlock();
   const int urc = upload_plan(v, *plan, &buf);
@@ -488,6 +532,17 @@ extern "C" int sand_view_create(sand_store* s, const sand_view_spec* spec, sand_
     delete v;
     return sand::cuda_error(e, "cudaStreamCreate(upload)");
   }
+  // ticket counters of the persistent kernels: zero between launches (each launch's last CTA
+  // clears its slot); successive launches rotate through the slots
+  e = cudaMalloc(&v->d_sched, 2 * sand::kSchedSlots * sizeof(uint32_t));
+  if (e == cudaSuccess) e = cudaMemset(v->d_sched, 0, 2 * sand::kSchedSlots * sizeof(uint32_t));
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  if (e != cudaSuccess) {
+    if (v->d_sched) cudaFree(v->d_sched);
+    cudaStreamDestroy(v->upload_stream);
+    delete v;
+    return sand::cuda_error(e, "cudaMalloc(scheduler counters)");
+  }
   s->live_views++;
   const int n_workers = sand::env_int("SAND_PLAN_THREADS", 2, 1, 16);
   for (int i = 0; i < n_workers; ++i) v->workers.emplace_back(sand::worker_loop, v);
@@ -538,6 +593,7 @@ extern "C" int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank,
   auto stream = static_cast<cudaStream_t>(out->stream);
   const uint64_t t0 = sand::now_ns();
   std::unique_lock<std::mutex> lk(v->mu);
+  v->lock_wait_ns += sand::now_ns() - t0;
   int urc = SAND_OK;
   auto plan = sand::get_plan(v, lk, epoch, rank, &urc);
   const uint64_t t1 = sand::now_ns();
@@ -585,6 +641,9 @@ extern "C" int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank,
   lp.dests = plan->d_dests;
   lp.n_views = s.n_views;
   lp.batch = s.batch_size;
+  lp.sched = v->d_sched;
+  lp.sched_slot = v->sched_seq;   // launch_materialize uses slots sched_slot and sched_slot + 1
+  v->sched_seq = (v->sched_seq + 2) % sand::kSchedSlots;
   for (uint32_t k = 0; k < s.n_views; ++k) {
     lp.out[k] = out->data[k];
     lp.views[k] = v->vconst[k];
@@ -697,6 +756,10 @@ extern "C" int sand_view_get_stats(const sand_view* v, sand_view_stats* out) {
   out->plan_build_ns = v->plan_build_ns;
   out->plan_wait_ns = v->plan_wait_ns;
   out->read_ns = v->read_ns;
+  out->plan_cpu_ns = v->plan_cpu_ns;
+  out->plan_buffer_wait_ns = v->plan_buffer_wait_ns;
+  out->lock_wait_ns = v->lock_wait_ns;
+  out->pending_waits = v->pending_waits;
   return SAND_OK;
 }
 
@@ -713,6 +776,7 @@ extern "C" int sand_view_destroy(sand_view* v) {
   for (auto& kv : v->plans) sand::release_plan_device(v, *kv.second);
   sand::free_pool(v);
   if (v->upload_stream) cudaStreamDestroy(v->upload_stream);
+  if (v->d_sched) cudaFree(v->d_sched);
   v->store->live_views--;
   delete v;
   return SAND_OK;
