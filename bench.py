@@ -15,6 +15,7 @@ arm for this paper: SAND's own engine is CPU code) on the same config.
 from __future__ import annotations
 
 import argparse
+import gc
 import json
 import os
 import subprocess
@@ -280,6 +281,27 @@ def run_sand(args):
     # the library plans epoch e+1 on its worker when epoch e's first batch is read
     view.prefetch_epoch(0, rank)
 
+    # algorithmic bytes of the timed batches (host-side, before the warm-up so that the timed
+    # region follows the warm-up directly)
+    first_timed = args.warmup
+    sample = sorted({step_id(first_timed + i) for i in range(0, args.steps, max(1, args.steps // 16))})
+    bb = [view.batch_bytes(e, rank, it) for e, it in sample]
+    alg_read = sum(b.src_bytes for b in bb) / len(bb)
+    alg_write = sum(b.out_bytes for b in bb) / len(bb)
+
+    # clock sampling starts before the warm-up so the timed region follows the warm-up steps
+    # with no idle gap (an idle GPU drops to a low-power state and the first step pays for it)
+    kstart = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    kend = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    start = torch.cuda.Event(enable_timing=True)
+    end = torch.cuda.Event(enable_timing=True)
+    # no Python garbage collection from the warm-up to the end of the timed loop: a full
+    # collection stalls the launching thread for milliseconds, longer than the queued GPU work
+    gc.collect()
+    gc.disable()
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.2)
     s = 0
     for _ in range(args.warmup):
         e, it = step_id(s)
@@ -287,22 +309,9 @@ def run_sand(args):
         s += 1
     stream.synchronize()
 
-    # algorithmic bytes of the timed batches (host-side, outside the timed region)
     first_timed = s
-    sample = sorted({step_id(first_timed + i) for i in range(0, args.steps, max(1, args.steps // 16))})
-    bb = [view.batch_bytes(e, rank, it) for e, it in sample]
-    alg_read = sum(b.src_bytes for b in bb) / len(bb)
-    alg_write = sum(b.out_bytes for b in bb) / len(bb)
-
-    kstart = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    kend = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    start = torch.cuda.Event(enable_timing=True)
-    end = torch.cuda.Event(enable_timing=True)
     st0 = view.stats()
     launches0 = st0.kernel_launches
-    clocks = ClockSampler(local)
-    clocks.start()
-    time.sleep(0.2)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
@@ -315,6 +324,7 @@ def run_sand(args):
         s += 1
     end.record(stream)
     torch.cuda.synchronize()
+    gc.enable()
     if world > 1:
         dist.barrier()
     clk = clocks.stop()

@@ -118,6 +118,7 @@ struct sand_view {
   uint32_t* d_sched = nullptr;   // kSchedSlots pairs of ticket counters (persistent kernels)
   uint32_t sched_seq = 0;        // next slot pair
   size_t n_buffers = 0;          // plan buffers allocated so far
+  std::vector<cudaEvent_t> inflight;   // ring of per-batch completion events (read-ahead bound)
 };
 
 namespace sand {

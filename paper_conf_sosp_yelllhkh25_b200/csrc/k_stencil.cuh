@@ -140,6 +140,94 @@ __device__ __forceinline__ float2 rint2(float2 v) {
   return __fadd2_rn(__fadd2_rn(v, make_float2(rs::kRound, rs::kRound)), make_float2(-rs::kRound, -rs::kRound));
 }
 
+// Rotation (R#15) of all three Q2 planes in place. Q3 rows are computed band by band (one
+// row per warp) into a ring, and row r is written back over Q2 row r once no later Q3 row can
+// tap it: every tap of Q3 row y lies in Q2 rows [y - D, y + D]. Coordinates and fractions are
+// computed once per pixel for the three channels.
+__device__ __forceinline__ void rotate_inplace(const GroupParams& g, uint32_t q2, size_t plane, uint32_t ring,
+                                               int ring_rows, int D, int Wo, int Ho, int warp, int nwarps,
+                                               int lane, int tid, int nthr) {
+  using namespace rs;
+  const float rc = g.rot_c, rsn = g.rot_s, nrs = -g.rot_s;
+  const float cxo = (float)(Wo - 1) * 0.5f, cyo = (float)(Ho - 1) * 0.5f;
+  const uint32_t P = (uint32_t)plane, rplane = (uint32_t)(ring_rows * Wo);
+  int committed = 0;   // Q2 rows [0, committed) hold Q3 already
+  for (int yb = 0; yb < Ho; yb += nwarps) {
+    const int oy = yb + warp;
+    if (oy < Ho) {
+      const float yc = __fsub_rn((float)oy, cyo);
+      const uint64_t txy = f2::pack(__fmul_rn(nrs, yc), __fmul_rn(rc, yc));   // row terms
+      const uint32_t orow = ring + (uint32_t)((oy % ring_rows) * Wo);
+      for (int ox = lane; ox < Wo; ox += 32) {
+        const float xc = __fsub_rn((float)ox, cxo);
+        // (sx, sy) = ((c*xc + (-s)*yc) + cx, (s*xc + c*yc) + cy), every op rounded: scalar
+        // IEEE ops (ptxas contracts packed mul + add pairs into FFMA2, which rounds once)
+        const float sx = __fadd_rn(__fadd_rn(__fmul_rn(rc, xc), f2::lof(txy)), cxo);
+        const float sy = __fadd_rn(__fadd_rn(__fmul_rn(rsn, xc), f2::hif(txy)), cyo);
+        // floor without the XU pipe: t = s + 1.5*2^23 rounds s to the nearest integer n (exact
+        // for |s| < 2^22), whose low mantissa bits are n; one less where n > s
+        const uint64_t t = f2::add(f2::pack(sx, sy), f2::splat(kRound));
+        const uint64_t nf = f2::add(t, f2::splat(-kRound));
+        const bool gx = f2::lof(nf) > sx, gy = f2::hif(nf) > sy;
+        const float fx = gx ? __fadd_rn(f2::lof(nf), -1.f) : f2::lof(nf);
+        const float fy = gy ? __fadd_rn(f2::hif(nf), -1.f) : f2::hif(nf);
+        const uint64_t l = f2::add(f2::pack(sx, sy), f2::pack(-fx, -fy));   // (lambda_x, lambda_y), exact
+        const int x0 = (int)(f2::lo(t) - 0x4B400000u) - (gx ? 1 : 0);
+        const int y0 = (int)(f2::hi(t) - 0x4B400000u) - (gy ? 1 : 0);
+        const uint64_t lx = f2::splat(f2::lof(l));
+        const float ly = f2::hif(l);
+        const bool inside = (unsigned)x0 < (unsigned)(Wo - 1) && (unsigned)y0 < (unsigned)(Ho - 1);
+        const uint32_t a0 = q2 + (uint32_t)(y0 * Wo + x0);
+        const bool in00 = x0 >= 0 && x0 < Wo && y0 >= 0 && y0 < Ho, in01 = x0 + 1 >= 0 && x0 + 1 < Wo && y0 >= 0 && y0 < Ho;
+        const bool in10 = x0 >= 0 && x0 < Wo && y0 + 1 >= 0 && y0 + 1 < Ho;
+        const bool in11 = x0 + 1 >= 0 && x0 + 1 < Wo && y0 + 1 >= 0 && y0 + 1 < Ho;
+#pragma unroll
+        for (int c = 0; c < 3; ++c) {
+          const uint32_t a = a0 + (uint32_t)c * P;
+          uint32_t b00, b01, b10, b11;   // taps outside the image read 0 (fill=None)
+          if (inside) {
+            b00 = ldsu8(a);
+            b01 = ldsu8(a + 1);
+            b10 = ldsu8(a + (uint32_t)Wo);
+            b11 = ldsu8(a + (uint32_t)Wo + 1);
+          } else {
+            b00 = in00 ? ldsu8(a) : 0u;
+            b01 = in01 ? ldsu8(a + 1) : 0u;
+            b10 = in10 ? ldsu8(a + (uint32_t)Wo) : 0u;
+            b11 = in11 ? ldsu8(a + (uint32_t)Wo + 1) : 0u;
+          }
+          // rows packed: (t00, t10) and (t01, t11) as biased floats 2^23 + t
+          const uint64_t T0 = f2::pack(0x4B000000u | b00, 0x4B000000u | b10);
+          const uint64_t T1 = f2::pack(0x4B000000u | b01, 0x4B000000u | b11);
+          const uint64_t d = f2::fma(T0, f2::splat(-1.f), T1);          // (t01 - t00, t11 - t10)
+          const uint64_t h = f2::fma(lx, d, f2::add(T0, f2::splat(-kBias)));   // (h0, h1)
+          const float h0 = f2::lof(h), h1 = f2::hif(h);
+          const float tq = __fadd_rn(__fmaf_rn(ly, __fsub_rn(h1, h0), h0), kRound);   // rint -> low byte
+          stsu8(orow + (uint32_t)c * rplane + (uint32_t)ox, __float_as_uint(tq) & 0xffu);
+        }
+      }
+    }
+    __syncthreads();                     // ring rows of this band written; Q2 reads done
+    const int last = min(yb + nwarps, Ho) - 1;
+    const int upto = last + 1 >= Ho ? Ho : max(committed, last - D + 1);   // rows < upto are dead in Q2
+    const int n = upto - committed;
+    if (n > 0) {                         // write back Q3 rows [committed, upto) of the three planes
+      for (int rr = warp; rr < 3 * n; rr += nwarps) {
+        const int c = rr / n, row = committed + rr - c * n;
+        const uint32_t from = ring + (uint32_t)c * rplane + (uint32_t)((row % ring_rows) * Wo);
+        const uint32_t to = q2 + (uint32_t)c * P + (uint32_t)(row * Wo);
+        if ((Wo & 3) == 0) {
+          for (int x = 4 * lane; x < Wo; x += 128) sts32(to + (uint32_t)x, st::lds32(from + (uint32_t)x));
+        } else {
+          for (int x = lane; x < Wo; x += 32) stsu8(to + (uint32_t)x, ldsu8(from + (uint32_t)x));
+        }
+      }
+      committed = upto;
+    }
+    __syncthreads();
+  }
+}
+
 constexpr int kBX = 8;        // blur: outputs per thread along the blocked axis
 
 // Separable Gaussian blur of one channel plane with radius R (R#16): horizontal pass into
@@ -151,6 +239,16 @@ __device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupPar
   const int pairs = (Wo + 1) >> 1;
   const int strip_rows = (int)(plane / ((size_t)Wo * 4));   // fp32 rows the scratch holds
   const int S = strip_rows - 2 * R;
+  // taps in registers (loaded once; the shared-memory stores below must not force reloads)
+  float wt[2 * R + 1];
+#pragma unroll
+  for (int i = 0; i <= 2 * R; ++i) wt[i] = __ldg(&g.blur_w[i]);
+  // word-aligned rows: interior blocks load their window as 32-bit words (the window's byte
+  // misalignment (-R) & 3 is a compile-time constant) and store 16 B per 4 columns
+  const bool words = (Wo & 3) == 0;
+  constexpr int kOff = (4 - (R & 3)) & 3;                 // (x0 - R) & 3 for x0 % 8 == 0
+  constexpr int kWin = kBX + 2 * R;
+  constexpr int kWords = (kOff + kWin + 3) / 4;
   for (int ys = 0; ys < Ho; ys += S) {
     const int ns = min(S, Ho - ys);
     const int jrows = ns + 2 * R;          // strip row j <-> image row reflect(ys - R + j)
@@ -163,63 +261,102 @@ __device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupPar
       const uint32_t rowa = src + (uint32_t)(reflect(ys - R + ja2, Ho) * Wo);
       const uint32_t rowb = src + (uint32_t)(reflect(ys - R + jb2, Ho) * Wo);
       const int x0 = xb * kBX;
-      float2 win[kBX + 2 * R];
+      // Window element k feeds outputs o = k - i for taps i; iterating k upwards and updating
+      // every output it feeds keeps each output's taps in order i = 0..2R (R#16), while only
+      // one converted element is live at a time.
+      uint64_t accs[kBX];
+#pragma unroll
+      for (int o = 0; o < kBX; ++o) accs[o] = 0ull;
+      auto feed = [&](int k, uint64_t v) {
+#pragma unroll
+        for (int o = 0; o < kBX; ++o)
+          if (k - o >= 0 && k - o <= 2 * R) accs[o] = rs::f2::fma(rs::f2::splat(wt[k - o]), v, accs[o]);
+      };
       const bool interior = x0 - R >= 0 && x0 + kBX - 1 + R < Wo;
+      if (interior && words) {
+        const uint32_t wb = (uint32_t)(x0 - R - kOff);   // 4-aligned
+        uint32_t wa[kWords], wbv[kWords];
 #pragma unroll
-      for (int k = 0; k < kBX + 2 * R; ++k) {
-        const int xx = interior ? x0 - R + k : reflect(min(x0 - R + k, 2 * Wo - 2), Wo);
-        win[k] = make_float2(u8f(ldsu8(rowa + (uint32_t)xx)), u8f(ldsu8(rowb + (uint32_t)xx)));
+        for (int k = 0; k < kWords; ++k) {
+          wa[k] = st::lds32(rowa + wb + 4u * k);
+          wbv[k] = st::lds32(rowb + wb + 4u * k);
+        }
+#pragma unroll
+        for (int k = 0; k < kWin; ++k) {
+          const int bi = kOff + k;
+          // biased floats 2^23 + byte of both rows, then one packed subtract
+          const uint32_t fa = __byte_perm(wa[bi >> 2], 0x4B000000u, 0x7440 | (bi & 3));
+          const uint32_t fb = __byte_perm(wbv[bi >> 2], 0x4B000000u, 0x7440 | (bi & 3));
+          feed(k, rs::f2::add(rs::f2::pack(fa, fb), rs::f2::splat(-rs::kBias)));
+        }
+      } else {
+#pragma unroll
+        for (int k = 0; k < kWin; ++k) {
+          const int xx = reflect(min(x0 - R + k, 2 * Wo - 2), Wo);
+          feed(k, rs::f2::pack(u8f(ldsu8(rowa + (uint32_t)xx)), u8f(ldsu8(rowb + (uint32_t)xx))));
+        }
       }
-      float2 accs[kBX];
+      if (words && x0 + kBX <= Wo) {               // 16 B stores: 4 columns of one strip row
 #pragma unroll
-      for (int o = 0; o < kBX; ++o) accs[o] = make_float2(0.f, 0.f);
+        for (int o = 0; o < kBX; o += 4) {
+          st::sts128(scratch + 4u * (uint32_t)(ja2 * Wo + x0 + o),
+                     make_uint4(rs::f2::lo(accs[o]), rs::f2::lo(accs[o + 1]), rs::f2::lo(accs[o + 2]),
+                                rs::f2::lo(accs[o + 3])));
+          st::sts128(scratch + 4u * (uint32_t)(jb2 * Wo + x0 + o),
+                     make_uint4(rs::f2::hi(accs[o]), rs::f2::hi(accs[o + 1]), rs::f2::hi(accs[o + 2]),
+                                rs::f2::hi(accs[o + 3])));
+        }
+      } else {
 #pragma unroll
-      for (int i = 0; i <= 2 * R; ++i) {           // taps in order: acc = fmaf(w_i, v, acc)
-        const float wi = g.blur_w[i];
-#pragma unroll
-        for (int o = 0; o < kBX; ++o) accs[o] = __ffma2_rn(make_float2(wi, wi), win[o + i], accs[o]);
-      }
-#pragma unroll
-      for (int o = 0; o < kBX; ++o) {
-        const float2 acc = accs[o];
-        if (x0 + o < Wo) {
-          asm volatile("st.shared.f32 [%0], %1;" ::"r"(scratch + 4u * (uint32_t)(ja2 * Wo + x0 + o)), "f"(acc.x)
-                       : "memory");
-          asm volatile("st.shared.f32 [%0], %1;" ::"r"(scratch + 4u * (uint32_t)(jb2 * Wo + x0 + o)), "f"(acc.y)
-                       : "memory");
+        for (int o = 0; o < kBX; ++o) {
+          if (x0 + o < Wo) {
+            sts32(scratch + 4u * (uint32_t)(ja2 * Wo + x0 + o), rs::f2::lo(accs[o]));
+            sts32(scratch + 4u * (uint32_t)(jb2 * Wo + x0 + o), rs::f2::hi(accs[o]));
+          }
         }
       }
     }
     __syncthreads();
-    // vertical pass: thread = column pair (x, x+1) x block of kBX output rows
-    const int rblocks = (ns + kBX - 1) / kBX;
+    // vertical pass: thread = column pair (x, x+1) x block of kBV output rows; window rows
+    // feed the outputs in tap order as in the horizontal pass
+    constexpr int kBV = 16;
+    const int rblocks = (ns + kBV - 1) / kBV;
     for (int e = tid; e < pairs * rblocks; e += nthr) {
       const int rb = e / pairs, pr2 = e - rb * pairs;
-      const int ox = 2 * pr2, y0 = rb * kBX;
+      const int ox = 2 * pr2, y0 = rb * kBV;
       const bool has_b = ox + 1 < Wo;
-      float2 win[kBX + 2 * R];
+      uint64_t accs[kBV];
 #pragma unroll
-      for (int k = 0; k < kBX + 2 * R; ++k) {
-        win[k] = make_float2(0.f, 0.f);
-        if (y0 + k < jrows) {
-          const uint32_t a = scratch + 4u * (uint32_t)((y0 + k) * Wo + ox);
-          win[k] = has_b && !(Wo & 1) ? lds64f(a) : make_float2(__uint_as_float(st::lds32(a)),
-                                                                  has_b ? __uint_as_float(st::lds32(a + 4)) : 0.f);
+      for (int o = 0; o < kBV; ++o) accs[o] = 0ull;
+      auto feed = [&](int k, uint64_t v) {
+#pragma unroll
+        for (int o = 0; o < kBV; ++o)
+          if (k - o >= 0 && k - o <= 2 * R) accs[o] = rs::f2::fma(rs::f2::splat(wt[k - o]), v, accs[o]);
+      };
+      const uint32_t a0 = scratch + 4u * (uint32_t)(y0 * Wo + ox);
+      const uint32_t rstep = 4u * (uint32_t)Wo;
+      if (has_b && !(Wo & 1) && y0 + kBV + 2 * R <= jrows) {
+#pragma unroll
+        for (int k = 0; k < kBV + 2 * R; ++k) {
+          const float2 v = lds64f(a0 + rstep * k);
+          feed(k, rs::f2::pack(v.x, v.y));
+        }
+      } else {
+#pragma unroll
+        for (int k = 0; k < kBV + 2 * R; ++k) {
+          uint64_t v = 0ull;
+          if (y0 + k < jrows) {
+            const uint32_t a = a0 + rstep * k;
+            v = rs::f2::pack(st::lds32(a), has_b ? st::lds32(a + 4) : 0u);
+          }
+          feed(k, v);
         }
       }
-      float2 accs[kBX];
 #pragma unroll
-      for (int o = 0; o < kBX; ++o) accs[o] = make_float2(0.f, 0.f);
-#pragma unroll
-      for (int i = 0; i <= 2 * R; ++i) {
-        const float wi = g.blur_w[i];
-#pragma unroll
-        for (int o = 0; o < kBX; ++o) accs[o] = __ffma2_rn(make_float2(wi, wi), win[o + i], accs[o]);
-      }
-#pragma unroll
-      for (int o = 0; o < kBX; ++o) {
+      for (int o = 0; o < kBV; ++o) {
         if (y0 + o >= ns) break;
-        store_q<DT, VEC>(p, cd, ys + y0 + o, ox, Wo, rint2(accs[o]), has_b);
+        store_q<DT, VEC>(p, cd, ys + y0 + o, ox, Wo, rint2(make_float2(rs::f2::lof(accs[o]), rs::f2::hif(accs[o]))),
+                         has_b);
       }
     }
     __syncthreads();
@@ -343,6 +480,17 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
   // ------------------------------------------------------------- phase 2: per channel
   const int r = g.blur_on ? g.blur_r : 0;
   const float cxo = (float)(Wo - 1) * 0.5f, cyo = (float)(Ho - 1) * 0.5f;
+  // a8 in place for all three channels when its ring fits the band/Q3 region; else per channel
+  bool rotated = false;
+  if (g.rot_on) {
+    const float bound = fabsf(g.rot_s) * cxo + (1.f - g.rot_c) * cyo;
+    const int D = (int)ceilf(bound) + 2;
+    const int ring_rows = D + nwarps + 1;
+    if ((size_t)ring_rows * 3 * Wo <= sh.ubytes && D < Ho) {
+      rotate_inplace(g, q2, sh.plane, ureg, ring_rows, D, Wo, Ho, warp, nwarps, lane, tid, nthr);
+      rotated = true;
+    }
+  }
   for (int c = 0; c < 3; ++c) {
     ChDests cd;
     cd.nd = nd;
@@ -352,7 +500,8 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
     if (nd > 1) cd.d1 = ch_dest(p, dests[1], c);
     uint32_t src = q2 + (uint32_t)(c * sh.plane);
     uint32_t scratch = ureg;
-    if (g.rot_on) {                            // a8: Q3 = rotate(Q2) (R#15)
+    size_t scratch_bytes = sh.ubytes;
+    if (g.rot_on && !rotated) {                // a8: Q3 = rotate(Q2) (R#15), one channel
       const uint32_t q3 = ureg;
       const float rc = g.rot_c, rsn = g.rot_s, nrs = -g.rot_s;
       for (int oy = warp; oy < Ho; oy += nwarps) {
@@ -393,21 +542,22 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
       __syncthreads();
       src = q3;
       scratch = q2 + (uint32_t)(c * sh.plane);   // this channel's Q2 plane is free now
+      scratch_bytes = sh.plane;
     }
     if (g.blur_on) {                           // a9: separable Gaussian in strips (R#16)
       switch (r) {
-        case 0: blur_plane<DT, VEC, 0>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 1: blur_plane<DT, VEC, 1>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 2: blur_plane<DT, VEC, 2>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 3: blur_plane<DT, VEC, 3>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 4: blur_plane<DT, VEC, 4>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 5: blur_plane<DT, VEC, 5>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 6: blur_plane<DT, VEC, 6>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 7: blur_plane<DT, VEC, 7>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 8: blur_plane<DT, VEC, 8>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 9: blur_plane<DT, VEC, 9>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        case 10: blur_plane<DT, VEC, 10>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
-        default: blur_plane<DT, VEC, 11>(p, g, cd, src, scratch, sh.plane, Wo, Ho, tid, nthr); break;
+        case 0: blur_plane<DT, VEC, 0>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;
+        case 1: blur_plane<DT, VEC, 1>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;
+        case 2: blur_plane<DT, VEC, 2>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;
+        case 3: blur_plane<DT, VEC, 3>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;
+        case 4: blur_plane<DT, VEC, 4>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;
+        case 5: blur_plane<DT, VEC, 5>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;
+        case 6: blur_plane<DT, VEC, 6>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;
+        case 7: blur_plane<DT, VEC, 7>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;
+        case 8: blur_plane<DT, VEC, 8>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;
+        case 9: blur_plane<DT, VEC, 9>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;
+        case 10: blur_plane<DT, VEC, 10>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;
+        default: blur_plane<DT, VEC, 11>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;
       }
     } else {                                   // no blur: normalise + store the (rotated) plane
       for (int oy = warp; oy < Ho; oy += nwarps) {

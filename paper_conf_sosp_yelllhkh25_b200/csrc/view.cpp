@@ -25,6 +25,7 @@ constexpr size_t kMaxPooled = 8;   // idle plan buffers kept for reuse
 constexpr size_t kPrealloc = 6;    // spare plan buffers allocated with the first one
 }  // namespace
 constexpr uint64_t kPlanAhead = 2;
+constexpr uint64_t kInflight = 48;   // batches of one view queued on the GPU at most
 namespace {
 constexpr double kPi = 3.14159265358979323846;
 
@@ -633,6 +634,23 @@ extern "C" int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank,
       }
     }
   }
+  // bound the read-ahead: at most kInflight batches of this view are queued on the GPU. An
+  // unbounded run-ahead keeps many epoch plans alive at once (more plan buffers, allocations
+  // and driver locks while batches are being read) for no gain.
+  const size_t slot = static_cast<size_t>(v->batches % sand::kInflight);
+  if (v->inflight.empty()) {
+    v->inflight.resize(sand::kInflight, nullptr);
+    for (auto& ev : v->inflight) {
+      e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming);
+      if (e != cudaSuccess) return sand::cuda_error(e, "cudaEventCreate(inflight)");
+    }
+  }
+  if (v->batches >= sand::kInflight) {
+    lk.unlock();
+    e = cudaEventSynchronize(v->inflight[slot]);
+    lk.lock();
+    if (e != cudaSuccess) return sand::cuda_error(e, "cudaEventSynchronize(inflight)");
+  }
   sand::LaunchParams lp{};
   lp.slab = st->slab;
   lp.items = plan->d_items + ib;
@@ -652,6 +670,7 @@ extern "C" int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank,
   int rc = sand::launch_materialize(lp, plan->shapes[it], v->stencil_smem, stream, &launched);
   if (rc != SAND_OK) return rc;
   e = cudaEventRecord(plan->last_use, stream);
+  if (e == cudaSuccess) e = cudaEventRecord(v->inflight[slot], stream);
   if (e != cudaSuccess) return sand::cuda_error(e, "cudaEventRecord");
   {
     std::lock_guard<std::mutex> slk(st->mu);
@@ -777,6 +796,8 @@ extern "C" int sand_view_destroy(sand_view* v) {
   sand::free_pool(v);
   if (v->upload_stream) cudaStreamDestroy(v->upload_stream);
   if (v->d_sched) cudaFree(v->d_sched);
+  for (auto& ev : v->inflight)
+    if (ev) cudaEventDestroy(ev);
   v->store->live_views--;
   delete v;
   return SAND_OK;
