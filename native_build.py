@@ -57,7 +57,8 @@ def build_oracle(force=False):
 
 PRODUCT_CPP = ["sand_api.cpp", "store.cpp", "planner.cpp", "view.cpp"]
 PRODUCT_CU = ["materialize.cu"]
-PRODUCT_HDR = ["internal.h", "plan_types.h", "planner.h", "k_resample.cuh", "k_stream.cuh", "k_stencil.cuh"]
+PRODUCT_HDR = ["internal.h", "plan_types.h", "planner.h", "k_resample.cuh", "k_stream.cuh", "k_stencil.cuh",
+               "k_direct.cuh"]
 
 
 def build_product(force=False, variant=None, defines=()):

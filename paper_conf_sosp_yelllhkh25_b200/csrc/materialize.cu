@@ -174,6 +174,7 @@ __global__ void __launch_bounds__(512) k_stencil(const LaunchParams p) {
 #include "k_resample.cuh"
 #include "k_stream.cuh"
 #include "k_stencil.cuh"
+#include "k_direct.cuh"
 
 namespace sand {
 
@@ -188,7 +189,7 @@ size_t smem_budget() {
 }
 
 struct ResampleCfg {
-  int mode;         // 0 gather, 1 raw bands, 2 stream
+  int mode;         // 0 gather, 1 raw bands, 2 stream, 3 direct
   int R;
   size_t smem;
   st::Shape st;
@@ -227,6 +228,7 @@ ResampleCfg choose_resample(const BatchShape& sh) {
       if (bytes <= smem_budget() || (r <= 8 && bytes <= 200 * 1024)) return {1, r, bytes, {}};
     }
   }
+  if (forced != 0) return {3, env_int("SAND_DIRECT_RB", 32), 0, {}};   // heavy down-scaling: direct gather
   for (int r : kCands) {
     const int span = (int)std::ceil((double)sh.max_scy * r) + 3;
     const size_t rows = (size_t)std::min(2 * r, span);
@@ -291,6 +293,14 @@ int launch_resample_dt(const LaunchParams& p, const BatchShape& sh, cudaStream_t
     return SAND_OK;
   }
   const int nbands = (sh.max_ho + cfg.R - 1) / cfg.R;
+  if (cfg.mode == 3) {
+    const int threads = std::min(128, ((pairs + 31) / 32) * 32);
+    const unsigned blocks = (unsigned)((uint64_t)p.n_items * nbands);
+    k_direct<DT, VEC><<<blocks, threads, 0, stream>>>(p, cfg.R, nbands);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_error(e, "k_direct launch");
+    return SAND_OK;
+  }
   const int threads = std::min(224, ((2 * pairs + 31) / 32) * 32);
   const unsigned blocks = (unsigned)((uint64_t)p.n_items * nbands);
   if (cfg.mode == 1)
