@@ -16,54 +16,54 @@
 namespace sand {
 namespace dg {
 
-// NV12 pixel x of a row pair (Y row, UV row) as an RGBx word
-__device__ __forceinline__ uint32_t pixel(const uint8_t* __restrict__ yrow, const uint8_t* __restrict__ uvrow, int x) {
-  const uint32_t Y = __ldg(yrow + x);
-  const uint32_t uv = __ldg(reinterpret_cast<const uint16_t*>(uvrow + (x & ~1)));
-  return st::rgbx_dpx(Y, st::chroma_at<0>(uv));
+// One NV12 pixel as three biased floats 2^23 + channel (R#11): the OpenCV integer BT.601
+// value sat((yy + term) >> 20) is relu(min(yy + term, 2^28 - 1)) >> 20 (one DPX add-min-relu),
+// and the shift plus the 0x4B exponent byte are one IMAD.HI with addend; no byte packing.
+struct Px3 {
+  uint32_t c[3];
+};
+__device__ __forceinline__ Px3 px3(uint32_t Y, uint32_t uv) {
+  const st::Chroma3 k = st::chroma_at<0>(uv);
+  const int yy = (int)max(Y, 16u) * 1220542 + ((1 << 19) - 16 * 1220542);
+  Px3 p;
+  p.c[0] = __umulhi((uint32_t)__viaddmin_s32_relu(yy, k.r, 0x0FFFFFFF), 1u << 12) + 0x4B000000u;
+  p.c[1] = __umulhi((uint32_t)__viaddmin_s32_relu(yy, k.g, 0x0FFFFFFF), 1u << 12) + 0x4B000000u;
+  p.c[2] = __umulhi((uint32_t)__viaddmin_s32_relu(yy, k.b, 0x0FFFFFFF), 1u << 12) + 0x4B000000u;
+  return p;
 }
 
-// horizontal lerps of source row y at the thread's four taps (R#12)
-__device__ __forceinline__ void hrow(rs::Row3& r, const uint8_t* __restrict__ Yp, const uint8_t* __restrict__ UVp,
-                                     uint32_t pitch, int y, int xa0, int xa1, int xb0, int xb1, uint64_t lx) {
-  const uint8_t* yrow = Yp + (size_t)y * pitch;
-  const uint8_t* uvrow = UVp + (size_t)(y >> 1) * pitch;
-  const uint32_t a0 = pixel(yrow, uvrow, xa0), a1 = pixel(yrow, uvrow, xa1);
-  const uint32_t b0 = pixel(yrow, uvrow, xb0), b1 = pixel(yrow, uvrow, xb1);
-  r.h[0] = rs::hlerp<0>(a0, a1, b0, b1, lx);
-  r.h[1] = rs::hlerp<1>(a0, a1, b0, b1, lx);
-  r.h[2] = rs::hlerp<2>(a0, a1, b0, b1, lx);
+// horizontal lerp of channel values given as biased floats, both columns packed (R#12)
+__device__ __forceinline__ uint64_t hlerp_b(uint32_t a0, uint32_t a1, uint32_t b0, uint32_t b1, uint64_t lx) {
+  const uint64_t P0 = rs::f2::pack(a0, b0), P1 = rs::f2::pack(a1, b1);
+  const uint64_t d = rs::f2::fma(P0, rs::f2::splat(-1.f), P1);     // p1 - p0 (exact)
+  return rs::f2::fma(lx, d, rs::f2::add(P0, rs::f2::splat(-rs::kBias)));   // fmaf(l, p1 - p0, p0)
 }
 
-// both source rows of an output row at once: the sixteen loads are issued before any
-// conversion so their latencies overlap
-__device__ __forceinline__ void hrow2(rs::Row3& t, rs::Row3& b, const uint8_t* __restrict__ Yp,
-                                      const uint8_t* __restrict__ UVp, uint32_t pitch, int y0, int y1, int xa0,
-                                      int xa1, int xb0, int xb1, uint64_t lx) {
-  const uint8_t* yr[2] = {Yp + (size_t)y0 * pitch, Yp + (size_t)y1 * pitch};
-  const uint8_t* uvr[2] = {UVp + (size_t)(y0 >> 1) * pitch, UVp + (size_t)(y1 >> 1) * pitch};
+// horizontal lerps of the source rows of `nr` (1 or 2) rows at the thread's four taps; all
+// loads are issued before any conversion so their latencies overlap
+template <int NR>
+__device__ __forceinline__ void hrows(rs::Row3* out, const uint8_t* __restrict__ Yp, const uint8_t* __restrict__ UVp,
+                                      uint32_t pitch, const int (&ys)[2], int xa0, int xa1, int xb0, int xb1,
+                                      uint64_t lx) {
   const int xs[4] = {xa0, xa1, xb0, xb1};
-  uint32_t Y[2][4], UV[2][4];
+  uint32_t Y[NR][4], UV[NR][4];
 #pragma unroll
-  for (int r = 0; r < 2; ++r)
+  for (int r = 0; r < NR; ++r) {
+    const uint8_t* yr = Yp + (size_t)ys[r] * pitch;
+    const uint8_t* uvr = UVp + (size_t)(ys[r] >> 1) * pitch;
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
-      Y[r][k] = __ldg(yr[r] + xs[k]);
-      UV[r][k] = __ldg(reinterpret_cast<const uint16_t*>(uvr[r] + (xs[k] & ~1)));
+      Y[r][k] = __ldg(yr + xs[k]);
+      UV[r][k] = __ldg(reinterpret_cast<const uint16_t*>(uvr + (xs[k] & ~1)));
     }
-  uint32_t q[2][4];
+  }
 #pragma unroll
-  for (int r = 0; r < 2; ++r)
+  for (int r = 0; r < NR; ++r) {
+    Px3 q[4];
 #pragma unroll
-    for (int k = 0; k < 4; ++k) q[r][k] = st::rgbx_dpx(Y[r][k], st::chroma_at<0>(UV[r][k]));
+    for (int k = 0; k < 4; ++k) q[k] = px3(Y[r][k], UV[r][k]);
 #pragma unroll
-  for (int c = 0; c < 3; ++c) {
-    t.h[c] = c == 0 ? rs::hlerp<0>(q[0][0], q[0][1], q[0][2], q[0][3], lx)
-                    : (c == 1 ? rs::hlerp<1>(q[0][0], q[0][1], q[0][2], q[0][3], lx)
-                              : rs::hlerp<2>(q[0][0], q[0][1], q[0][2], q[0][3], lx));
-    b.h[c] = c == 0 ? rs::hlerp<0>(q[1][0], q[1][1], q[1][2], q[1][3], lx)
-                    : (c == 1 ? rs::hlerp<1>(q[1][0], q[1][1], q[1][2], q[1][3], lx)
-                              : rs::hlerp<2>(q[1][0], q[1][1], q[1][2], q[1][3], lx));
+    for (int c = 0; c < 3; ++c) out[r].h[c] = hlerp_b(q[0].c[c], q[1].c[c], q[2].c[c], q[3].c[c], lx);
   }
 }
 
@@ -113,8 +113,12 @@ __global__ void __launch_bounds__(128, 5) k_direct(const LaunchParams p, int RB,
       int y0, y1;
       float ly;
       tap(g.sc_y, g.off_y, oy0 + rr, g.lim_y, g.org_y, y0, y1, ly);
+      const int ys2[2] = {y0, y1};
       if (y0 != yT && y0 != yB && y1 != yB && y1 != y0) {   // both rows new (the usual case)
-        dg::hrow2(T, B, Yp, UVp, pitch, y0, y1, xa0, xa1, xb0, xb1, lx);
+        Row3 tb[2];
+        dg::hrows<2>(tb, Yp, UVp, pitch, ys2, xa0, xa1, xb0, xb1, lx);
+        T = tb[0];
+        B = tb[1];
         yT = y0;
         yB = y1;
       }
@@ -122,13 +126,17 @@ __global__ void __launch_bounds__(128, 5) k_direct(const LaunchParams p, int RB,
         if (y0 == yB) {
           T = B;
         } else {
-          dg::hrow(T, Yp, UVp, pitch, y0, xa0, xa1, xb0, xb1, lx);
+          dg::hrows<1>(&T, Yp, UVp, pitch, ys2, xa0, xa1, xb0, xb1, lx);
         }
         yT = y0;
       }
       if (y1 != yB) {
-        if (y1 == yT) B = T;
-        else dg::hrow(B, Yp, UVp, pitch, y1, xa0, xa1, xb0, xb1, lx);
+        if (y1 == yT) {
+          B = T;
+        } else {
+          const int ys1[2] = {y1, y1};
+          dg::hrows<1>(&B, Yp, UVp, pitch, ys1, xa0, xa1, xb0, xb1, lx);
+        }
         yB = y1;
       }
       emit<DT, kInlineDests, VEC>(T, B, ly, dl, dt, p, dests, nd, oy0 + rr, ox, vec, has_b);
