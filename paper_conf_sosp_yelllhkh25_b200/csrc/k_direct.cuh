@@ -69,26 +69,37 @@ __device__ __forceinline__ void hrows(rs::Row3* out, const uint8_t* __restrict__
 
 }  // namespace dg
 
-// One CTA = one work item x one band of RB output rows; thread = output column pair.
+// One CTA = one work item x one band of RB output rows x one chunk of P column pairs; the
+// band is split into two halves and thread t = (half t / P, column pair chunk * P + t % P),
+// so P = 112 gives 224 threads (seven full warps) for 224-wide outputs.
+#ifndef SAND_DIRECT_MINB
+#define SAND_DIRECT_MINB 3
+#endif
 template <int DT, bool VEC>
-__global__ void __launch_bounds__(128, 5) k_direct(const LaunchParams p, int RB, int nbands) {
+__global__ void __launch_bounds__(256, SAND_DIRECT_MINB) k_direct(const LaunchParams p, int RB, int nbands, int nchunks) {
   using namespace rs;
-  const int item_idx = blockIdx.x / nbands;
-  const int band = blockIdx.x - item_idx * nbands;
+  const int item_idx = blockIdx.x / (nbands * nchunks);
+  const int rest = blockIdx.x - item_idx * (nbands * nchunks);
+  const int band = rest / nchunks, chunk = rest - band * nchunks;
   const WorkItem w = p.items[item_idx];
   if (w.flags & 1u) return;
   const GroupParams& g = p.groups[w.gp];
   const int Wo = g.out_w, Ho = g.out_h;
-  const int oy0 = band * RB;
-  if (oy0 >= Ho) return;
-  const int nr = min(RB, Ho - oy0);
+  const int pairs = (Wo + 1) >> 1;
+  const int P = (int)blockDim.x >> 1;                  // threads per half-band
+  const int half = (int)threadIdx.x >= P ? 1 : 0;
+  const int pair = chunk * P + (int)threadIdx.x - half * P;
+  const int hb = (RB + 1) >> 1;
+  const int oy0 = band * RB + half * hb;
+  const int band_end = min(Ho, band * RB + RB);
+  if (oy0 >= band_end || pair >= pairs) return;
+  const int nr = min(hb, band_end - oy0);
   const uint8_t* Yp = p.slab + w.y_off;
   const uint8_t* UVp = Yp + (size_t)w.pitch * w.src_h;
   const uint32_t pitch = w.pitch;
   const int nd = (int)w.n_dest;
   const uint32_t* dests = p.dests + w.dest_begin;
-  const int pairs = (Wo + 1) >> 1;
-  for (int pair = threadIdx.x; pair < pairs; pair += blockDim.x) {
+  {
     const int ox = 2 * pair;
     const bool has_b = ox + 1 < Wo;
     const bool vec = has_b && !(Wo & 1);

@@ -27,6 +27,7 @@ struct Shape {
   int grid_rows;    // grid / raw capacity in rows per band
   size_t plane;     // bytes of one uint8 plane (Ho*Wo, 16-aligned)
   size_t ubytes;    // bytes of the shared band/Q3 region
+  int skip;         // profiling only (SAND_STENCIL_SKIP): bit0 rotation, bit1 blur, bit2 Q2 walk
 };
 
 __host__ __device__ inline size_t band_bytes(int maxWo, int R, int grid_rows, int gw) {
@@ -425,7 +426,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
     __syncthreads();
     st::convert_rows(s_grid, s_rawb, gw, y_lo, y_hi, y_lo, 1 << 30, 5u, warp, nwarps, lane);   // no wrap
     __syncthreads();
-    if (grp < groups && pr < pairs) {
+    if (grp < groups && pr < pairs && !(sh.skip & 4)) {
       const int ox = 2 * pr;
       const bool has_b = ox + 1 < Wo;
       const int ja = g.flip ? Wo - 1 - ox : ox;
@@ -482,7 +483,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
   const float cxo = (float)(Wo - 1) * 0.5f, cyo = (float)(Ho - 1) * 0.5f;
   // a8 in place for all three channels when its ring fits the band/Q3 region; else per channel
   bool rotated = false;
-  if (g.rot_on) {
+  if (g.rot_on && !(sh.skip & 1)) {
     const float bound = fabsf(g.rot_s) * cxo + (1.f - g.rot_c) * cyo;
     const int D = (int)ceilf(bound) + 2;
     const int ring_rows = D + nwarps + 1;
@@ -501,7 +502,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
     uint32_t src = q2 + (uint32_t)(c * sh.plane);
     uint32_t scratch = ureg;
     size_t scratch_bytes = sh.ubytes;
-    if (g.rot_on && !rotated) {                // a8: Q3 = rotate(Q2) (R#15), one channel
+    if (g.rot_on && !rotated && !(sh.skip & 1)) {              // a8: Q3 = rotate(Q2) (R#15), one channel
       const uint32_t q3 = ureg;
       const float rc = g.rot_c, rsn = g.rot_s, nrs = -g.rot_s;
       for (int oy = warp; oy < Ho; oy += nwarps) {
@@ -544,7 +545,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
       scratch = q2 + (uint32_t)(c * sh.plane);   // this channel's Q2 plane is free now
       scratch_bytes = sh.plane;
     }
-    if (g.blur_on) {                           // a9: separable Gaussian in strips (R#16)
+    if (g.blur_on && !(sh.skip & 2)) {         // a9: separable Gaussian in strips (R#16)
       switch (r) {
         case 0: blur_plane<DT, VEC, 0>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;
         case 1: blur_plane<DT, VEC, 1>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;

@@ -294,9 +294,11 @@ int launch_resample_dt(const LaunchParams& p, const BatchShape& sh, cudaStream_t
   }
   const int nbands = (sh.max_ho + cfg.R - 1) / cfg.R;
   if (cfg.mode == 3) {
-    const int threads = std::min(128, ((pairs + 31) / 32) * 32);
-    const unsigned blocks = (unsigned)((uint64_t)p.n_items * nbands);
-    k_direct<DT, VEC><<<blocks, threads, 0, stream>>>(p, cfg.R, nbands);
+    const int P = std::min(112, pairs);                       // column pairs per CTA
+    const int nchunks = (pairs + P - 1) / P;
+    const int threads = ((2 * P + 31) / 32) * 32;             // two half-bands of P threads
+    const unsigned blocks = (unsigned)((uint64_t)p.n_items * nbands * nchunks);
+    k_direct<DT, VEC><<<blocks, threads, 0, stream>>>(p, cfg.R, nbands, nchunks);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_error(e, "k_direct launch");
     return SAND_OK;
@@ -325,7 +327,7 @@ bool choose_stencil(const BatchShape& sh, sc::Shape* out, size_t* smem) {
     const size_t u = std::max(plane, band);
     const size_t total = 3 * plane + u;
     if (total <= 227 * 1024) {
-      *out = sc::Shape{r, gw, rows, plane, u};
+      *out = sc::Shape{r, gw, rows, plane, u, env_int("SAND_STENCIL_SKIP", 0)};
       *smem = total;
       return true;
     }
