@@ -141,86 +141,87 @@ __device__ __forceinline__ float2 rint2(float2 v) {
   return __fadd2_rn(__fadd2_rn(v, make_float2(rs::kRound, rs::kRound)), make_float2(-rs::kRound, -rs::kRound));
 }
 
+// floor of a packed pair: s + 1.5*2^23 rounded toward -inf is 1.5*2^23 + floor(s) exactly for
+// |s| < 2^22 (FADD2.RM), so the integer sits in the low mantissa bits
+__device__ __forceinline__ uint64_t add_rm2(uint64_t a, uint64_t b) {
+  uint64_t d;
+  asm("add.rm.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+
 // Rotation (R#15) of all three Q2 planes in place. Q3 rows are computed band by band (one
-// row per warp) into a ring, and row r is written back over Q2 row r once no later Q3 row can
-// tap it: every tap of Q3 row y lies in Q2 rows [y - D, y + D]. Coordinates and fractions are
-// computed once per pixel for the three channels.
+// row per warp) into a ring of ring_rows (a power of two) rows, and row r is written back over
+// Q2 row r once no later Q3 row can tap it: every tap of Q3 row y lies in Q2 rows
+// [y - D, y + D]. Coordinates and fractions are computed once per pixel for the three channels.
 __device__ __forceinline__ void rotate_inplace(const GroupParams& g, uint32_t q2, size_t plane, uint32_t ring,
                                                int ring_rows, int D, int Wo, int Ho, int warp, int nwarps,
-                                               int lane, int tid, int nthr) {
+                                               int lane) {
   using namespace rs;
   const float rc = g.rot_c, rsn = g.rot_s, nrs = -g.rot_s;
   const float cxo = (float)(Wo - 1) * 0.5f, cyo = (float)(Ho - 1) * 0.5f;
-  const uint32_t P = (uint32_t)plane, rplane = (uint32_t)(ring_rows * Wo);
+  const uint32_t P = (uint32_t)plane, rplane = (uint32_t)(ring_rows * Wo), rmask = (uint32_t)ring_rows - 1u;
+  const uint64_t c2 = f2::pack(cxo, cyo), kr2 = f2::splat(kRound), nkr2 = f2::splat(-kRound);
+  const uint64_t nb2 = f2::splat(-kBias), m1 = f2::splat(-1.f);
   int committed = 0;   // Q2 rows [0, committed) hold Q3 already
   for (int yb = 0; yb < Ho; yb += nwarps) {
     const int oy = yb + warp;
     if (oy < Ho) {
       const float yc = __fsub_rn((float)oy, cyo);
       const uint64_t txy = f2::pack(__fmul_rn(nrs, yc), __fmul_rn(rc, yc));   // row terms
-      const uint32_t orow = ring + (uint32_t)((oy % ring_rows) * Wo);
-      for (int ox = lane; ox < Wo; ox += 32) {
-        const float xc = __fsub_rn((float)ox, cxo);
-        // (sx, sy) = ((c*xc + (-s)*yc) + cx, (s*xc + c*yc) + cy), every op rounded: scalar
-        // IEEE ops (ptxas contracts packed mul + add pairs into FFMA2, which rounds once)
-        const float sx = __fadd_rn(__fadd_rn(__fmul_rn(rc, xc), f2::lof(txy)), cxo);
-        const float sy = __fadd_rn(__fadd_rn(__fmul_rn(rsn, xc), f2::hif(txy)), cyo);
-        // floor without the XU pipe: t = s + 1.5*2^23 rounds s to the nearest integer n (exact
-        // for |s| < 2^22), whose low mantissa bits are n; one less where n > s
-        const uint64_t t = f2::add(f2::pack(sx, sy), f2::splat(kRound));
-        const uint64_t nf = f2::add(t, f2::splat(-kRound));
-        const bool gx = f2::lof(nf) > sx, gy = f2::hif(nf) > sy;
-        const float fx = gx ? __fadd_rn(f2::lof(nf), -1.f) : f2::lof(nf);
-        const float fy = gy ? __fadd_rn(f2::hif(nf), -1.f) : f2::hif(nf);
-        const uint64_t l = f2::add(f2::pack(sx, sy), f2::pack(-fx, -fy));   // (lambda_x, lambda_y), exact
-        const int x0 = (int)(f2::lo(t) - 0x4B400000u) - (gx ? 1 : 0);
-        const int y0 = (int)(f2::hi(t) - 0x4B400000u) - (gy ? 1 : 0);
+      const uint32_t orow = ring + ((uint32_t)oy & rmask) * (uint32_t)Wo;
+      float xc = __fsub_rn((float)lane, cxo);
+      for (int ox = lane; ox < Wo; ox += 32, xc = __fadd_rn(xc, 32.f)) {
+        // (sx, sy) = ((c*xc + (-s)*yc) + cx, (s*xc + c*yc) + cy), every op rounded (.rn ops
+        // are not contracted)
+        const uint64_t s2 = f2::add(f2::add(f2::pack(__fmul_rn(rc, xc), __fmul_rn(rsn, xc)), txy), c2);
+        const uint64_t t = add_rm2(s2, kr2);                      // 1.5*2^23 + floor
+        const uint64_t l = f2::fma(f2::add(t, nkr2), m1, s2);     // s - floor(s), exact
+        const int x0 = (int)(f2::lo(t) - 0x4B400000u), y0 = (int)(f2::hi(t) - 0x4B400000u);
         const uint64_t lx = f2::splat(f2::lof(l));
         const float ly = f2::hif(l);
-        const bool inside = (unsigned)x0 < (unsigned)(Wo - 1) && (unsigned)y0 < (unsigned)(Ho - 1);
         const uint32_t a0 = q2 + (uint32_t)(y0 * Wo + x0);
-        const bool in00 = x0 >= 0 && x0 < Wo && y0 >= 0 && y0 < Ho, in01 = x0 + 1 >= 0 && x0 + 1 < Wo && y0 >= 0 && y0 < Ho;
-        const bool in10 = x0 >= 0 && x0 < Wo && y0 + 1 >= 0 && y0 + 1 < Ho;
-        const bool in11 = x0 + 1 >= 0 && x0 + 1 < Wo && y0 + 1 >= 0 && y0 + 1 < Ho;
-#pragma unroll
-        for (int c = 0; c < 3; ++c) {
-          const uint32_t a = a0 + (uint32_t)c * P;
-          uint32_t b00, b01, b10, b11;   // taps outside the image read 0 (fill=None)
-          if (inside) {
-            b00 = ldsu8(a);
-            b01 = ldsu8(a + 1);
-            b10 = ldsu8(a + (uint32_t)Wo);
-            b11 = ldsu8(a + (uint32_t)Wo + 1);
-          } else {
-            b00 = in00 ? ldsu8(a) : 0u;
-            b01 = in01 ? ldsu8(a + 1) : 0u;
-            b10 = in10 ? ldsu8(a + (uint32_t)Wo) : 0u;
-            b11 = in11 ? ldsu8(a + (uint32_t)Wo + 1) : 0u;
-          }
+        auto lerp = [&](uint32_t b00, uint32_t b01, uint32_t b10, uint32_t b11) {
           // rows packed: (t00, t10) and (t01, t11) as biased floats 2^23 + t
           const uint64_t T0 = f2::pack(0x4B000000u | b00, 0x4B000000u | b10);
           const uint64_t T1 = f2::pack(0x4B000000u | b01, 0x4B000000u | b11);
-          const uint64_t d = f2::fma(T0, f2::splat(-1.f), T1);          // (t01 - t00, t11 - t10)
-          const uint64_t h = f2::fma(lx, d, f2::add(T0, f2::splat(-kBias)));   // (h0, h1)
+          const uint64_t h = f2::fma(lx, f2::fma(T0, m1, T1), f2::add(T0, nb2));   // (h0, h1)
           const float h0 = f2::lof(h), h1 = f2::hif(h);
-          const float tq = __fadd_rn(__fmaf_rn(ly, __fsub_rn(h1, h0), h0), kRound);   // rint -> low byte
-          stsu8(orow + (uint32_t)c * rplane + (uint32_t)ox, __float_as_uint(tq) & 0xffu);
+          return __float_as_uint(__fadd_rn(__fmaf_rn(ly, __fsub_rn(h1, h0), h0), kRound));   // rint -> low byte
+        };
+        if ((unsigned)x0 < (unsigned)(Wo - 1) && (unsigned)y0 < (unsigned)(Ho - 1)) {
+#pragma unroll
+          for (int c = 0; c < 3; ++c) {
+            const uint32_t a = a0 + (uint32_t)c * P, aw = a + (uint32_t)Wo;
+            stsu8(orow + (uint32_t)c * rplane + (uint32_t)ox, lerp(ldsu8(a), ldsu8(a + 1), ldsu8(aw), ldsu8(aw + 1)));
+          }
+        } else {                                 // taps outside the image read 0 (fill=None)
+          const bool in00 = x0 >= 0 && x0 < Wo && y0 >= 0 && y0 < Ho, in01 = x0 + 1 >= 0 && x0 + 1 < Wo && y0 >= 0 && y0 < Ho;
+          const bool in10 = x0 >= 0 && x0 < Wo && y0 + 1 >= 0 && y0 + 1 < Ho;
+          const bool in11 = x0 + 1 >= 0 && x0 + 1 < Wo && y0 + 1 >= 0 && y0 + 1 < Ho;
+#pragma unroll
+          for (int c = 0; c < 3; ++c) {
+            const uint32_t a = a0 + (uint32_t)c * P;
+            stsu8(orow + (uint32_t)c * rplane + (uint32_t)ox,
+                  lerp(in00 ? ldsu8(a) : 0u, in01 ? ldsu8(a + 1) : 0u, in10 ? ldsu8(a + (uint32_t)Wo) : 0u,
+                       in11 ? ldsu8(a + (uint32_t)Wo + 1) : 0u));
+          }
         }
       }
     }
     __syncthreads();                     // ring rows of this band written; Q2 reads done
     const int last = min(yb + nwarps, Ho) - 1;
     const int upto = last + 1 >= Ho ? Ho : max(committed, last - D + 1);   // rows < upto are dead in Q2
-    const int n = upto - committed;
-    if (n > 0) {                         // write back Q3 rows [committed, upto) of the three planes
-      for (int rr = warp; rr < 3 * n; rr += nwarps) {
-        const int c = rr / n, row = committed + rr - c * n;
-        const uint32_t from = ring + (uint32_t)c * rplane + (uint32_t)((row % ring_rows) * Wo);
-        const uint32_t to = q2 + (uint32_t)c * P + (uint32_t)(row * Wo);
-        if ((Wo & 3) == 0) {
-          for (int x = 4 * lane; x < Wo; x += 128) sts32(to + (uint32_t)x, st::lds32(from + (uint32_t)x));
-        } else {
-          for (int x = lane; x < Wo; x += 32) stsu8(to + (uint32_t)x, ldsu8(from + (uint32_t)x));
+    if (upto > committed) {              // write back Q3 rows [committed, upto) of the three planes
+#pragma unroll 1
+      for (int c = 0; c < 3; ++c) {
+        for (int row = committed + warp; row < upto; row += nwarps) {
+          const uint32_t from = ring + (uint32_t)c * rplane + ((uint32_t)row & rmask) * (uint32_t)Wo;
+          const uint32_t to = q2 + (uint32_t)c * P + (uint32_t)(row * Wo);
+          if ((Wo & 3) == 0) {
+            for (int x = 4 * lane; x < Wo; x += 128) sts32(to + (uint32_t)x, st::lds32(from + (uint32_t)x));
+          } else {
+            for (int x = lane; x < Wo; x += 32) stsu8(to + (uint32_t)x, ldsu8(from + (uint32_t)x));
+          }
         }
       }
       committed = upto;
@@ -229,77 +230,109 @@ __device__ __forceinline__ void rotate_inplace(const GroupParams& g, uint32_t q2
   }
 }
 
-constexpr int kBX = 8;        // blur: outputs per thread along the blocked axis
+constexpr int kBX = 16;       // blur: columns per thread in the horizontal pass
+constexpr int kBV = 16;       // blur: rows per thread in the vertical pass
 
-// Separable Gaussian blur of one channel plane with radius R (R#16): horizontal pass into
-// the fp32 scratch in row strips, vertical pass, rint (Q4), normalise and store.
+// Byte (relative to the window's 4-aligned word base) of horizontal window element k, i.e. of
+// column x0 - R + k reflected (R#16), for the three block kinds: MODE 0 interior (base
+// x0 - R - kOff), MODE 1 left border (x0 = 0, base 0), MODE 2 right border (x0 = Wo - kBX,
+// base x0 - R - kOff). All compile-time for a given (R, MODE).
+template <int R>
+constexpr int blur_koff() { return (4 - (R & 3)) & 3; }
+template <int R, int MODE>
+__host__ __device__ constexpr int widx(int k) {
+  return MODE == 0 ? blur_koff<R>() + k
+                   : (MODE == 1 ? (k < R ? R - k : k - R)
+                                : (k < kBX + R ? blur_koff<R>() + k : blur_koff<R>() + 2 * (kBX - 1) + 2 * R - k));
+}
+template <int R, int MODE>
+constexpr int wwords() {
+  return (MODE == 0 ? blur_koff<R>() + kBX + 2 * R - 1 : (MODE == 1 ? kBX + R - 1 : blur_koff<R>() + kBX + R - 1)) / 4 + 1;
+}
+
+// horizontal pass of one block: kBX outputs of strip rows (a, b) packed as pairs; window element
+// k feeds outputs o = k - i (taps i in order 0..2R, R#16), one converted element live at a time
+template <int R, int MODE>
+__device__ __forceinline__ void hblur_block(uint32_t rowa, uint32_t rowb, uint32_t wb, const float (&wt)[2 * R + 1],
+                                            uint64_t (&accs)[kBX]) {
+  constexpr int kW = wwords<R, MODE>();
+  uint32_t wa[kW], wv[kW];
+#pragma unroll
+  for (int k = 0; k < kW; ++k) {
+    wa[k] = st::lds32(rowa + wb + 4u * k);
+    wv[k] = st::lds32(rowb + wb + 4u * k);
+  }
+#pragma unroll
+  for (int o = 0; o < kBX; ++o) accs[o] = 0ull;
+#pragma unroll
+  for (int k = 0; k < kBX + 2 * R; ++k) {
+    const int bi = widx<R, MODE>(k);
+    // biased floats 2^23 + byte of both rows, then one packed subtract
+    const uint32_t fa = __byte_perm(wa[bi >> 2], 0x4B000000u, 0x7440 | (bi & 3));
+    const uint32_t fb = __byte_perm(wv[bi >> 2], 0x4B000000u, 0x7440 | (bi & 3));
+    const uint64_t v = rs::f2::add(rs::f2::pack(fa, fb), rs::f2::splat(-rs::kBias));
+#pragma unroll
+    for (int o = 0; o < kBX; ++o)
+      if (k - o >= 0 && k - o <= 2 * R) accs[o] = rs::f2::fma(rs::f2::splat(wt[k - o]), v, accs[o]);
+  }
+}
+
+// Separable Gaussian blur of one channel plane with radius R (R#16): horizontal pass into the
+// fp32 scratch in row strips, vertical pass, rint (Q4), normalise and store. Every output's taps
+// are accumulated from 0 in order i = 0..2R with fmaf in both passes (bit-identical to the
+// oracle). Fast path (Wo % kBX == 0, Wo % 4 == 0, Wo >= 2 kBX + R): word loads with
+// compile-time reflect maps for the border blocks; otherwise per-byte loads with reflect.
 template <int DT, bool VEC, int R>
 __device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupParams& g, const ChDests& cd,
-                                           uint32_t src, uint32_t scratch, size_t plane, int Wo, int Ho,
+                                           uint32_t src, uint32_t scratch, size_t scratch_bytes, int Wo, int Ho,
                                            int tid, int nthr) {
   const int pairs = (Wo + 1) >> 1;
-  const int strip_rows = (int)(plane / ((size_t)Wo * 4));   // fp32 rows the scratch holds
-  const int S = strip_rows - 2 * R;
-  // taps in registers (loaded once; the shared-memory stores below must not force reloads)
+  const int cap_rows = (int)(scratch_bytes / ((size_t)Wo * 4));   // fp32 rows the scratch holds
+  // vertical mapping: G groups of `pairs` threads, each group takes kBV-row blocks of the strip
+  const int G = max(1, nthr / pairs);
+  const int vgrp = tid / pairs, vpr = tid - vgrp * pairs;
+  // strip height: the largest multiple of G * kBV that fits (so row blocks spread evenly over
+  // the groups), else whatever fits
+  int S = ((cap_rows - 2 * R) / (G * kBV)) * (G * kBV);
+  if (S <= 0) S = cap_rows - 2 * R;
+  S = min(S, Ho);
   float wt[2 * R + 1];
 #pragma unroll
   for (int i = 0; i <= 2 * R; ++i) wt[i] = __ldg(&g.blur_w[i]);
-  // word-aligned rows: interior blocks load their window as 32-bit words (the window's byte
-  // misalignment (-R) & 3 is a compile-time constant) and store 16 B per 4 columns
-  const bool words = (Wo & 3) == 0;
-  constexpr int kOff = (4 - (R & 3)) & 3;                 // (x0 - R) & 3 for x0 % 8 == 0
-  constexpr int kWin = kBX + 2 * R;
-  constexpr int kWords = (kOff + kWin + 3) / 4;
+  const bool fast = (Wo & 3) == 0 && Wo % kBX == 0 && Wo >= 2 * kBX + R + 3;
+  const int xblocks = fast ? Wo / kBX : (Wo + kBX - 1) / kBX;
+  constexpr int kOff = blur_koff<R>();
   for (int ys = 0; ys < Ho; ys += S) {
     const int ns = min(S, Ho - ys);
     const int jrows = ns + 2 * R;          // strip row j <-> image row reflect(ys - R + j)
-    // horizontal pass: thread = (pair of strip rows j, j + half) x block of kBX columns
     const int half = (jrows + 1) >> 1;
-    const int xblocks = (Wo + kBX - 1) / kBX;
-    for (int e = tid; e < half * xblocks; e += nthr) {
-      const int j = e / xblocks, xb = e - j * xblocks;
-      const int ja2 = j, jb2 = min(j + half, jrows - 1);
-      const uint32_t rowa = src + (uint32_t)(reflect(ys - R + ja2, Ho) * Wo);
-      const uint32_t rowb = src + (uint32_t)(reflect(ys - R + jb2, Ho) * Wo);
-      const int x0 = xb * kBX;
-      // Window element k feeds outputs o = k - i for taps i; iterating k upwards and updating
-      // every output it feeds keeps each output's taps in order i = 0..2R (R#16), while only
-      // one converted element is live at a time.
-      uint64_t accs[kBX];
-#pragma unroll
-      for (int o = 0; o < kBX; ++o) accs[o] = 0ull;
-      auto feed = [&](int k, uint64_t v) {
-#pragma unroll
-        for (int o = 0; o < kBX; ++o)
-          if (k - o >= 0 && k - o <= 2 * R) accs[o] = rs::f2::fma(rs::f2::splat(wt[k - o]), v, accs[o]);
-      };
-      const bool interior = x0 - R >= 0 && x0 + kBX - 1 + R < Wo;
-      if (interior && words) {
-        const uint32_t wb = (uint32_t)(x0 - R - kOff);   // 4-aligned
-        uint32_t wa[kWords], wbv[kWords];
-#pragma unroll
-        for (int k = 0; k < kWords; ++k) {
-          wa[k] = st::lds32(rowa + wb + 4u * k);
-          wbv[k] = st::lds32(rowb + wb + 4u * k);
+    // ---- horizontal pass: unit = (strip rows j, j + half) x block of kBX columns. Interior
+    // units first (lanes along the row), then the two border blocks of every row pair, so a
+    // warp runs one block kind.
+    if (fast) {
+      const int nib = xblocks - 2;         // interior blocks per row
+      const int n_int = half * nib, n_all = half * xblocks;
+      for (int e = tid; e < n_all; e += nthr) {
+        int j, x0, mode;
+        if (e < n_int) {
+          j = e / nib;
+          x0 = (e - j * nib + 1) * kBX;
+          mode = 0;
+        } else {
+          const int e2 = e - n_int;
+          j = e2 >> 1;
+          mode = 1 + (e2 & 1);
+          x0 = mode == 1 ? 0 : Wo - kBX;
         }
+        const int ja2 = j, jb2 = min(j + half, jrows - 1);
+        const uint32_t rowa = src + (uint32_t)(reflect(ys - R + ja2, Ho) * Wo);
+        const uint32_t rowb = src + (uint32_t)(reflect(ys - R + jb2, Ho) * Wo);
+        uint64_t accs[kBX];
+        if (mode == 0) hblur_block<R, 0>(rowa, rowb, (uint32_t)(x0 - R - kOff), wt, accs);
+        else if (mode == 1) hblur_block<R, 1>(rowa, rowb, 0u, wt, accs);
+        else hblur_block<R, 2>(rowa, rowb, (uint32_t)(x0 - R - kOff), wt, accs);
 #pragma unroll
-        for (int k = 0; k < kWin; ++k) {
-          const int bi = kOff + k;
-          // biased floats 2^23 + byte of both rows, then one packed subtract
-          const uint32_t fa = __byte_perm(wa[bi >> 2], 0x4B000000u, 0x7440 | (bi & 3));
-          const uint32_t fb = __byte_perm(wbv[bi >> 2], 0x4B000000u, 0x7440 | (bi & 3));
-          feed(k, rs::f2::add(rs::f2::pack(fa, fb), rs::f2::splat(-rs::kBias)));
-        }
-      } else {
-#pragma unroll
-        for (int k = 0; k < kWin; ++k) {
-          const int xx = reflect(min(x0 - R + k, 2 * Wo - 2), Wo);
-          feed(k, rs::f2::pack(u8f(ldsu8(rowa + (uint32_t)xx)), u8f(ldsu8(rowb + (uint32_t)xx))));
-        }
-      }
-      if (words && x0 + kBX <= Wo) {               // 16 B stores: 4 columns of one strip row
-#pragma unroll
-        for (int o = 0; o < kBX; o += 4) {
+        for (int o = 0; o < kBX; o += 4) {   // 16 B stores: 4 columns of one strip row
           st::sts128(scratch + 4u * (uint32_t)(ja2 * Wo + x0 + o),
                      make_uint4(rs::f2::lo(accs[o]), rs::f2::lo(accs[o + 1]), rs::f2::lo(accs[o + 2]),
                                 rs::f2::lo(accs[o + 3])));
@@ -307,7 +340,24 @@ __device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupPar
                      make_uint4(rs::f2::hi(accs[o]), rs::f2::hi(accs[o + 1]), rs::f2::hi(accs[o + 2]),
                                 rs::f2::hi(accs[o + 3])));
         }
-      } else {
+      }
+    } else {
+      for (int e = tid; e < half * xblocks; e += nthr) {
+        const int j = e / xblocks, x0 = (e - j * xblocks) * kBX;
+        const int ja2 = j, jb2 = min(j + half, jrows - 1);
+        const uint32_t rowa = src + (uint32_t)(reflect(ys - R + ja2, Ho) * Wo);
+        const uint32_t rowb = src + (uint32_t)(reflect(ys - R + jb2, Ho) * Wo);
+        uint64_t accs[kBX];
+#pragma unroll
+        for (int o = 0; o < kBX; ++o) accs[o] = 0ull;
+#pragma unroll
+        for (int k = 0; k < kBX + 2 * R; ++k) {
+          const int xx = reflect(min(x0 - R + k, 2 * Wo - 2), Wo);
+          const uint64_t v = rs::f2::pack(u8f(ldsu8(rowa + (uint32_t)xx)), u8f(ldsu8(rowb + (uint32_t)xx)));
+#pragma unroll
+          for (int o = 0; o < kBX; ++o)
+            if (k - o >= 0 && k - o <= 2 * R) accs[o] = rs::f2::fma(rs::f2::splat(wt[k - o]), v, accs[o]);
+        }
 #pragma unroll
         for (int o = 0; o < kBX; ++o) {
           if (x0 + o < Wo) {
@@ -318,46 +368,42 @@ __device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupPar
       }
     }
     __syncthreads();
-    // vertical pass: thread = column pair (x, x+1) x block of kBV output rows; window rows
+    // ---- vertical pass: thread = column pair (x, x+1) x blocks of kBV output rows; window rows
     // feed the outputs in tap order as in the horizontal pass
-    constexpr int kBV = 16;
-    const int rblocks = (ns + kBV - 1) / kBV;
-    for (int e = tid; e < pairs * rblocks; e += nthr) {
-      const int rb = e / pairs, pr2 = e - rb * pairs;
-      const int ox = 2 * pr2, y0 = rb * kBV;
+    if (vgrp < G) {
+      const int nblk = (ns + kBV - 1) / kBV;
+      const int ox = 2 * vpr;
       const bool has_b = ox + 1 < Wo;
-      uint64_t accs[kBV];
-#pragma unroll
-      for (int o = 0; o < kBV; ++o) accs[o] = 0ull;
-      auto feed = [&](int k, uint64_t v) {
-#pragma unroll
-        for (int o = 0; o < kBV; ++o)
-          if (k - o >= 0 && k - o <= 2 * R) accs[o] = rs::f2::fma(rs::f2::splat(wt[k - o]), v, accs[o]);
-      };
-      const uint32_t a0 = scratch + 4u * (uint32_t)(y0 * Wo + ox);
+      const bool pair_ok = has_b && !(Wo & 1);
       const uint32_t rstep = 4u * (uint32_t)Wo;
-      if (has_b && !(Wo & 1) && y0 + kBV + 2 * R <= jrows) {
+      for (int blk = vgrp; blk < nblk; blk += G) {
+        const int y0 = blk * kBV;
+        uint64_t accs[kBV];
+#pragma unroll
+        for (int o = 0; o < kBV; ++o) accs[o] = 0ull;
+        const uint32_t a0 = scratch + 4u * (uint32_t)(y0 * Wo + ox);
+        const bool full = y0 + kBV + 2 * R <= jrows;
 #pragma unroll
         for (int k = 0; k < kBV + 2 * R; ++k) {
-          const float2 v = lds64f(a0 + rstep * k);
-          feed(k, rs::f2::pack(v.x, v.y));
-        }
-      } else {
-#pragma unroll
-        for (int k = 0; k < kBV + 2 * R; ++k) {
-          uint64_t v = 0ull;
-          if (y0 + k < jrows) {
-            const uint32_t a = a0 + rstep * k;
+          // rows past the strip only feed outputs that are not stored: clamp their address
+          const uint32_t a = full ? a0 + rstep * k : scratch + 4u * (uint32_t)(min(y0 + k, jrows - 1) * Wo + ox);
+          uint64_t v;
+          if (pair_ok) {
+            const float2 f = lds64f(a);
+            v = rs::f2::pack(f.x, f.y);
+          } else {
             v = rs::f2::pack(st::lds32(a), has_b ? st::lds32(a + 4) : 0u);
           }
-          feed(k, v);
-        }
-      }
 #pragma unroll
-      for (int o = 0; o < kBV; ++o) {
-        if (y0 + o >= ns) break;
-        store_q<DT, VEC>(p, cd, ys + y0 + o, ox, Wo, rint2(make_float2(rs::f2::lof(accs[o]), rs::f2::hif(accs[o]))),
-                         has_b);
+          for (int o = 0; o < kBV; ++o)
+            if (k - o >= 0 && k - o <= 2 * R) accs[o] = rs::f2::fma(rs::f2::splat(wt[k - o]), v, accs[o]);
+        }
+#pragma unroll
+        for (int o = 0; o < kBV; ++o) {
+          if (y0 + o >= ns) break;
+          store_q<DT, VEC>(p, cd, ys + y0 + o, ox, Wo, rint2(make_float2(rs::f2::lof(accs[o]), rs::f2::hif(accs[o]))),
+                           has_b);
+        }
       }
     }
     __syncthreads();
@@ -486,13 +532,16 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
   if (g.rot_on && !(sh.skip & 1)) {
     const float bound = fabsf(g.rot_s) * cxo + (1.f - g.rot_c) * cyo;
     const int D = (int)ceilf(bound) + 2;
-    const int ring_rows = D + nwarps + 1;
+    int ring_rows = 1;
+    while (ring_rows < D + nwarps + 1) ring_rows <<= 1;
     if ((size_t)ring_rows * 3 * Wo <= sh.ubytes && D < Ho) {
-      rotate_inplace(g, q2, sh.plane, ureg, ring_rows, D, Wo, Ho, warp, nwarps, lane, tid, nthr);
+      rotate_inplace(g, q2, sh.plane, ureg, ring_rows, D, Wo, Ho, warp, nwarps, lane);
       rotated = true;
     }
   }
-  for (int c = 0; c < 3; ++c) {
+  // channels last to first: once channel c is done its plane joins the scratch of the next
+  // (planes are contiguous and the band/Q3 region follows plane 2)
+  for (int c = 2; c >= 0; --c) {
     ChDests cd;
     cd.nd = nd;
     cd.dests = dests;
@@ -500,8 +549,8 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
     cd.d0 = ch_dest(p, dests[0], c);
     if (nd > 1) cd.d1 = ch_dest(p, dests[1], c);
     uint32_t src = q2 + (uint32_t)(c * sh.plane);
-    uint32_t scratch = ureg;
-    size_t scratch_bytes = sh.ubytes;
+    uint32_t scratch = q2 + (uint32_t)((c + 1) * sh.plane);
+    size_t scratch_bytes = (size_t)(2 - c) * sh.plane + sh.ubytes;
     if (g.rot_on && !rotated && !(sh.skip & 1)) {              // a8: Q3 = rotate(Q2) (R#15), one channel
       const uint32_t q3 = ureg;
       const float rc = g.rot_c, rsn = g.rot_s, nrs = -g.rot_s;
@@ -542,8 +591,8 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
       }
       __syncthreads();
       src = q3;
-      scratch = q2 + (uint32_t)(c * sh.plane);   // this channel's Q2 plane is free now
-      scratch_bytes = sh.plane;
+      scratch = q2 + (uint32_t)(c * sh.plane);   // this channel's Q2 plane (and the done ones) are free now
+      scratch_bytes = (size_t)(3 - c) * sh.plane;
     }
     if (g.blur_on && !(sh.skip & 2)) {         // a9: separable Gaussian in strips (R#16)
       switch (r) {
@@ -561,12 +610,28 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
         default: blur_plane<DT, VEC, 11>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;
       }
     } else {                                   // no blur: normalise + store the (rotated) plane
-      for (int oy = warp; oy < Ho; oy += nwarps) {
-        const uint32_t row = src + (uint32_t)(oy * Wo);
-        for (int ox = 2 * lane; ox < Wo; ox += 64) {
-          const bool has_b = ox + 1 < Wo;
-          const float2 q = make_float2(u8f(ldsu8(row + ox)), has_b ? u8f(ldsu8(row + ox + 1)) : 0.f);
-          store_q<DT, VEC>(p, cd, oy, ox, Wo, q, has_b);
+      if ((Wo & 3) == 0) {                     // 4 pixels per thread from one word
+        const int q4 = Wo >> 2;
+        const int dy = nthr / q4, dq = nthr - dy * q4;   // unit e = oy * q4 + q, stepped without divisions
+        int oy = tid / q4, q = tid - oy * q4;
+        for (; oy < Ho; oy += dy, q += dq, (q >= q4 ? (q -= q4, ++oy) : 0)) {
+          const int ox = 4 * q;
+          const uint32_t wv = st::lds32(src + (uint32_t)(oy * Wo + ox));
+          const uint64_t q01 = rs::f2::add(rs::f2::pack(__byte_perm(wv, 0x4B000000u, 0x7440), __byte_perm(wv, 0x4B000000u, 0x7441)),
+                                           rs::f2::splat(-rs::kBias));
+          const uint64_t q23 = rs::f2::add(rs::f2::pack(__byte_perm(wv, 0x4B000000u, 0x7442), __byte_perm(wv, 0x4B000000u, 0x7443)),
+                                           rs::f2::splat(-rs::kBias));
+          store_q<DT, VEC>(p, cd, oy, ox, Wo, make_float2(rs::f2::lof(q01), rs::f2::hif(q01)), true);
+          store_q<DT, VEC>(p, cd, oy, ox + 2, Wo, make_float2(rs::f2::lof(q23), rs::f2::hif(q23)), true);
+        }
+      } else {
+        for (int oy = warp; oy < Ho; oy += nwarps) {
+          const uint32_t row = src + (uint32_t)(oy * Wo);
+          for (int ox = 2 * lane; ox < Wo; ox += 64) {
+            const bool has_b = ox + 1 < Wo;
+            const float2 q = make_float2(u8f(ldsu8(row + ox)), has_b ? u8f(ldsu8(row + ox + 1)) : 0.f);
+            store_q<DT, VEC>(p, cd, oy, ox, Wo, q, has_b);
+          }
         }
       }
       __syncthreads();

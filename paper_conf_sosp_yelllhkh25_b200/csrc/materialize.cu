@@ -324,7 +324,10 @@ bool choose_stencil(const BatchShape& sh, sc::Shape* out, size_t* smem) {
   for (int r : kCands) {
     const int rows = (int)std::ceil((double)sh.st_max_scy * r) + 3;
     const size_t band = sc::band_bytes(sh.st_max_wo, r, rows, gw);
-    const size_t u = std::max(plane, band);
+    // the band/Q3 region takes everything the three planes leave (one CTA per SM anyway): a
+    // larger rotation ring and taller blur strips
+    const size_t rest = 3 * plane < (size_t)227 * 1024 ? (size_t)227 * 1024 - 3 * plane : 0;
+    const size_t u = std::max(std::max(plane, band), rest);
     const size_t total = 3 * plane + u;
     if (total <= 227 * 1024) {
       *out = sc::Shape{r, gw, rows, plane, u, env_int("SAND_STENCIL_SKIP", 0)};
@@ -380,33 +383,38 @@ int launch_materialize(const LaunchParams& p, const BatchShape& shape, size_t st
   *n_launched = 0;
   if (p.n_items == 0) return SAND_OK;
   if (shape.has_direct) {
+    LaunchParams pd = p;
+    pd.n_items = shape.n_direct;
     int rc;
     // specialised instantiations: one dtype for every view and even output widths (the
     // 4-byte pair stores are aligned); anything else takes the generic instantiation
     switch (shape.even_wo ? shape.dtype : -1) {
-      case SAND_U8: rc = launch_resample_dt<SAND_U8, true>(p, shape, stream); break;
-      case SAND_BF16: rc = launch_resample_dt<SAND_BF16, true>(p, shape, stream); break;
-      case SAND_F32: rc = launch_resample_dt<SAND_F32, true>(p, shape, stream); break;
-      default: rc = launch_resample_dt<-1, false>(p, shape, stream); break;
+      case SAND_U8: rc = launch_resample_dt<SAND_U8, true>(pd, shape, stream); break;
+      case SAND_BF16: rc = launch_resample_dt<SAND_BF16, true>(pd, shape, stream); break;
+      case SAND_F32: rc = launch_resample_dt<SAND_F32, true>(pd, shape, stream); break;
+      default: rc = launch_resample_dt<-1, false>(pd, shape, stream); break;
     }
     if (rc != SAND_OK) return rc;
     ++*n_launched;
   }
   if (shape.has_stencil) {
+    LaunchParams ps = p;
+    ps.items = p.items + shape.n_direct;
+    ps.n_items = p.n_items - shape.n_direct;
     sc::Shape scs;
     size_t smem2;
     if (getenv("SAND_STENCIL_V1") == nullptr && choose_stencil(shape, &scs, &smem2)) {
       const int dt = shape.even_wo ? shape.dtype : -1;
-      if (dt == SAND_U8) k_stencil2<SAND_U8, true><<<p.n_items, 512, smem2, stream>>>(p, scs, shape.st_max_wo);
-      else if (dt == SAND_BF16) k_stencil2<SAND_BF16, true><<<p.n_items, 512, smem2, stream>>>(p, scs, shape.st_max_wo);
-      else if (dt == SAND_F32) k_stencil2<SAND_F32, true><<<p.n_items, 512, smem2, stream>>>(p, scs, shape.st_max_wo);
-      else k_stencil2<-1, false><<<p.n_items, 512, smem2, stream>>>(p, scs, shape.st_max_wo);
+      if (dt == SAND_U8) k_stencil2<SAND_U8, true><<<ps.n_items, 512, smem2, stream>>>(ps, scs, shape.st_max_wo);
+      else if (dt == SAND_BF16) k_stencil2<SAND_BF16, true><<<ps.n_items, 512, smem2, stream>>>(ps, scs, shape.st_max_wo);
+      else if (dt == SAND_F32) k_stencil2<SAND_F32, true><<<ps.n_items, 512, smem2, stream>>>(ps, scs, shape.st_max_wo);
+      else k_stencil2<-1, false><<<ps.n_items, 512, smem2, stream>>>(ps, scs, shape.st_max_wo);
       cudaError_t e = cudaGetLastError();
       if (e != cudaSuccess) return cuda_error(e, "k_stencil2 launch");
       ++*n_launched;
       return SAND_OK;
     }
-    k_stencil<<<p.n_items, 512, stencil_smem, stream>>>(p);
+    k_stencil<<<ps.n_items, 512, stencil_smem, stream>>>(ps);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_error(e, "k_stencil launch");
     ++*n_launched;

@@ -72,6 +72,7 @@ struct BatchShape {
   // stencil (rotation/blur) items
   int32_t st_max_wo, st_max_ho, st_cols_bound;
   float st_max_scy;
+  uint32_t n_direct;      // items [0, n_direct) of the batch are direct, the rest stencil items
 };
 
 struct LaunchParams {

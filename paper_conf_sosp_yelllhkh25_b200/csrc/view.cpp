@@ -227,6 +227,13 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
       i = j;
     }
     plan->fetch_begin.push_back(static_cast<uint32_t>(plan->fetch_keys.size()));
+    // direct items first, stencil items after (order kept within each class): each kernel
+    // then walks a dense slice instead of skipping the other class's items
+    {
+      auto first = plan->items.begin() + plan->item_begin.back();
+      auto mid = std::stable_partition(first, plan->items.end(), [](const sand::WorkItem& w) { return !(w.flags & 1u); });
+      shape.n_direct = static_cast<uint32_t>(mid - first);
+    }
     plan->item_begin.push_back(static_cast<uint32_t>(plan->items.size()));
     plan->shapes.push_back(shape);
   }
