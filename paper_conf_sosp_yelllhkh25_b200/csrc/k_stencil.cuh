@@ -137,6 +137,26 @@ __device__ __forceinline__ void store_q(const LaunchParams& p, const ChDests& cd
   for (int d = 2; d < cd.nd; ++d) put_q<DT, VEC>(ch_dest(p, cd.dests[d], cd.c), oy, ox, Wo, q, has_b);
 }
 
+// q pair (biased: 1.5*2^23 + q per lane, the rint result) -> normalise (R#17) -> one 2-element
+// store at o (compile-time dtype, aligned pair)
+template <int DT>
+__device__ __forceinline__ void put_pair(uint8_t* o, uint64_t tq, uint64_t na, uint64_t nb) {
+  using namespace rs;
+  if constexpr (DT == SAND_U8) {
+    *reinterpret_cast<uint16_t*>(o) = (uint16_t)__byte_perm(f2::lo(tq), f2::hi(tq), 0x0040);
+  } else {
+    const uint64_t y = f2::fma(f2::add(tq, f2::splat(-kRound)), na, nb);   // fmaf(q, a_c, b_c)
+    if constexpr (DT == SAND_BF16) {
+      const __nv_bfloat162 v = __floats2bfloat162_rn(f2::lof(y), f2::hif(y));
+      *reinterpret_cast<uint32_t*>(o) = *reinterpret_cast<const uint32_t*>(&v);
+    } else {
+      *reinterpret_cast<uint2*>(o) = make_uint2(f2::lo(y), f2::hi(y));
+    }
+  }
+}
+template <int DT>
+constexpr int dt_bytes() { return DT == SAND_U8 ? 1 : (DT == SAND_BF16 ? 2 : 4); }
+
 __device__ __forceinline__ float2 rint2(float2 v) {
   return __fadd2_rn(__fadd2_rn(v, make_float2(rs::kRound, rs::kRound)), make_float2(-rs::kRound, -rs::kRound));
 }
@@ -230,8 +250,76 @@ __device__ __forceinline__ void rotate_inplace(const GroupParams& g, uint32_t q2
   }
 }
 
-constexpr int kBX = 16;       // blur: columns per thread in the horizontal pass
-constexpr int kBV = 16;       // blur: rows per thread in the vertical pass
+// Rotation (R#15) of the three Q2 planes straight to the output when no blur follows: Q3 is
+// rint'ed, normalised (R#17) and stored per pixel (2/4/1-byte stores, a warp writes one
+// contiguous row segment per channel). Q2 is only read, so no barriers are needed.
+template <int DT>
+__device__ __forceinline__ void rotate_direct(const GroupParams& g, uint32_t q2, size_t plane, int Wo, int Ho,
+                                              int warp, int nwarps, int lane, uint8_t* const (&obase)[3],
+                                              const float (&na)[3], const float (&nb)[3]) {
+  using namespace rs;
+  const float rc = g.rot_c, rsn = g.rot_s, nrs = -g.rot_s;
+  const float cxo = (float)(Wo - 1) * 0.5f, cyo = (float)(Ho - 1) * 0.5f;
+  const uint32_t P = (uint32_t)plane;
+  const uint64_t c2 = f2::pack(cxo, cyo), kr2 = f2::splat(kRound), nkr2 = f2::splat(-kRound);
+  const uint64_t nb2 = f2::splat(-kBias), m1 = f2::splat(-1.f);
+  for (int oy = warp; oy < Ho; oy += nwarps) {
+    const float yc = __fsub_rn((float)oy, cyo);
+    const uint64_t txy = f2::pack(__fmul_rn(nrs, yc), __fmul_rn(rc, yc));
+    const size_t orow = (size_t)oy * Wo;
+    float xc = __fsub_rn((float)lane, cxo);
+    for (int ox = lane; ox < Wo; ox += 32, xc = __fadd_rn(xc, 32.f)) {
+      const uint64_t s2 = f2::add(f2::add(f2::pack(__fmul_rn(rc, xc), __fmul_rn(rsn, xc)), txy), c2);
+      const uint64_t t = add_rm2(s2, kr2);
+      const uint64_t l = f2::fma(f2::add(t, nkr2), m1, s2);
+      const int x0 = (int)(f2::lo(t) - 0x4B400000u), y0 = (int)(f2::hi(t) - 0x4B400000u);
+      const uint64_t lx = f2::splat(f2::lof(l));
+      const float ly = f2::hif(l);
+      const uint32_t a0 = q2 + (uint32_t)(y0 * Wo + x0);
+      auto emit = [&](int c, uint32_t b00, uint32_t b01, uint32_t b10, uint32_t b11) {
+        const uint64_t T0 = f2::pack(0x4B000000u | b00, 0x4B000000u | b10);
+        const uint64_t T1 = f2::pack(0x4B000000u | b01, 0x4B000000u | b11);
+        const uint64_t h = f2::fma(lx, f2::fma(T0, m1, T1), f2::add(T0, nb2));
+        const float h0 = f2::lof(h), h1 = f2::hif(h);
+        const float tq = __fadd_rn(__fmaf_rn(ly, __fsub_rn(h1, h0), h0), kRound);   // 1.5*2^23 + q
+        uint8_t* o = obase[c] + (orow + (size_t)ox) * dt_bytes<DT>();
+        if constexpr (DT == SAND_U8) {
+          *o = (uint8_t)(__float_as_uint(tq) & 0xffu);
+        } else {
+          const float y = __fmaf_rn(__fadd_rn(tq, -kRound), na[c], nb[c]);
+          if constexpr (DT == SAND_BF16) *reinterpret_cast<__nv_bfloat16*>(o) = __float2bfloat16_rn(y);
+          else *reinterpret_cast<float*>(o) = y;
+        }
+      };
+      if ((unsigned)x0 < (unsigned)(Wo - 1) && (unsigned)y0 < (unsigned)(Ho - 1)) {
+#pragma unroll
+        for (int c = 0; c < 3; ++c) {
+          const uint32_t a = a0 + (uint32_t)c * P, aw = a + (uint32_t)Wo;
+          emit(c, ldsu8(a), ldsu8(a + 1), ldsu8(aw), ldsu8(aw + 1));
+        }
+      } else {                                   // taps outside the image read 0 (fill=None)
+        const bool in00 = x0 >= 0 && x0 < Wo && y0 >= 0 && y0 < Ho, in01 = x0 + 1 >= 0 && x0 + 1 < Wo && y0 >= 0 && y0 < Ho;
+        const bool in10 = x0 >= 0 && x0 < Wo && y0 + 1 >= 0 && y0 + 1 < Ho;
+        const bool in11 = x0 + 1 >= 0 && x0 + 1 < Wo && y0 + 1 >= 0 && y0 + 1 < Ho;
+#pragma unroll
+        for (int c = 0; c < 3; ++c) {
+          const uint32_t a = a0 + (uint32_t)c * P;
+          emit(c, in00 ? ldsu8(a) : 0u, in01 ? ldsu8(a + 1) : 0u, in10 ? ldsu8(a + (uint32_t)Wo) : 0u,
+               in11 ? ldsu8(a + (uint32_t)Wo + 1) : 0u);
+        }
+      }
+    }
+  }
+}
+
+#ifndef SAND_BLUR_BX
+#define SAND_BLUR_BX 16
+#endif
+#ifndef SAND_BLUR_BV
+#define SAND_BLUR_BV 16
+#endif
+constexpr int kBX = SAND_BLUR_BX;   // blur: columns per thread in the horizontal pass (multiple of 4)
+constexpr int kBV = SAND_BLUR_BV;   // blur: rows per thread in the vertical pass
 
 // Byte (relative to the window's 4-aligned word base) of horizontal window element k, i.e. of
 // column x0 - R + k reflected (R#16), for the three block kinds: MODE 0 interior (base
@@ -376,6 +464,9 @@ __device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupPar
       const bool has_b = ox + 1 < Wo;
       const bool pair_ok = has_b && !(Wo & 1);
       const uint32_t rstep = 4u * (uint32_t)Wo;
+      const bool fast_st = cd.nd == 1 && pair_ok;
+      uint8_t* const obase = cd.d0.base;
+      const uint64_t na = rs::f2::splat(cd.d0.a), nb = rs::f2::splat(cd.d0.b);
       for (int blk = vgrp; blk < nblk; blk += G) {
         const int y0 = blk * kBV;
         uint64_t accs[kBV];
@@ -397,6 +488,19 @@ __device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupPar
 #pragma unroll
           for (int o = 0; o < kBV; ++o)
             if (k - o >= 0 && k - o <= 2 * R) accs[o] = rs::f2::fma(rs::f2::splat(wt[k - o]), v, accs[o]);
+        }
+        if constexpr (DT >= 0) {
+          if (fast_st) {                     // one destination: incremental row pointer
+            uint8_t* o = obase + ((size_t)(ys + y0) * Wo + ox) * dt_bytes<DT>();
+            const size_t rsb = (size_t)Wo * dt_bytes<DT>();
+#pragma unroll
+            for (int oo = 0; oo < kBV; ++oo) {
+              if (y0 + oo >= ns) break;
+              put_pair<DT>(o, rs::f2::add(accs[oo], rs::f2::splat(rs::kRound)), na, nb);
+              o += rsb;
+            }
+            continue;
+          }
         }
 #pragma unroll
         for (int o = 0; o < kBV; ++o) {
@@ -445,6 +549,19 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
   const uint32_t rowbytes = (uint32_t)gw * 4u;
   const uint8_t* Yp = p.slab + w.y_off;
   const uint8_t* UVp = Yp + (size_t)w.pitch * w.src_h;
+  // source rows of the band starting at output row oy_lo
+  auto band = [&](int oy_lo, int& nr, int& y_lo, int& y_hi) {
+    nr = min(sh.R, Ho - oy_lo);
+    y_lo = tap0(g.sc_y, g.off_y, oy_lo, g.org_y);
+    int d0;
+    float f0;
+    tap(g.sc_y, g.off_y, oy_lo + nr - 1, g.lim_y, g.org_y, d0, y_hi, f0);
+  };
+  {                                           // band 0's NV12 rows are in flight while the tables are built
+    int nr0, ylo0, yhi0;
+    band(0, nr0, ylo0, yhi0);
+    st::stage_rows_cp(s_rawb, Yp + x16, UVp + x16, w.pitch, gw, ylo0, yhi0, warp, nwarps, lane);
+  }
   for (int j = tid; j < Wo; j += nthr) {
     int x0, x1;
     float lx;
@@ -455,12 +572,11 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
   const int groups = max(1, nthr / pairs);
   const int grp = tid / pairs, pr = tid - grp * pairs;
   for (int oy_lo = 0; oy_lo < Ho; oy_lo += sh.R) {
-    const int nr = min(sh.R, Ho - oy_lo);
-    const int y_lo = tap0(g.sc_y, g.off_y, oy_lo, g.org_y);
-    int y_hi;
-    tap(g.sc_y, g.off_y, oy_lo + nr - 1, g.lim_y, g.org_y, dmy, y_hi, fl);
-    __syncthreads();                          // previous band's walkers are done with the grid
-    st::stage_rows_cp(s_rawb, Yp + x16, UVp + x16, w.pitch, gw, y_lo, y_hi, warp, nwarps, lane);
+    int nr, y_lo, y_hi;
+    band(oy_lo, nr, y_lo, y_hi);
+    asm volatile("cp.async.wait_group 0;\n" ::: "memory");
+    __syncthreads();                          // raw of this band landed; the previous walk is done with grid/rtab
+    st::convert_rows(s_grid, s_rawb, gw, y_lo, y_hi, y_lo, 1 << 30, 5u, warp, nwarps, lane);   // no wrap
     for (int r = tid; r < nr; r += nthr) {
       int y0, y1;
       float ly;
@@ -468,10 +584,12 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
       rtab[r] = make_uint4((uint32_t)(y0 - y_lo) * rowbytes, (uint32_t)(y1 - y_lo) * rowbytes, (uint32_t)y0,
                            __float_as_uint(ly));
     }
-    asm volatile("cp.async.wait_group 0;\n" ::: "memory");
-    __syncthreads();
-    st::convert_rows(s_grid, s_rawb, gw, y_lo, y_hi, y_lo, 1 << 30, 5u, warp, nwarps, lane);   // no wrap
-    __syncthreads();
+    __syncthreads();                          // grid + rtab ready, raw drained
+    if (oy_lo + sh.R < Ho) {                  // the next band's rows load while this band is walked
+      int nr1, ylo1, yhi1;
+      band(oy_lo + sh.R, nr1, ylo1, yhi1);
+      st::stage_rows_cp(s_rawb, Yp + x16, UVp + x16, w.pitch, gw, ylo1, yhi1, warp, nwarps, lane);
+    }
     if (grp < groups && pr < pairs && !(sh.skip & 4)) {
       const int ox = 2 * pr;
       const bool has_b = ox + 1 < Wo;
@@ -527,6 +645,21 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
   // ------------------------------------------------------------- phase 2: per channel
   const int r = g.blur_on ? g.blur_r : 0;
   const float cxo = (float)(Wo - 1) * 0.5f, cyo = (float)(Ho - 1) * 0.5f;
+  if constexpr (DT >= 0) {
+    if (g.rot_on && !g.blur_on && nd == 1 && !(sh.skip & 1)) {   // a8 + a10 straight to the output
+      uint8_t* ob[3];
+      float na[3], nb[3];
+#pragma unroll
+      for (int c = 0; c < 3; ++c) {
+        const ChDest d = ch_dest(p, dests[0], c);
+        ob[c] = d.base;
+        na[c] = d.a;
+        nb[c] = d.b;
+      }
+      rotate_direct<DT>(g, q2, sh.plane, Wo, Ho, warp, nwarps, lane, ob, na, nb);
+      return;
+    }
+  }
   // a8 in place for all three channels when its ring fits the band/Q3 region; else per channel
   bool rotated = false;
   if (g.rot_on && !(sh.skip & 1)) {
@@ -617,10 +750,19 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
         for (; oy < Ho; oy += dy, q += dq, (q >= q4 ? (q -= q4, ++oy) : 0)) {
           const int ox = 4 * q;
           const uint32_t wv = st::lds32(src + (uint32_t)(oy * Wo + ox));
-          const uint64_t q01 = rs::f2::add(rs::f2::pack(__byte_perm(wv, 0x4B000000u, 0x7440), __byte_perm(wv, 0x4B000000u, 0x7441)),
-                                           rs::f2::splat(-rs::kBias));
-          const uint64_t q23 = rs::f2::add(rs::f2::pack(__byte_perm(wv, 0x4B000000u, 0x7442), __byte_perm(wv, 0x4B000000u, 0x7443)),
-                                           rs::f2::splat(-rs::kBias));
+          // 1.5*2^23 + q per byte (the rint-result form put_pair takes)
+          const uint64_t t01 = rs::f2::pack(__byte_perm(wv, 0x4B400000u, 0x7640), __byte_perm(wv, 0x4B400000u, 0x7641));
+          const uint64_t t23 = rs::f2::pack(__byte_perm(wv, 0x4B400000u, 0x7642), __byte_perm(wv, 0x4B400000u, 0x7643));
+          if constexpr (DT >= 0) {
+            if (nd == 1) {
+              const uint64_t na = rs::f2::splat(cd.d0.a), nb = rs::f2::splat(cd.d0.b);
+              uint8_t* o = cd.d0.base + ((size_t)oy * Wo + ox) * dt_bytes<DT>();
+              put_pair<DT>(o, t01, na, nb);
+              put_pair<DT>(o + 2 * dt_bytes<DT>(), t23, na, nb);
+              continue;
+            }
+          }
+          const uint64_t q01 = rs::f2::add(t01, rs::f2::splat(-rs::kRound)), q23 = rs::f2::add(t23, rs::f2::splat(-rs::kRound));
           store_q<DT, VEC>(p, cd, oy, ox, Wo, make_float2(rs::f2::lof(q01), rs::f2::hif(q01)), true);
           store_q<DT, VEC>(p, cd, oy, ox + 2, Wo, make_float2(rs::f2::lof(q23), rs::f2::hif(q23)), true);
         }

@@ -104,15 +104,21 @@ def test_reduced_store_whole_batch(name, n_videos, clips):
         _teardown(store, view)
 
 
-def test_twoview_rotate_blur_sampled_clips():
+@pytest.mark.parametrize("dtype", [configs.BF16, configs.U8, configs.F32])
+def test_twoview_rotate_blur_sampled_clips(dtype):
     w = configs.twoview()
     w.spec.batch_size = 8
+    for v in w.spec.views:
+        v.out_dtype = dtype
     store, view, ospec, ods, vids = _setup(w, 24)
     try:
         for it in range(view.iterations(0, 0)):
             _check_meta(view, w.spec, ospec, ods, 24, 1, 0, it)
         metas = oracle.plan_batch(ospec, ods, 24, 1, 0, 0)
-        assert any(m.rot_on[0] or m.rot_on[1] for m in metas) and any(m.blur_on[0] or m.blur_on[1] for m in metas)
+        # every stencil kernel path is exercised: rotation only (rotated straight to the output),
+        # blur only, rotation then blur, and the plain resample
+        combos = {(bool(m.rot_on[g]), bool(m.blur_on[g])) for m in metas for g in range(2)}
+        assert combos == {(False, False), (True, False), (False, True), (True, True)}, combos
         samples = [(b, k, t) for b in range(8) for k in range(2) for t in (0, 7, 15)]
         _check_outputs(view, w.spec, ospec, ods, vids, 1, 0, 0, samples=samples)
     finally:
