@@ -84,6 +84,24 @@ int sand_store_put_frames(sand_store* s, uint32_t video, uint32_t first_frame, u
                           const uint8_t* uv, uint64_t uv_pitch, uint64_t uv_frame_stride,
                           int src_on_device, sand_stream_t stream);
 
+/* Copy n frames of possibly different videos into the store in one call: frame i is
+ * (videos[i], frames[i]); its Y plane starts at src + i * frame_stride (rows `pitch` bytes
+ * apart) and its interleaved UV plane at src + i * frame_stride + uv_offset (same pitch).
+ * All n frames must have the same width/height (their videos' dims). This is the
+ * decoder-output path of the store (§6: decoded frames become objects of the
+ * store): a host source (src_on_device == 0; pinned memory keeps it asynchronous) is
+ * moved with ONE host->device copy into a store-owned staging buffer, then one scatter
+ * kernel writes every frame into its pitched slot; a device source is scattered directly.
+ * Stream-ordered on `stream`; the caller keeps src valid until the stream reaches the
+ * copy. The call waits (host side) until the previous batch put's scatter has run, so
+ * the staging buffer is never overwritten while still being read. Putting a frame again
+ * overwrites it and resets its counters. Nothing is copied if any (video, frame) is
+ * unknown. Errors: ERANGE (unknown video / frame), EINVAL (null pointers, frames of
+ * different sizes, pitch/uv_offset/frame_stride too small), ECUDA. */
+int sand_store_put_frame_batch(sand_store* s, uint32_t n, const uint32_t* videos, const uint32_t* frames,
+                               const uint8_t* src, uint64_t frame_stride, uint64_t pitch, uint64_t uv_offset,
+                               int src_on_device, sand_stream_t stream);
+
 /* Device address and layout of one stored frame (for tests / zero-copy producers such
  * as a decoder writing NV12 in place). Errors: ERANGE. */
 typedef struct {

@@ -56,7 +56,7 @@ def build_oracle(force=False):
 
 
 PRODUCT_CPP = ["sand_api.cpp", "store.cpp", "planner.cpp", "view.cpp"]
-PRODUCT_CU = ["materialize.cu"]
+PRODUCT_CU = ["materialize.cu", "store_kernels.cu"]
 PRODUCT_HDR = ["internal.h", "plan_types.h", "planner.h", "k_resample.cuh", "k_stream.cuh", "k_stencil.cuh",
                "k_direct.cuh"]
 

@@ -110,6 +110,17 @@ class Store:
                                           uv_ptr, uv_pitch, uv_frame_stride, int(src_on_device), stream),
               "sand_store_put_frames")
 
+    def put_frame_batch(self, videos, frames, src_ptr: int, frame_stride: int, pitch: int, uv_offset: int,
+                        src_on_device: bool, stream: int = 0) -> None:
+        """n frames of any videos from one packed buffer (one H2D copy + one scatter kernel)."""
+        n = len(videos)
+        assert len(frames) == n
+        va = (ctypes.c_uint32 * max(n, 1))(*videos)
+        fa = (ctypes.c_uint32 * max(n, 1))(*frames)
+        check(lib().sand_store_put_frame_batch(self._h, n, ctypes.cast(va, ctypes.c_void_p),
+                                               ctypes.cast(fa, ctypes.c_void_p), src_ptr, frame_stride, pitch,
+                                               uv_offset, int(src_on_device), stream), "sand_store_put_frame_batch")
+
     def frame_layout(self, video: int, frame: int) -> _abi.sand_frame_layout:
         out = _abi.sand_frame_layout()
         check(lib().sand_store_frame_layout(self._h, video, frame, ctypes.byref(out)), "sand_store_frame_layout")

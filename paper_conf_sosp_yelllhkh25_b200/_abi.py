@@ -88,6 +88,7 @@ SIGNATURES = {
     "sand_store_create": (ctypes.c_int, [ctypes.c_int, u64, P(vp)]),
     "sand_store_add_video": (ctypes.c_int, [vp, u32, u32, u32, u32]),
     "sand_store_put_frames": (ctypes.c_int, [vp, u32, u32, u32, vp, u64, u64, vp, u64, u64, ctypes.c_int, vp]),
+    "sand_store_put_frame_batch": (ctypes.c_int, [vp, u32, vp, vp, vp, u64, u64, u64, ctypes.c_int, vp]),
     "sand_store_frame_layout": (ctypes.c_int, [vp, u32, u32, P(sand_frame_layout)]),
     "sand_store_mark_present": (ctypes.c_int, [vp, u32, u32, u32]),
     "sand_store_counters": (ctypes.c_int, [vp, P(sand_counters)]),

@@ -35,6 +35,20 @@ struct VideoEntry {
 
 }  // namespace sand
 
+namespace sand {
+// one frame of sand_store_put_frame_batch: source (packed buffer) and destination (slab) offsets
+struct PutDesc {
+  uint64_t src;       // byte offset of the frame's Y plane in the source buffer
+  uint64_t dst;       // byte offset of the frame's slot in the slab
+  uint32_t width, height, dst_pitch, pad;
+};
+// scatter n packed frames (Y rows then UV rows, source row pitch src_pitch, UV plane at
+// src + uv_offset) into their slab slots with `word`-byte (16, 4 or 1) copies; stream-ordered
+// (store_kernels.cu)
+int launch_put_scatter(const uint8_t* src, uint64_t src_pitch, uint64_t uv_offset, uint8_t* slab,
+                       const PutDesc* desc, uint32_t n, int word, cudaStream_t stream);
+}  // namespace sand
+
 struct sand_store {
   int device = 0;
   uint8_t* slab = nullptr;
@@ -43,6 +57,14 @@ struct sand_store {
   std::atomic<int> live_views{0};
   uint64_t batches = 0;
   std::mutex mu;   // guards counters updated by read_batch (views may live on several threads)
+  // sand_store_put_frame_batch: device staging of packed host frames + per-frame descriptors,
+  // reused across calls once `put_done` (recorded after the scatter) has completed
+  uint8_t* put_stage = nullptr;
+  uint64_t put_stage_bytes = 0;
+  sand::PutDesc* put_desc = nullptr;        // device
+  sand::PutDesc* put_desc_host = nullptr;   // pinned
+  uint32_t put_desc_cap = 0;
+  cudaEvent_t put_done = nullptr;
 };
 
 namespace sand {

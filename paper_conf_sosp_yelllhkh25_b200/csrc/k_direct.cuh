@@ -72,6 +72,9 @@ __device__ __forceinline__ void hrows(rs::Row3* out, const uint8_t* __restrict__
 // One CTA = one work item x one band of RB output rows x one chunk of P column pairs; the
 // band is split into two halves and thread t = (half t / P, column pair chunk * P + t % P),
 // so P = 112 gives 224 threads (seven full warps) for 224-wide outputs.
+#ifndef SAND_DIRECT_PF
+#define SAND_DIRECT_PF 0
+#endif
 #ifndef SAND_DIRECT_MINB
 #define SAND_DIRECT_MINB 3
 #endif
@@ -118,6 +121,57 @@ __global__ void __launch_bounds__(256, SAND_DIRECT_MINB) k_direct(const LaunchPa
         dl[d] = make_dest(p, dests[d], oy0, ox);
         dt[d] = DT >= 0 ? DT : p.views[dests[d] >> 24].dtype;
       }
+#if SAND_DIRECT_PF
+    // software-pipelined walk: the 16 NV12 loads of output row rr + 1 are in flight while row
+    // rr is converted, lerped and stored (both tap rows are reconverted every row, which only
+    // repeats work when the vertical step is below 2)
+    {
+      uint32_t Yc[2][4], UVc[2][4];
+      float lyc;
+      auto load_row = [&](int oy, uint32_t (&Yv)[2][4], uint32_t (&UVv)[2][4], float& ly) {
+        int y0, y1;
+        tap(g.sc_y, g.off_y, oy, g.lim_y, g.org_y, y0, y1, ly);
+        const int xs[4] = {xa0, xa1, xb0, xb1};
+        const int ys[2] = {y0, y1};
+#pragma unroll
+        for (int r = 0; r < 2; ++r) {
+          const uint8_t* yr = Yp + (size_t)ys[r] * pitch;
+          const uint8_t* uvr = UVp + (size_t)(ys[r] >> 1) * pitch;
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            Yv[r][k] = __ldg(yr + xs[k]);
+            UVv[r][k] = __ldg(reinterpret_cast<const uint16_t*>(uvr + (xs[k] & ~1)));
+          }
+        }
+      };
+      load_row(oy0, Yc, UVc, lyc);
+      for (int rr = 0; rr < nr; ++rr) {
+        uint32_t Yn[2][4], UVn[2][4];
+        float lyn = 0.f;
+        if (rr + 1 < nr) load_row(oy0 + rr + 1, Yn, UVn, lyn);
+        Row3 tb[2];
+#pragma unroll
+        for (int r = 0; r < 2; ++r) {
+          dg::Px3 q[4];
+#pragma unroll
+          for (int k = 0; k < 4; ++k) q[k] = dg::px3(Yc[r][k], UVc[r][k]);
+#pragma unroll
+          for (int c = 0; c < 3; ++c) tb[r].h[c] = dg::hlerp_b(q[0].c[c], q[1].c[c], q[2].c[c], q[3].c[c], lx);
+        }
+        // y1 == y0 at the bottom edge: both rows are the same row, lerp weight irrelevant
+        emit<DT, kInlineDests, VEC>(tb[0], tb[1], lyc, dl, dt, p, dests, nd, oy0 + rr, ox, vec, has_b);
+#pragma unroll
+        for (int r = 0; r < 2; ++r)
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            Yc[r][k] = Yn[r][k];
+            UVc[r][k] = UVn[r][k];
+          }
+        lyc = lyn;
+      }
+    }
+    return;
+#endif
     Row3 T, B;              // horizontal lerps of source rows yT (top) and yB (bottom)
     int yT = -1, yB = -1;
     for (int rr = 0; rr < nr; ++rr) {

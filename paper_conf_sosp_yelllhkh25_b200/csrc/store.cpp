@@ -4,6 +4,7 @@
 // one pitched device slab, NV12, row pitch a multiple of 64 B.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstring>
 
 #include "internal.h"
@@ -99,6 +100,90 @@ extern "C" int sand_store_put_frames(sand_store* s, uint32_t video, uint32_t fir
   return SAND_OK;
 }
 
+extern "C" int sand_store_put_frame_batch(sand_store* s, uint32_t n, const uint32_t* videos, const uint32_t* frames,
+                                          const uint8_t* src, uint64_t frame_stride, uint64_t pitch,
+                                          uint64_t uv_offset, int src_on_device, sand_stream_t stream) {
+  if (!s || (n > 0 && (!videos || !frames || !src))) return sand::set_error(SAND_EINVAL, "null argument");
+  if (n == 0) return SAND_OK;
+  std::lock_guard<std::mutex> lk(s->mu);
+  // validate every (video, frame) first: nothing is copied on error
+  uint32_t width = 0, height = 0;
+  for (uint32_t i = 0; i < n; ++i) {
+    auto it = s->videos.find(videos[i]);
+    if (it == s->videos.end() || frames[i] >= it->second.n_frames)
+      return sand::set_error(SAND_ERANGE, "unknown (video, frame) in batch put");
+    const VideoEntry& v = it->second;
+    if (i == 0) {
+      width = v.width;
+      height = v.height;
+    } else if (v.width != width || v.height != height) {
+      return sand::set_error(SAND_EINVAL, "batch put frames must share width and height");
+    }
+  }
+  if (pitch < width || uv_offset < pitch * height || frame_stride < uv_offset + pitch * (height / 2 - 1) + width)
+    return sand::set_error(SAND_EINVAL, "pitch / uv_offset / frame_stride do not fit the frames");
+  cudaError_t e = cudaSetDevice(s->device);
+  if (e != cudaSuccess) return sand::cuda_error(e, "cudaSetDevice");
+  auto st = static_cast<cudaStream_t>(stream);
+  if (!s->put_done) {
+    e = cudaEventCreateWithFlags(&s->put_done, cudaEventDisableTiming);
+    if (e != cudaSuccess) return sand::cuda_error(e, "cudaEventCreate(put_done)");
+  }
+  // the staging buffers of the previous call are reusable once its scatter has run
+  e = cudaEventSynchronize(s->put_done);
+  if (e != cudaSuccess) return sand::cuda_error(e, "cudaEventSynchronize(put_done)");
+  if (s->put_desc_cap < n) {
+    cudaFree(s->put_desc);
+    cudaFreeHost(s->put_desc_host);
+    s->put_desc = nullptr;
+    s->put_desc_host = nullptr;
+    s->put_desc_cap = 0;
+    const uint32_t cap = std::max<uint32_t>(n, 1024);
+    e = cudaMalloc(reinterpret_cast<void**>(&s->put_desc), sizeof(sand::PutDesc) * cap);
+    if (e == cudaSuccess) e = cudaMallocHost(reinterpret_cast<void**>(&s->put_desc_host), sizeof(sand::PutDesc) * cap);
+    if (e != cudaSuccess) return sand::cuda_error(e, "batch put descriptor buffers");
+    s->put_desc_cap = cap;
+  }
+  const uint64_t bytes = frame_stride * (n - 1) + uv_offset + pitch * (height / 2 - 1) + width;
+  const uint8_t* dsrc = src;
+  if (!src_on_device) {                  // one host->device transfer of the whole packed batch
+    if (s->put_stage_bytes < bytes) {
+      cudaFree(s->put_stage);
+      s->put_stage = nullptr;
+      s->put_stage_bytes = 0;
+      e = cudaMalloc(reinterpret_cast<void**>(&s->put_stage), bytes);
+      if (e != cudaSuccess) return sand::cuda_error(e, "batch put staging buffer");
+      s->put_stage_bytes = bytes;
+    }
+    e = cudaMemcpyAsync(s->put_stage, src, bytes, cudaMemcpyHostToDevice, st);
+    if (e != cudaSuccess) return sand::cuda_error(e, "cudaMemcpyAsync(batch put)");
+    dsrc = s->put_stage;
+  }
+  for (uint32_t i = 0; i < n; ++i) {
+    VideoEntry& v = s->videos.find(videos[i])->second;
+    sand::PutDesc& d = s->put_desc_host[i];
+    d.src = frame_stride * i;
+    d.dst = v.offset + v.frame_stride * frames[i];
+    d.width = v.width;
+    d.height = v.height;
+    d.dst_pitch = v.pitch;
+    d.pad = 0;
+    v.present[frames[i]] = 1;
+    v.fetches[frames[i]] = 0;
+    v.uses[frames[i]] = 0;
+  }
+  e = cudaMemcpyAsync(s->put_desc, s->put_desc_host, sizeof(sand::PutDesc) * n, cudaMemcpyHostToDevice, st);
+  if (e != cudaSuccess) return sand::cuda_error(e, "cudaMemcpyAsync(batch put descriptors)");
+  // widest copy word every row start allows (slab rows are 64 B aligned)
+  const uint64_t al = reinterpret_cast<uintptr_t>(dsrc) | frame_stride | pitch | uv_offset | width;
+  const int word = (al & 15) == 0 ? 16 : ((al & 3) == 0 ? 4 : 1);
+  const int rc = sand::launch_put_scatter(dsrc, pitch, uv_offset, s->slab, s->put_desc, n, word, st);
+  if (rc != SAND_OK) return rc;
+  e = cudaEventRecord(s->put_done, st);
+  if (e != cudaSuccess) return sand::cuda_error(e, "cudaEventRecord(put_done)");
+  return SAND_OK;
+}
+
 extern "C" int sand_store_frame_layout(const sand_store* s, uint32_t video, uint32_t frame,
                                        sand_frame_layout* out) {
   if (!s || !out) return sand::set_error(SAND_EINVAL, "null argument");
@@ -171,6 +256,10 @@ extern "C" int sand_store_destroy(sand_store* s) {
   cudaSetDevice(s->device);
   cudaDeviceSynchronize();
   cudaFree(s->slab);
+  cudaFree(s->put_stage);
+  cudaFree(s->put_desc);
+  cudaFreeHost(s->put_desc_host);
+  if (s->put_done) cudaEventDestroy(s->put_done);
   delete s;
   return SAND_OK;
 }

@@ -249,3 +249,68 @@ def test_error_paths():
     finally:
         view.close()
         store.close()
+
+
+# ------------------------------------------------------------------ batch put (decoder-output path)
+
+def test_batch_put_matches_per_frame_fill():
+    """sand_store_put_frame_batch (one H2D copy + scatter kernel) stores the same bytes as the
+    per-frame path: the batch read from a store filled frame batch by frame batch is
+    bit-identical to the one read from a store filled by the device generator."""
+    w = configs.k400()
+    n_videos = 8
+    w.spec.batch_size = 4
+    vids = videos_of(w, n_videos)
+    store_a, view_a, ospec, ods, _ = _setup(w, n_videos)
+    W, H, F = w.width, w.height, w.n_frames
+    fb = W * H * 3 // 2
+    per_frame = (W + 63) // 64 * 64 * H * 3 // 2 + 256
+    store_b = sand.Store(0, len(vids) * F * per_frame + (1 << 20))
+    try:
+        for v in vids:
+            store_b.add_video(v[0], F, W, H)
+        chunk = 100                              # several calls: the staging buffer is reused
+        for v in vids:
+            for f0 in range(0, F, chunk):
+                n = min(chunk, F - f0)
+                y, uv = synth.frames(synth.UNIFORM, SEED, v[0], f0, n, W, H)
+                host = torch.empty((n, fb), dtype=torch.uint8).pin_memory()
+                hv = host.numpy()
+                hv[:, : W * H] = y.reshape(n, -1)
+                hv[:, W * H:] = uv.reshape(n, -1)
+                # frames given in reverse order: the scatter follows the (video, frame) lists
+                order = list(range(n))[::-1]
+                packed = torch.stack([host[i] for i in order]).pin_memory()
+                store_b.put_frame_batch([v[0]] * n, [f0 + i for i in order], packed.data_ptr(), fb, W, W * H,
+                                        False, torch.cuda.current_stream().cuda_stream)
+                torch.cuda.synchronize()
+        assert store_b.counters().frames_present == n_videos * F
+        view_b = sand.View(store_b, w.spec, [v[0] for v in vids])
+        try:
+            for it in range(view_a.iterations(0, 0)):
+                oa, ob = view_a.alloc_outputs(), view_b.alloc_outputs()
+                view_a.read_batch(0, 0, it, oa)
+                view_b.read_batch(0, 0, it, ob)
+                torch.cuda.synchronize()
+                for x, y2 in zip(oa, ob):
+                    assert torch.equal(x.view(torch.int16), y2.view(torch.int16))
+        finally:
+            view_b.close()
+    finally:
+        _teardown(store_a, view_a)
+        store_b.close()
+
+
+def test_batch_put_rejects_unknown_frames():
+    store = sand.Store(0, 1 << 24)
+    try:
+        store.add_video(5, 4, 64, 64)
+        buf = torch.zeros(64 * 64 * 3 // 2 * 2, dtype=torch.uint8, device="cuda")
+        with pytest.raises(sand.SandError):
+            store.put_frame_batch([5, 5], [0, 4], buf.data_ptr(), 64 * 96, 64, 64 * 64, True)
+        assert store.counters().frames_present == 0      # nothing copied on error
+        store.put_frame_batch([5, 5], [0, 3], buf.data_ptr(), 64 * 96, 64, 64 * 64, True)
+        torch.cuda.synchronize()
+        assert store.counters().frames_present == 2
+    finally:
+        store.close()

@@ -72,8 +72,12 @@ def main():
     rep, obj, kernel = sys.argv[1:4]
     top = int(sys.argv[4]) if len(sys.argv) > 4 else 40
     mangled = sys.argv[5] if len(sys.argv) > 5 else kernel
-    csvtxt = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
-                            capture_output=True, text=True).stdout
+    if rep.endswith(".csv.gz"):      # a saved `--page source --print-source sass --csv` export
+        import gzip
+        csvtxt = gzip.open(rep, "rt").read()
+    else:
+        csvtxt = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
+                                capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(csvtxt)))
     hdr = None
     blocks, cur = [], None
