@@ -164,6 +164,9 @@ typedef struct {
   uint32_t n_videos;
   uint32_t n_views;         /* 1..SAND_MAX_VIEWS                                        */
   int32_t shared_window;    /* P:L295 shared window across RRC groups (R#18)           */
+  uint32_t pool_epochs;     /* k: a clip's shared frame pool is drawn once per chunk of
+                               k epochs and reused by all of them ("decoded once and
+                               cached for exactly k epochs"; R#25); 0 or 1: every epoch   */
   sand_view_desc views[SAND_MAX_VIEWS];
 } sand_view_spec;
 

@@ -46,7 +46,7 @@ class Spec(ctypes.Structure):
     _fields_ = [
         ("seed", ctypes.c_uint64), ("world_size", ctypes.c_uint32), ("batch_size", ctypes.c_uint32),
         ("samples_per_video", ctypes.c_uint32), ("drop_last", ctypes.c_int32),
-        ("n_views", ctypes.c_uint32), ("shared_window", ctypes.c_int32),
+        ("n_views", ctypes.c_uint32), ("shared_window", ctypes.c_int32), ("pool_epochs", ctypes.c_uint32),
         ("views", View * MAX_VIEWS),
     ]
 
@@ -300,6 +300,7 @@ class SpecDesc:
     samples_per_video: int = 1
     drop_last: bool = False
     shared_window: bool = False
+    pool_epochs: int = 1
     views: list = field(default_factory=lambda: [ViewDesc()])
 
 
@@ -311,6 +312,7 @@ def make_spec(sd: SpecDesc) -> Spec:
     s.samples_per_video = sd.samples_per_video
     s.drop_last = int(sd.drop_last)
     s.shared_window = int(sd.shared_window)
+    s.pool_epochs = int(sd.pool_epochs)
     s.n_views = len(sd.views)
     for i, v in enumerate(sd.views):
         o = s.views[i]

@@ -61,6 +61,7 @@ typedef struct {
   int32_t drop_last;
   uint32_t n_views;
   int32_t shared_window;           /* P:L295 shared window over all RRC groups */
+  uint32_t pool_epochs;            /* pool drawn once per chunk of k epochs (R#25) */
   oracle_view views[OR_MAX_VIEWS];
 } oracle_spec;
 
@@ -184,7 +185,10 @@ void oracle_temporal(const oracle_spec* spec, uint64_t epoch, uint32_t clip, uin
   uint32_t P = (L - 1) * g + 1;                  /* frames covered by the pool */
   uint32_t F = n_frames_video;
   uint32_t x[4];
-  draw(spec->seed, OR_TEMPORAL, 0, 0, 0, clip, epoch, x);
+  /* "videos are decoded once and cached for exactly k epochs before refreshing" --
+     the pool start is drawn per chunk floor(epoch / k); offsets below stay per epoch (R#25) */
+  uint64_t chunk = spec->pool_epochs > 1 ? epoch / spec->pool_epochs : epoch;
+  draw(spec->seed, OR_TEMPORAL, 0, 0, 0, clip, chunk, x);
   uint32_t start = oracle_bounded(x[0], (F > P ? F - P : 0) + 1);
   meta->pool_start = start;
   for (uint32_t k = 0; k < spec->n_views; ++k) {

@@ -46,6 +46,7 @@ def make_spec(spec: Spec, videos) -> tuple[_abi.sand_view_spec, object]:
     s.n_videos = len(videos)
     s.n_views = len(spec.views)
     s.shared_window = int(spec.shared_window)
+    s.pool_epochs = int(getattr(spec, "pool_epochs", 1))
     for i, v in enumerate(spec.views):
         o = s.views[i]
         o.clip_len, o.stride, o.pool_offset, o.spatial_group = v.clip_len, v.stride, v.pool_offset, v.spatial_group

@@ -51,7 +51,7 @@ class sand_view_spec(ctypes.Structure):
     _fields_ = [
         ("seed", u64), ("world_size", u32), ("batch_size", u32), ("samples_per_video", u32),
         ("drop_last", i32), ("videos", ctypes.POINTER(u32)), ("n_videos", u32), ("n_views", u32),
-        ("shared_window", i32), ("views", sand_view_desc * MAX_VIEWS),
+        ("shared_window", i32), ("pool_epochs", u32), ("views", sand_view_desc * MAX_VIEWS),
     ]
 
 

@@ -47,6 +47,7 @@ class Spec:
     samples_per_video: int = 1
     drop_last: bool = False
     shared_window: bool = False
+    pool_epochs: int = 1          # k-epoch shared frame pool
     views: list = field(default_factory=lambda: [ViewSpec()])
 
 

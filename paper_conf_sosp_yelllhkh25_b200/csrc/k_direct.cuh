@@ -73,7 +73,7 @@ __device__ __forceinline__ void hrows(rs::Row3* out, const uint8_t* __restrict__
 // band is split into two halves and thread t = (half t / P, column pair chunk * P + t % P),
 // so P = 112 gives 224 threads (seven full warps) for 224-wide outputs.
 #ifndef SAND_DIRECT_PF
-#define SAND_DIRECT_PF 0
+#define SAND_DIRECT_PF 1
 #endif
 #ifndef SAND_DIRECT_MINB
 #define SAND_DIRECT_MINB 3

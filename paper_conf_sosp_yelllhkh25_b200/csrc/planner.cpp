@@ -189,7 +189,11 @@ void plan_clip(const SpecInfo& info, uint64_t epoch, uint32_t clip, sand_clip_me
   // a2: shared frame pool (R#4, R#5)
   const uint32_t g = info.g, L = info.pool_len;
   const uint32_t pool_frames = (L - 1) * g + 1;
-  const uint32_t start = draw_below(d.get(Purpose::kTemporal, 0, 0, 0, clip)[0],
+  // the pool is drawn once per chunk of k = pool_epochs epochs (R#25); the views'
+  // offsets inside it stay per epoch
+  const uint64_t chunk = s.pool_epochs > 1 ? epoch / s.pool_epochs : epoch;
+  const EpochDraws dpool(s.seed, chunk);
+  const uint32_t start = draw_below(dpool.get(Purpose::kTemporal, 0, 0, 0, clip)[0],
                                     (F > pool_frames ? F - pool_frames : 0u) + 1u);
   m->pool_start = start;
   for (uint32_t k = 0; k < s.n_views; ++k) {

@@ -25,7 +25,7 @@ def to_oracle(spec) -> oracle.Spec:
                              out_dtype=v.out_dtype) for v in spec.views]
     return oracle.make_spec(oracle.SpecDesc(seed=spec.seed, world_size=spec.world_size,
                                             batch_size=spec.batch_size, samples_per_video=spec.samples_per_video,
-                                            drop_last=spec.drop_last, shared_window=spec.shared_window,
+                                            drop_last=spec.drop_last, shared_window=spec.shared_window, pool_epochs=spec.pool_epochs,
                                             views=views))
 
 

@@ -308,3 +308,70 @@ def test_world_size_invariance_of_clip_plans():
                 assert oracle.meta_to_dict(spec8, m) == by_clip[m.clip]
                 seen += 1
     assert seen == 64
+
+
+# ------------------------------------------------------------------ §8(f) f1: k-epoch shared frame pool
+
+def _pool_meta(spec_desc, vids, epoch, clip):
+    ospec = oracle.make_spec(spec_desc)
+    ods = oracle.make_dataset(vids)
+    ref = oracle.ClipMeta()
+    oracle.lib().oracle_plan_clip(oracle.ctypes.byref(ospec), ods, epoch, clip, oracle.ctypes.byref(ref))
+    return ref
+
+
+def _k400_desc(k, views=None):
+    views = views or [oracle.ViewDesc(clip_len=16, stride=4, out_h=224, out_w=224)]
+    return oracle.SpecDesc(seed=11, batch_size=4, pool_epochs=k, views=views)
+
+
+def test_k_epoch_pool_is_the_chunk_pool():
+    """P:L270 (pool cached for exactly k epochs), R#25: with pool_epochs = k the pool start of
+    epoch e is the start the per-epoch planner (k = 1) draws at epoch floor(e / k); k = 0 and
+    k = 1 are the per-epoch planner itself."""
+    vids = [(1000 + i, 300, 340, 256) for i in range(12)]
+    for clip in range(12):
+        for e in range(13):
+            one = _pool_meta(_k400_desc(1), vids, e, clip)
+            assert _pool_meta(_k400_desc(0), vids, e, clip).pool_start == one.pool_start
+            for k in (2, 5):
+                got = _pool_meta(_k400_desc(k), vids, e, clip)
+                chunk = _pool_meta(_k400_desc(1), vids, e // k, clip)
+                assert got.pool_start == chunk.pool_start
+                assert list(got.frames[0][:16]) == list(chunk.frames[0][:16])   # single view: span == pool
+
+
+def test_k_epoch_pool_keeps_per_epoch_offsets_and_spatial_draws():
+    """Inside a chunk the pool is fixed, but a view shorter than the pool still draws its offset
+    per epoch, and the spatial draws stay per epoch (randomness preserved)."""
+    vids = [(1000 + i, 150, 1920, 1080) for i in range(16)]
+    views = [oracle.ViewDesc(clip_len=16, stride=4, out_h=224, out_w=224),
+             oracle.ViewDesc(clip_len=8, stride=4, out_h=224, out_w=224, spatial_group=1)]
+    desc = _k400_desc(10, views)
+    offsets_vary = boxes_vary = 0
+    for clip in range(16):
+        m = [_pool_meta(desc, vids, e, clip) for e in range(10)]
+        assert len({x.pool_start for x in m}) == 1
+        offsets_vary += len({x.frames[1][0] for x in m}) > 1
+        boxes_vary += len({tuple(x.box[0]) for x in m}) > 1
+    assert offsets_vary >= 12 and boxes_vary == 16
+
+
+def test_k_epoch_pool_frame_reuse_over_ten_epochs():
+    """Fig. 19 analogue on synthetic 300-frame videos, K400 clips (16 x stride 4):
+    over ten epochs every selected frame is selected ten times with k = 10, while with fresh
+    pools (k = 1) few frames are selected four or more times."""
+    vids = [(1000 + i, 300, 340, 256) for i in range(64)]
+
+    def counts(k):
+        c = {}
+        for e in range(10):
+            for clip in range(64):
+                m = _pool_meta(_k400_desc(k), vids, e, clip)
+                for f in m.frames[0][:16]:
+                    c[(m.video, f)] = c.get((m.video, f), 0) + 1
+        return np.array(list(c.values()))
+
+    c1, c10 = counts(1), counts(10)
+    assert np.all(c10 == 10)
+    assert np.mean(c1 >= 4) < 0.15

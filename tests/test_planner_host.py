@@ -73,3 +73,19 @@ def test_invalid_specs_rejected_on_host():
     two.views[1].spatial_group = 0           # same group, different augmentation -> invalid
     with pytest.raises(sand.SandError):
         sand.plan_clip(two, videos_of(configs.twoview(), 4), 0, 0)
+
+
+@pytest.mark.parametrize("name,k", [("k400", 4), ("slowfast", 10), ("ray", 3)])
+def test_host_plan_k_epoch_pool_matches_oracle(name, k):
+    """§8(f) f1: with pool_epochs = k the host planner still matches the oracle bit-exactly."""
+    w = configs.get(name)
+    w.spec.pool_epochs = k
+    vids = videos_of(w, min(w.n_videos, 32))
+    ospec = to_oracle(w.spec)
+    ods = oracle.make_dataset(vids)
+    for epoch in (0, k - 1, k, 3 * k + 1):
+        for clip in range(0, len(vids), 3):
+            got = sand.plan_clip(w.spec, vids, epoch, clip)
+            ref = oracle.ClipMeta()
+            oracle.lib().oracle_plan_clip(oracle.ctypes.byref(ospec), ods, epoch, clip, oracle.ctypes.byref(ref))
+            assert meta_fields(w.spec, got) == meta_fields(w.spec, ref), (name, k, epoch, clip)
