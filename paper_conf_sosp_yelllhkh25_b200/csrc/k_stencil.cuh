@@ -169,6 +169,11 @@ __device__ __forceinline__ uint64_t add_rm2(uint64_t a, uint64_t b) {
   return d;
 }
 
+#ifndef SAND_ROT_RPW
+#define SAND_ROT_RPW 2
+#endif
+constexpr int kRotRPW = SAND_ROT_RPW;   // Q3 rows per warp per ring band (fewer barriers)
+
 // Rotation (R#15) of all three Q2 planes in place. Q3 rows are computed band by band (one
 // row per warp) into a ring of ring_rows (a power of two) rows, and row r is written back over
 // Q2 row r once no later Q3 row can tap it: every tap of Q3 row y lies in Q2 rows
@@ -183,8 +188,10 @@ __device__ __forceinline__ void rotate_inplace(const GroupParams& g, uint32_t q2
   const uint64_t c2 = f2::pack(cxo, cyo), kr2 = f2::splat(kRound), nkr2 = f2::splat(-kRound);
   const uint64_t nb2 = f2::splat(-kBias), m1 = f2::splat(-1.f);
   int committed = 0;   // Q2 rows [0, committed) hold Q3 already
-  for (int yb = 0; yb < Ho; yb += nwarps) {
-    const int oy = yb + warp;
+  for (int yb = 0; yb < Ho; yb += kRotRPW * nwarps) {
+#pragma unroll 1
+   for (int qr = 0; qr < kRotRPW; ++qr) {
+    const int oy = yb + qr * nwarps + warp;
     if (oy < Ho) {
       const float yc = __fsub_rn((float)oy, cyo);
       const uint64_t txy = f2::pack(__fmul_rn(nrs, yc), __fmul_rn(rc, yc));   // row terms
@@ -228,8 +235,9 @@ __device__ __forceinline__ void rotate_inplace(const GroupParams& g, uint32_t q2
         }
       }
     }
+   }
     __syncthreads();                     // ring rows of this band written; Q2 reads done
-    const int last = min(yb + nwarps, Ho) - 1;
+    const int last = min(yb + kRotRPW * nwarps, Ho) - 1;
     const int upto = last + 1 >= Ho ? Ho : max(committed, last - D + 1);   // rows < upto are dead in Q2
     if (upto > committed) {              // write back Q3 rows [committed, upto) of the three planes
 #pragma unroll 1
@@ -473,21 +481,26 @@ __device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupPar
 #pragma unroll
         for (int o = 0; o < kBV; ++o) accs[o] = 0ull;
         const uint32_t a0 = scratch + 4u * (uint32_t)(y0 * Wo + ox);
-        const bool full = y0 + kBV + 2 * R <= jrows;
+        if (pair_ok && y0 + kBV + 2 * R <= jrows) {   // fast path: no per-row branches or clamps
 #pragma unroll
-        for (int k = 0; k < kBV + 2 * R; ++k) {
-          // rows past the strip only feed outputs that are not stored: clamp their address
-          const uint32_t a = full ? a0 + rstep * k : scratch + 4u * (uint32_t)(min(y0 + k, jrows - 1) * Wo + ox);
-          uint64_t v;
-          if (pair_ok) {
-            const float2 f = lds64f(a);
-            v = rs::f2::pack(f.x, f.y);
-          } else {
-            v = rs::f2::pack(st::lds32(a), has_b ? st::lds32(a + 4) : 0u);
+          for (int k = 0; k < kBV + 2 * R; ++k) {
+            const float2 f = lds64f(a0 + rstep * k);
+            const uint64_t v = rs::f2::pack(f.x, f.y);
+#pragma unroll
+            for (int o = 0; o < kBV; ++o)
+              if (k - o >= 0 && k - o <= 2 * R) accs[o] = rs::f2::fma(rs::f2::splat(wt[k - o]), v, accs[o]);
           }
+        } else {
 #pragma unroll
-          for (int o = 0; o < kBV; ++o)
-            if (k - o >= 0 && k - o <= 2 * R) accs[o] = rs::f2::fma(rs::f2::splat(wt[k - o]), v, accs[o]);
+          for (int k = 0; k < kBV + 2 * R; ++k) {
+            // rows past the strip only feed outputs that are not stored: clamp their address
+            const uint32_t a = scratch + 4u * (uint32_t)(min(y0 + k, jrows - 1) * Wo + ox);
+            const uint32_t xa = st::lds32(a), xb = st::lds32(a + (has_b ? 4u : 0u));
+            const uint64_t v = rs::f2::pack(xa, has_b ? xb : 0u);
+#pragma unroll
+            for (int o = 0; o < kBV; ++o)
+              if (k - o >= 0 && k - o <= 2 * R) accs[o] = rs::f2::fma(rs::f2::splat(wt[k - o]), v, accs[o]);
+          }
         }
         if constexpr (DT >= 0) {
           if (fast_st) {                     // one destination: incremental row pointer
@@ -666,7 +679,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
     const float bound = fabsf(g.rot_s) * cxo + (1.f - g.rot_c) * cyo;
     const int D = (int)ceilf(bound) + 2;
     int ring_rows = 1;
-    while (ring_rows < D + nwarps + 1) ring_rows <<= 1;
+    while (ring_rows < D + kRotRPW * nwarps + 1) ring_rows <<= 1;
     if ((size_t)ring_rows * 3 * Wo <= sh.ubytes && D < Ho) {
       rotate_inplace(g, q2, sh.plane, ureg, ring_rows, D, Wo, Ho, warp, nwarps, lane);
       rotated = true;
