@@ -505,12 +505,17 @@ __device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupPar
         if constexpr (DT >= 0) {
           if (fast_st) {                     // one destination: incremental row pointer
             uint8_t* o = obase + ((size_t)(ys + y0) * Wo + ox) * dt_bytes<DT>();
-            const size_t rsb = (size_t)Wo * dt_bytes<DT>();
+            const uint32_t rsb = (uint32_t)Wo * dt_bytes<DT>();
+            if (y0 + kBV <= ns) {            // whole block: no per-row checks
 #pragma unroll
-            for (int oo = 0; oo < kBV; ++oo) {
-              if (y0 + oo >= ns) break;
-              put_pair<DT>(o, rs::f2::add(accs[oo], rs::f2::splat(rs::kRound)), na, nb);
-              o += rsb;
+              for (int oo = 0; oo < kBV; ++oo)
+                put_pair<DT>(o + oo * rsb, rs::f2::add(accs[oo], rs::f2::splat(rs::kRound)), na, nb);
+            } else {
+#pragma unroll
+              for (int oo = 0; oo < kBV; ++oo) {
+                if (y0 + oo >= ns) break;
+                put_pair<DT>(o + oo * rsb, rs::f2::add(accs[oo], rs::f2::splat(rs::kRound)), na, nb);
+              }
             }
             continue;
           }
