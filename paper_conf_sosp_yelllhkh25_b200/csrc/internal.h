@@ -141,6 +141,10 @@ struct sand_view {
   uint32_t sched_seq = 0;        // next slot pair
   size_t n_buffers = 0;          // plan buffers allocated so far
   std::vector<cudaEvent_t> inflight;   // ring of per-batch completion events (read-ahead bound)
+  // batches with both direct and stencil items: the direct kernel runs on aux_stream (forked
+  // from / joined to the caller's stream) so it fills the SMs the stencil kernel's tail leaves idle
+  cudaStream_t aux_stream = nullptr;
+  cudaEvent_t fork_ev = nullptr, join_ev = nullptr;
 };
 
 namespace sand {
@@ -153,7 +157,8 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
 // kernels (materialize.cu)
 size_t stencil_smem_bytes(int max_h, int max_w, int max_r);
 int configure_kernels(size_t stencil_smem);
+// aux/fork/join may be null (then the kernels run back to back on `stream`)
 int launch_materialize(const LaunchParams& p, const BatchShape& shape, size_t stencil_smem, cudaStream_t stream,
-                       int* n_launched);
+                       cudaStream_t aux, cudaEvent_t fork, cudaEvent_t join, int* n_launched);
 
 }  // namespace sand

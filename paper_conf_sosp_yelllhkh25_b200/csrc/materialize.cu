@@ -379,23 +379,19 @@ int configure_kernels(size_t stencil_smem) {
 }
 
 int launch_materialize(const LaunchParams& p, const BatchShape& shape, size_t stencil_smem, cudaStream_t stream,
-                       int* n_launched) {
+                       cudaStream_t aux, cudaEvent_t fork, cudaEvent_t join, int* n_launched) {
   *n_launched = 0;
   if (p.n_items == 0) return SAND_OK;
-  if (shape.has_direct) {
-    LaunchParams pd = p;
-    pd.n_items = shape.n_direct;
-    int rc;
-    // specialised instantiations: one dtype for every view and even output widths (the
-    // 4-byte pair stores are aligned); anything else takes the generic instantiation
-    switch (shape.even_wo ? shape.dtype : -1) {
-      case SAND_U8: rc = launch_resample_dt<SAND_U8, true>(pd, shape, stream); break;
-      case SAND_BF16: rc = launch_resample_dt<SAND_BF16, true>(pd, shape, stream); break;
-      case SAND_F32: rc = launch_resample_dt<SAND_F32, true>(pd, shape, stream); break;
-      default: rc = launch_resample_dt<-1, false>(pd, shape, stream); break;
-    }
-    if (rc != SAND_OK) return rc;
-    ++*n_launched;
+  // both kinds in one batch: the stencil kernel (one 227 KB CTA per SM) goes first on the
+  // caller's stream, the direct kernel on the forked aux stream, whose CTAs take the SMs the
+  // stencil grid's last wave leaves idle; the caller's stream joins the aux work
+  const bool fork_direct = shape.has_direct && shape.has_stencil && aux && fork && join;
+  cudaStream_t direct_stream = stream;
+  if (fork_direct) {
+    cudaError_t e = cudaEventRecord(fork, stream);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(aux, fork, 0);
+    if (e != cudaSuccess) return cuda_error(e, "fork of the direct kernel");
+    direct_stream = aux;
   }
   if (shape.has_stencil) {
     LaunchParams ps = p;
@@ -411,13 +407,32 @@ int launch_materialize(const LaunchParams& p, const BatchShape& shape, size_t st
       else k_stencil2<-1, false><<<ps.n_items, 512, smem2, stream>>>(ps, scs, shape.st_max_wo);
       cudaError_t e = cudaGetLastError();
       if (e != cudaSuccess) return cuda_error(e, "k_stencil2 launch");
-      ++*n_launched;
-      return SAND_OK;
+    } else {
+      k_stencil<<<ps.n_items, 512, stencil_smem, stream>>>(ps);
+      cudaError_t e = cudaGetLastError();
+      if (e != cudaSuccess) return cuda_error(e, "k_stencil launch");
     }
-    k_stencil<<<ps.n_items, 512, stencil_smem, stream>>>(ps);
-    cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) return cuda_error(e, "k_stencil launch");
     ++*n_launched;
+  }
+  if (shape.has_direct) {
+    LaunchParams pd = p;
+    pd.n_items = shape.n_direct;
+    int rc;
+    // specialised instantiations: one dtype for every view and even output widths (the
+    // 4-byte pair stores are aligned); anything else takes the generic instantiation
+    switch (shape.even_wo ? shape.dtype : -1) {
+      case SAND_U8: rc = launch_resample_dt<SAND_U8, true>(pd, shape, direct_stream); break;
+      case SAND_BF16: rc = launch_resample_dt<SAND_BF16, true>(pd, shape, direct_stream); break;
+      case SAND_F32: rc = launch_resample_dt<SAND_F32, true>(pd, shape, direct_stream); break;
+      default: rc = launch_resample_dt<-1, false>(pd, shape, direct_stream); break;
+    }
+    if (rc != SAND_OK) return rc;
+    ++*n_launched;
+  }
+  if (fork_direct) {
+    cudaError_t e = cudaEventRecord(join, aux);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(stream, join, 0);
+    if (e != cudaSuccess) return cuda_error(e, "join of the direct kernel");
   }
   return SAND_OK;
 }

@@ -674,7 +674,15 @@ extern "C" int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank,
     lp.views[k] = v->vconst[k];
   }
   int launched = 0;
-  int rc = sand::launch_materialize(lp, plan->shapes[it], v->stencil_smem, stream, &launched);
+  const sand::BatchShape& bshape = plan->shapes[it];
+  if (bshape.has_direct && bshape.has_stencil && !v->aux_stream && getenv("SAND_NO_FORK") == nullptr) {
+    e = cudaStreamCreateWithFlags(&v->aux_stream, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&v->fork_ev, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&v->join_ev, cudaEventDisableTiming);
+    if (e != cudaSuccess) return sand::cuda_error(e, "aux stream for the direct kernel");
+  }
+  int rc = sand::launch_materialize(lp, bshape, v->stencil_smem, stream, v->aux_stream, v->fork_ev, v->join_ev,
+                                    &launched);
   if (rc != SAND_OK) return rc;
   e = cudaEventRecord(plan->last_use, stream);
   if (e == cudaSuccess) e = cudaEventRecord(v->inflight[slot], stream);
@@ -802,6 +810,9 @@ extern "C" int sand_view_destroy(sand_view* v) {
   for (auto& kv : v->plans) sand::release_plan_device(v, *kv.second);
   sand::free_pool(v);
   if (v->upload_stream) cudaStreamDestroy(v->upload_stream);
+  if (v->aux_stream) cudaStreamDestroy(v->aux_stream);
+  if (v->fork_ev) cudaEventDestroy(v->fork_ev);
+  if (v->join_ev) cudaEventDestroy(v->join_ev);
   if (v->d_sched) cudaFree(v->d_sched);
   for (auto& ev : v->inflight)
     if (ev) cudaEventDestroy(ev);
