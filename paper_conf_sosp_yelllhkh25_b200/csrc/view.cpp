@@ -233,6 +233,15 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
       auto first = plan->items.begin() + plan->item_begin.back();
       auto mid = std::stable_partition(first, plan->items.end(), [](const sand::WorkItem& w) { return !(w.flags & 1u); });
       shape.n_direct = static_cast<uint32_t>(mid - first);
+      // stencil items longest first (one CTA per item, dispatched in order): the grid's last
+      // wave then holds the cheapest items. Cost model in lane instructions per output value
+      // (ncu): resample ~15, rotation ~28, blur ~10 + 3 r.
+      auto cost = [&](const sand::WorkItem& w) {
+        const sand::GroupParams& g = plan->groups[w.gp];
+        return 15 + (g.rot_on ? 28 : 0) + (g.blur_on ? 10 + 3 * g.blur_r : 0);
+      };
+      std::stable_sort(mid, plan->items.end(),
+                       [&](const sand::WorkItem& a, const sand::WorkItem& b) { return cost(a) > cost(b); });
     }
     plan->item_begin.push_back(static_cast<uint32_t>(plan->items.size()));
     plan->shapes.push_back(shape);
