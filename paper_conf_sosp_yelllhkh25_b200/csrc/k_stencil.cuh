@@ -376,7 +376,7 @@ __device__ __forceinline__ void hblur_block(uint32_t rowa, uint32_t rowb, uint32
 // Separable Gaussian blur of one channel plane with radius R (R#16): horizontal pass into the
 // fp32 scratch in row strips, vertical pass, rint (Q4), normalise and store. Every output's taps
 // are accumulated from 0 in order i = 0..2R with fmaf in both passes (bit-identical to the
-// oracle). Fast path (Wo % kBX == 0, Wo % 4 == 0, Wo >= 2 kBX + R): word loads with
+// oracle). Fast path (R <= kBX, Wo % kBX == 0, Wo % 4 == 0, Wo >= 2 kBX + R + 3): word loads with
 // compile-time reflect maps for the border blocks; otherwise per-byte loads with reflect.
 template <int DT, bool VEC, int R>
 __device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupParams& g, const ChDests& cd,
@@ -395,7 +395,9 @@ __device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupPar
   float wt[2 * R + 1];
 #pragma unroll
   for (int i = 0; i <= 2 * R; ++i) wt[i] = __ldg(&g.blur_w[i]);
-  const bool fast = (Wo & 3) == 0 && Wo % kBX == 0 && Wo >= 2 * kBX + R + 3;
+  // the compile-time border maps cover the first and last block only, so every other block
+  // must be interior: R <= kBX (R > kBX, i.e. sigma > 2.1 with kBX = 8, takes the generic path)
+  const bool fast = R <= kBX && (Wo & 3) == 0 && Wo % kBX == 0 && Wo >= 2 * kBX + R + 3;
   const int xblocks = fast ? Wo / kBX : (Wo + kBX - 1) / kBX;
   constexpr int kOff = blur_koff<R>();
   for (int ys = 0; ys < Ho; ys += S) {
@@ -611,6 +613,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
     if (grp < groups && pr < pairs && !(sh.skip & 4)) {
       const int ox = 2 * pr;
       const bool has_b = ox + 1 < Wo;
+      const bool even_w = !(Wo & 1);
       const int ja = g.flip ? Wo - 1 - ox : ox;
       const int jb = has_b ? (g.flip ? Wo - 2 - ox : ox + 1) : ja;
       const uint2 ta = ctab[ja], tb = ctab[jb];
@@ -634,8 +637,13 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
             const uint64_t tq = rint_biased(f2::fma(ly, dv, top.h[c]));   // low bytes = q
             const uint32_t pair = __byte_perm(f2::lo(tq), f2::hi(tq), 0x0040);
             const uint32_t plane = q2 + (uint32_t)(c * sh.plane) + pix;
-            if (has_b) stsu16(plane, pair);
-            else stsu8(plane, pair);
+            if (VEC || (has_b && even_w)) {    // VEC: every width is even (host-checked)
+              if (VEC || has_b) stsu16(plane, pair);   // pix is even: 2-byte aligned
+              else stsu8(plane, pair);
+            } else {                           // odd plane width: pixel pairs can straddle
+              stsu8(plane, pair);
+              if (has_b) stsu8(plane + 1, pair >> 8);
+            }
           }
         };
         if (y0 & 1) {

@@ -314,3 +314,39 @@ def test_batch_put_rejects_unknown_frames():
         assert store.counters().frames_present == 2
     finally:
         store.close()
+
+
+# ------------------------------------------------------------------ ragged shapes / generic kernel paths
+
+@pytest.mark.parametrize("case", ["stencil_odd", "mixed_dtypes", "heavy_downscale", "blur_max_radius"])
+def test_ragged_shapes_whole_batch(case):
+    """Shapes off the bench's fast paths: odd output widths (no pair stores, per-byte blur
+    windows), mixed dtypes across views (the generic instantiation), heavy down-scaling of a
+    small source (the direct-gather kernel at odd sizes), and the largest blur radius (k = 23,
+    sigma = 2.9 -> r = 11) with rotation. Whole batches against the oracle."""
+    V = configs.ViewSpec
+    if case == "stencil_odd":
+        views = [V(clip_len=4, stride=3, out_h=29, out_w=37, rot_p=1.0, rot_max_deg=15.0, blur_p=0.5),
+                 V(clip_len=4, stride=3, out_h=29, out_w=37, spatial_group=1, blur_p=1.0, flip_p=1.0)]
+        src = (98, 70)
+    elif case == "mixed_dtypes":
+        views = [V(clip_len=6, stride=2, out_h=40, out_w=44, out_dtype=configs.U8, rot_p=0.5, rot_max_deg=10.0),
+                 V(clip_len=3, stride=4, out_h=40, out_w=44, spatial_group=1, out_dtype=configs.F32, blur_p=0.5)]
+        src = (120, 96)
+    elif case == "heavy_downscale":
+        views = [V(clip_len=5, stride=2, out_h=21, out_w=23, scale=(0.5, 1.0)),
+                 V(clip_len=5, stride=2, out_h=21, out_w=23, spatial_group=1, scale=(0.3, 1.0), out_dtype=configs.F32)]
+        src = (640, 360)
+    else:
+        views = [V(clip_len=4, stride=2, out_h=64, out_w=64, rot_p=1.0, rot_max_deg=10.0, blur_p=1.0,
+                   sigma=(2.9, 2.9))]
+        src = (160, 128)
+    w = configs.Workload(case, configs.Spec(batch_size=3, shared_window=(case == "heavy_downscale"), views=views),
+                         6, 24, src[0], src[1], case)
+    store, view, ospec, ods, vids = _setup(w)
+    try:
+        for epoch in (0, 5):
+            _check_meta(view, w.spec, ospec, ods, len(vids), epoch, 0, 0)
+            _check_outputs(view, w.spec, ospec, ods, vids, epoch, 0, 0)
+    finally:
+        _teardown(store, view)
