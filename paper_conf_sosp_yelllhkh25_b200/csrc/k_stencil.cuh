@@ -169,6 +169,10 @@ __device__ __forceinline__ uint64_t add_rm2(uint64_t a, uint64_t b) {
   return d;
 }
 
+#ifndef SAND_ROT_UNROLL
+#define SAND_ROT_UNROLL 2
+#endif
+constexpr int kRotUnroll = SAND_ROT_UNROLL;   // rotation pixel-loop unroll (ILP for the tap loads)
 #ifndef SAND_ROT_RPW
 #define SAND_ROT_RPW 2
 #endif
@@ -197,6 +201,7 @@ __device__ __forceinline__ void rotate_inplace(const GroupParams& g, uint32_t q2
       const uint64_t txy = f2::pack(__fmul_rn(nrs, yc), __fmul_rn(rc, yc));   // row terms
       const uint32_t orow = ring + ((uint32_t)oy & rmask) * (uint32_t)Wo;
       float xc = __fsub_rn((float)lane, cxo);
+      #pragma unroll (kRotUnroll)
       for (int ox = lane; ox < Wo; ox += 32, xc = __fadd_rn(xc, 32.f)) {
         // (sx, sy) = ((c*xc + (-s)*yc) + cx, (s*xc + c*yc) + cy), every op rounded (.rn ops
         // are not contracted)
@@ -276,6 +281,7 @@ __device__ __forceinline__ void rotate_direct(const GroupParams& g, uint32_t q2,
     const uint64_t txy = f2::pack(__fmul_rn(nrs, yc), __fmul_rn(rc, yc));
     const size_t orow = (size_t)oy * Wo;
     float xc = __fsub_rn((float)lane, cxo);
+    #pragma unroll (kRotUnroll)
     for (int ox = lane; ox < Wo; ox += 32, xc = __fadd_rn(xc, 32.f)) {
       const uint64_t s2 = f2::add(f2::add(f2::pack(__fmul_rn(rc, xc), __fmul_rn(rsn, xc)), txy), c2);
       const uint64_t t = add_rm2(s2, kr2);
