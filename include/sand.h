@@ -154,6 +154,10 @@ typedef struct {
   double blur_truncate;     /* radius = min((k-1)/2, floor(truncate*sigma+0.5)); 0 = cap  */
   double mean[3], std[3];   /* per-channel normalisation (R#17)                         */
   int32_t out_dtype;        /* SAND_U8 / SAND_BF16 / SAND_F32                           */
+  int32_t subsample_of;     /* -1: frames from the shared pool (R#4, R#5). k >= 0: this view's
+                               T frames are view k's frames at positions floor(t (T_k - 1) / (T - 1))
+                               (PySlowFast linspace slow pathway); view k
+                               must itself draw from the pool; stride/pool_offset are unused */
 } sand_view_desc;
 
 typedef struct {

@@ -38,7 +38,7 @@ class View(ctypes.Structure):
         ("blur_p", ctypes.c_double), ("sigma_min", ctypes.c_double), ("sigma_max", ctypes.c_double),
         ("blur_ksize", ctypes.c_uint32), ("blur_truncate", ctypes.c_double),
         ("mean", ctypes.c_double * 3), ("std", ctypes.c_double * 3),
-        ("out_dtype", ctypes.c_int32),
+        ("out_dtype", ctypes.c_int32), ("subsample_of", ctypes.c_int32),
     ]
 
 
@@ -96,6 +96,7 @@ def lib():
             "oracle_philox4x32_10": (None, [P(u32), P(u32), P(u32)]),
             "oracle_u01": (dbl, [u32]),
             "oracle_bounded": (u32, [u32, u32]),
+            "oracle_linspace_index": (u32, [u32, u32, u32]),
             "oracle_bern": (ctypes.c_int, [u32, dbl]),
             "oracle_permutation": (None, [u32, u64, u64, P(u32)]),
             "oracle_num_samples": (u32, [u32, u32, ctypes.c_int]),
@@ -290,6 +291,7 @@ class ViewDesc:
     mean: tuple = (0.485, 0.456, 0.406)
     std: tuple = (0.229, 0.224, 0.225)
     out_dtype: int = BF16
+    subsample_of: int = -1
 
 
 @dataclass
@@ -328,6 +330,7 @@ def make_spec(sd: SpecDesc) -> Spec:
             o.mean[c] = v.mean[c]
             o.std[c] = v.std[c]
         o.out_dtype = v.out_dtype
+        o.subsample_of = v.subsample_of
     return s
 
 

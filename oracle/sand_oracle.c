@@ -53,6 +53,7 @@ typedef struct {
   double blur_truncate;
   double mean[3], std[3];
   int32_t out_dtype;               /* OR_U8 / OR_BF16 / OR_F32 */
+  int32_t subsample_of;            /* -1: pool view; k: linspace sub-sample of view k (R#26) */
 } oracle_view;
 
 typedef struct {
@@ -172,15 +173,25 @@ static uint32_t gcd_u32(uint32_t a, uint32_t b) {
   return a;
 }
 
+/* Position i of linspace(0, n - 1, steps) truncated to an integer, exactly (R#26):
+   floor(i * (n - 1) / (steps - 1)). PySlowFast's torch.linspace(...).long() gives the same
+   positions except where float32 rounding lands just below an integer. */
+uint32_t oracle_linspace_index(uint32_t i, uint32_t steps, uint32_t n) {
+  if (steps <= 1) return 0;
+  return (uint32_t)(((uint64_t)i * (n - 1)) / (steps - 1));
+}
+
 void oracle_temporal(const oracle_spec* spec, uint64_t epoch, uint32_t clip, uint32_t n_frames_video,
                      oracle_clip_meta* meta) {
+  /* the pool is built from the views that draw from it (subsample_of < 0) */
   uint32_t g = 0;
-  for (uint32_t k = 0; k < spec->n_views; ++k) g = gcd_u32(g, spec->views[k].stride);
+  for (uint32_t k = 0; k < spec->n_views; ++k)
+    if (spec->views[k].subsample_of < 0) g = gcd_u32(g, spec->views[k].stride);
   uint32_t span[OR_MAX_VIEWS];
   uint32_t L = 0;
   for (uint32_t k = 0; k < spec->n_views; ++k) {
     span[k] = (spec->views[k].clip_len - 1) * (spec->views[k].stride / g) + 1;
-    if (span[k] > L) L = span[k];
+    if (spec->views[k].subsample_of < 0 && span[k] > L) L = span[k];
   }
   uint32_t P = (L - 1) * g + 1;                  /* frames covered by the pool */
   uint32_t F = n_frames_video;
@@ -193,6 +204,7 @@ void oracle_temporal(const oracle_spec* spec, uint64_t epoch, uint32_t clip, uin
   meta->pool_start = start;
   for (uint32_t k = 0; k < spec->n_views; ++k) {
     uint32_t o;
+    if (spec->views[k].subsample_of >= 0) continue;     /* filled below from its parent */
     if (spec->views[k].pool_offset >= 0) {
       o = (uint32_t)spec->views[k].pool_offset;
     } else {
@@ -203,6 +215,13 @@ void oracle_temporal(const oracle_spec* spec, uint64_t epoch, uint32_t clip, uin
       uint32_t idx = start + (o + t * (spec->views[k].stride / g)) * g;
       meta->frames[k][t] = idx < F - 1 ? idx : F - 1;   /* clamp to the last frame (R#4) */
     }
+  }
+  /* PySlowFast slow pathway (R#26): the parent's frames at linspace positions */
+  for (uint32_t k = 0; k < spec->n_views; ++k) {
+    int32_t p = spec->views[k].subsample_of;
+    if (p < 0) continue;
+    for (uint32_t t = 0; t < spec->views[k].clip_len; ++t)
+      meta->frames[k][t] = meta->frames[p][oracle_linspace_index(t, spec->views[k].clip_len, spec->views[p].clip_len)];
   }
 }
 

@@ -61,6 +61,7 @@ def make_spec(spec: Spec, videos) -> tuple[_abi.sand_view_spec, object]:
             o.mean[c] = v.mean[c]
             o.std[c] = v.std[c]
         o.out_dtype = v.out_dtype
+        o.subsample_of = int(getattr(v, "subsample_of", -1))
     return s, arr
 
 

@@ -37,6 +37,7 @@ class ViewSpec:
     mean: tuple = IMAGENET_MEAN
     std: tuple = IMAGENET_STD
     out_dtype: int = BF16
+    subsample_of: int = -1        # >= 0: linspace sub-sample of that view's frames (f4, R#26)
 
 
 @dataclass
@@ -87,6 +88,16 @@ def slowfast() -> Workload:
     slow = ViewSpec(clip_len=8, stride=8, **common)
     return Workload("slowfast", Spec(batch_size=16, views=[fast, slow]), 1024, 300, 340, 256,
                     "SlowFast-shaped: fast 32/2 + slow 8/8 of one clip, short side 256 -> crop 224, flip, B=16 bf16")
+
+
+def slowfast_linspace() -> Workload:
+    """SlowFast with PySlowFast's slow pathway: the 8 slow frames are the fast clip's frames at
+    torch.linspace(0, 31, 8).long() = {0, 4, 8, 13, 17, 22, 26, 31} (SURVEY §8(f) f4, R#26)."""
+    w = slowfast()
+    w.name = "slowfast_linspace"
+    w.spec.views[1].subsample_of = 0
+    w.description = "SlowFast-shaped with the PySlowFast linspace slow pathway"
+    return w
 
 
 def twoview() -> Workload:

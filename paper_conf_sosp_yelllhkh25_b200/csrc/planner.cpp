@@ -75,15 +75,20 @@ int validate_spec(const sand_view_spec& s, std::string* why) {
     for (uint32_t j = 0; j < k; ++j)
       if (s.views[j].spatial_group == v.spatial_group && !same_spatial(s.views[j], v))
         return bad("views of one spatial_group must share all spatial/augmentation fields");
+    if (v.subsample_of >= 0 &&
+        (static_cast<uint32_t>(v.subsample_of) >= s.n_views || v.subsample_of == static_cast<int32_t>(k) ||
+         s.views[v.subsample_of].subsample_of >= 0))
+      return bad("subsample_of must name another view that draws from the pool");
   }
   uint32_t g = 0;
-  for (uint32_t k = 0; k < s.n_views; ++k) g = std::gcd(g, s.views[k].stride);
+  for (uint32_t k = 0; k < s.n_views; ++k)
+    if (s.views[k].subsample_of < 0) g = std::gcd(g, s.views[k].stride);
   uint32_t L = 0;
   for (uint32_t k = 0; k < s.n_views; ++k)
-    L = std::max(L, (s.views[k].clip_len - 1) * (s.views[k].stride / g) + 1);
+    if (s.views[k].subsample_of < 0) L = std::max(L, (s.views[k].clip_len - 1) * (s.views[k].stride / g) + 1);
   for (uint32_t k = 0; k < s.n_views; ++k) {
     const sand_view_desc& v = s.views[k];
-    if (v.pool_offset >= 0 &&
+    if (v.subsample_of < 0 && v.pool_offset >= 0 &&
         static_cast<uint32_t>(v.pool_offset) + (v.clip_len - 1) * (v.stride / g) + 1 > L)
       return bad("pool_offset + span exceeds the shared pool");
   }
@@ -103,13 +108,14 @@ void derive_spec(SpecInfo* info) {
   }
   for (uint32_t q = 0; q < SAND_MAX_GROUPS; ++q)
     if (info->leader[q] >= 0) info->groups.push_back(q);
-  uint32_t g = 0;
-  for (uint32_t k = 0; k < s.n_views; ++k) g = std::gcd(g, s.views[k].stride);
+  uint32_t g = 0;   // the pool is built from the views that draw from it
+  for (uint32_t k = 0; k < s.n_views; ++k)
+    if (s.views[k].subsample_of < 0) g = std::gcd(g, s.views[k].stride);
   info->g = g;
   info->pool_len = 0;
   for (uint32_t k = 0; k < s.n_views; ++k) {
     info->span[k] = (s.views[k].clip_len - 1) * (s.views[k].stride / g) + 1;
-    info->pool_len = std::max(info->pool_len, info->span[k]);
+    if (s.views[k].subsample_of < 0) info->pool_len = std::max(info->pool_len, info->span[k]);
   }
 }
 
@@ -198,12 +204,24 @@ void plan_clip(const SpecInfo& info, uint64_t epoch, uint32_t clip, sand_clip_me
   m->pool_start = start;
   for (uint32_t k = 0; k < s.n_views; ++k) {
     const sand_view_desc& v = s.views[k];
+    if (v.subsample_of >= 0) continue;   // filled from its parent below
     const uint32_t off = v.pool_offset >= 0
                              ? static_cast<uint32_t>(v.pool_offset)
                              : draw_below(d.get(Purpose::kTemporal, 0, 1 + k, 0, clip)[0], L - info.span[k] + 1);
     const uint32_t step = v.stride / g;
     for (uint32_t t = 0; t < v.clip_len; ++t)
       m->frames[k][t] = std::min(start + (off + t * step) * g, F - 1);
+  }
+  // PySlowFast slow pathway (f4, R#26): the parent's frames at the exact linspace positions
+  // floor(t * (T_p - 1) / (T - 1))
+  for (uint32_t k = 0; k < s.n_views; ++k) {
+    const sand_view_desc& v = s.views[k];
+    if (v.subsample_of < 0) continue;
+    const uint32_t tp = s.views[v.subsample_of].clip_len;
+    for (uint32_t t = 0; t < v.clip_len; ++t) {
+      const uint32_t pos = v.clip_len > 1 ? static_cast<uint32_t>(static_cast<uint64_t>(t) * (tp - 1) / (v.clip_len - 1)) : 0u;
+      m->frames[k][t] = m->frames[v.subsample_of][pos];
+    }
   }
 
   // a3: crop boxes

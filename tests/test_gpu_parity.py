@@ -87,9 +87,10 @@ def test_tiny_all_epochs_exact(dtype, family):
 
 # ------------------------------------------------------------------ reduced stores: whole batches
 
-@pytest.mark.parametrize("name,n_videos,clips", [("k400", 40, None), ("slowfast", 20, None), ("ray", 20, 3)])
+@pytest.mark.parametrize("name,n_videos,clips", [("k400", 40, None), ("slowfast", 20, None), ("ray", 20, 3),
+                                                  ("slowfast_linspace", 20, None)])
 def test_reduced_store_whole_batch(name, n_videos, clips):
-    w = configs.get(name)
+    w = configs.slowfast_linspace() if name == "slowfast_linspace" else configs.get(name)
     store, view, ospec, ods, vids = _setup(w, n_videos)
     try:
         n_it = view.iterations(0, 0)

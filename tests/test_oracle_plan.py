@@ -375,3 +375,41 @@ def test_k_epoch_pool_frame_reuse_over_ten_epochs():
     c1, c10 = counts(1), counts(10)
     assert np.all(c10 == 10)
     assert np.mean(c1 >= 4) < 0.15
+
+
+# ------------------------------------------------------------------ §8(f) f4: PySlowFast linspace slow pathway
+
+def test_linspace_index_is_linspace_truncated():
+    """R#26 pin: the oracle's index law is torch.linspace(0, n - 1, T) truncated, for every
+    T, n <= 64: against float64 linspace wherever it is not within 1e-9 of an integer (there it
+    must be that integer), and equal to PySlowFast's float32 torch.linspace(...).long() for the
+    SlowFast 32 -> 8 selection."""
+    L = oracle.lib()
+    for n in range(1, 65):
+        for T in range(1, 65):
+            ref = torch.linspace(0, n - 1, T, dtype=torch.float64).tolist()
+            for i in range(T):
+                got = L.oracle_linspace_index(i, T, n)
+                r = ref[i]
+                assert got == (round(r) if abs(r - round(r)) < 1e-9 else math.floor(r)), (n, T, i)
+    assert [L.oracle_linspace_index(i, 8, 32) for i in range(8)] == torch.linspace(0, 31, 8).long().tolist()
+
+
+def test_slowfast_linspace_slow_is_fast_at_linspace_positions():
+    from paper_conf_sosp_yelllhkh25_b200 import configs
+    w = configs.slowfast_linspace()
+    import sys
+    import os
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+    from helpers import to_oracle
+    ospec = to_oracle(w.spec)
+    vids = [(1000 + i, 300, 340, 256) for i in range(8)]
+    ods = oracle.make_dataset(vids)
+    pos = torch.linspace(0, 31, 8).long().tolist()
+    assert pos == [0, 4, 8, 13, 17, 22, 26, 31]
+    for e in (0, 3):
+        for clip in range(8):
+            m = oracle.ClipMeta()
+            oracle.lib().oracle_plan_clip(ctypes.byref(ospec), ods, e, clip, ctypes.byref(m))
+            fast = list(m.frames[0][:32])
+            assert list(m.frames[1][:8]) == [fast[p] for p in pos]

@@ -89,3 +89,21 @@ def test_host_plan_k_epoch_pool_matches_oracle(name, k):
             ref = oracle.ClipMeta()
             oracle.lib().oracle_plan_clip(oracle.ctypes.byref(ospec), ods, epoch, clip, oracle.ctypes.byref(ref))
             assert meta_fields(w.spec, got) == meta_fields(w.spec, ref), (name, k, epoch, clip)
+
+
+def test_host_plan_linspace_slow_pathway_matches_oracle():
+    """§8(f) f4 (R#26): the linspace slow pathway plans bit-exactly like the oracle."""
+    w = configs.slowfast_linspace()
+    vids = videos_of(w, 16)
+    ospec = to_oracle(w.spec)
+    ods = oracle.make_dataset(vids)
+    for epoch in (0, 2, 9):
+        for clip in range(16):
+            got = sand.plan_clip(w.spec, vids, epoch, clip)
+            ref = oracle.ClipMeta()
+            oracle.lib().oracle_plan_clip(oracle.ctypes.byref(ospec), ods, epoch, clip, oracle.ctypes.byref(ref))
+            assert meta_fields(w.spec, got) == meta_fields(w.spec, ref), (epoch, clip)
+    bad = configs.slowfast_linspace().spec
+    bad.views[0].subsample_of = 1            # a sub-sample of a sub-sample
+    with pytest.raises(sand.SandError):
+        sand.plan_clip(bad, vids, 0, 0)
