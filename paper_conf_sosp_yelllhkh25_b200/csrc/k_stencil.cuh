@@ -279,10 +279,14 @@ __device__ __forceinline__ void rotate_direct(const GroupParams& g, uint32_t q2,
   for (int oy = warp; oy < Ho; oy += nwarps) {
     const float yc = __fsub_rn((float)oy, cyo);
     const uint64_t txy = f2::pack(__fmul_rn(nrs, yc), __fmul_rn(rc, yc));
-    const size_t orow = (size_t)oy * Wo;
+    uint8_t* op[3];                      // this lane's output pixel of the row, per channel
+#pragma unroll
+    for (int c = 0; c < 3; ++c) op[c] = obase[c] + ((size_t)oy * Wo + lane) * dt_bytes<DT>();
     float xc = __fsub_rn((float)lane, cxo);
     #pragma unroll (kRotUnroll)
-    for (int ox = lane; ox < Wo; ox += 32, xc = __fadd_rn(xc, 32.f)) {
+    for (int ox = lane; ox < Wo;
+         ox += 32, xc = __fadd_rn(xc, 32.f), op[0] += 32 * dt_bytes<DT>(), op[1] += 32 * dt_bytes<DT>(),
+         op[2] += 32 * dt_bytes<DT>()) {
       const uint64_t s2 = f2::add(f2::add(f2::pack(__fmul_rn(rc, xc), __fmul_rn(rsn, xc)), txy), c2);
       const uint64_t t = add_rm2(s2, kr2);
       const uint64_t l = f2::fma(f2::add(t, nkr2), m1, s2);
@@ -296,7 +300,7 @@ __device__ __forceinline__ void rotate_direct(const GroupParams& g, uint32_t q2,
         const uint64_t h = f2::fma(lx, f2::fma(T0, m1, T1), f2::add(T0, nb2));
         const float h0 = f2::lof(h), h1 = f2::hif(h);
         const float tq = __fadd_rn(__fmaf_rn(ly, __fsub_rn(h1, h0), h0), kRound);   // 1.5*2^23 + q
-        uint8_t* o = obase[c] + (orow + (size_t)ox) * dt_bytes<DT>();
+        uint8_t* o = op[c];
         if constexpr (DT == SAND_U8) {
           *o = (uint8_t)(__float_as_uint(tq) & 0xffu);
         } else {
