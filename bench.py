@@ -104,7 +104,7 @@ def measured_peaks():
 
 # the kernel that dominates each config's step (the roofline's subject; `achieved` divides the
 # step's algorithmic bytes by the summed duration of every kernel read_batch launched)
-DOMINANT_KERNEL = {"tiny": "k_stream", "k400": "k_stream", "slowfast": "k_stream",
+DOMINANT_KERNEL = {"tiny": "k_stream", "k400": "k_stream", "slowfast": "k_copy",
                    "twoview": "k_stencil2 (with k_stream for the plain items)", "ray": "k_direct"}
 
 

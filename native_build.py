@@ -58,7 +58,7 @@ def build_oracle(force=False):
 PRODUCT_CPP = ["sand_api.cpp", "store.cpp", "planner.cpp", "view.cpp"]
 PRODUCT_CU = ["materialize.cu", "store_kernels.cu"]
 PRODUCT_HDR = ["internal.h", "plan_types.h", "planner.h", "k_resample.cuh", "k_stream.cuh", "k_stencil.cuh",
-               "k_direct.cuh"]
+               "k_direct.cuh", "k_copy.cuh"]
 
 
 def build_product(force=False, variant=None, defines=()):

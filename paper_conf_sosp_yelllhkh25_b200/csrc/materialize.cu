@@ -175,6 +175,7 @@ __global__ void __launch_bounds__(512) k_stencil(const LaunchParams p) {
 #include "k_stream.cuh"
 #include "k_stencil.cuh"
 #include "k_direct.cuh"
+#include "k_copy.cuh"
 
 namespace sand {
 
@@ -269,6 +270,22 @@ unsigned persistent_grid(K kernel, int threads, size_t smem, uint64_t tasks) {
 
 template <int DT, bool VEC>
 int launch_resample_dt(const LaunchParams& p, const BatchShape& sh, cudaStream_t stream) {
+  // identity-scale batches (every direct item samples the source 1:1): the lerps are dead
+  // (lambda = 0), so the copy-convert kernel renders the same bits without them
+  static const int copy_env = env_int("SAND_COPY", 1);
+  if constexpr (VEC && DT >= 0) {
+    if (copy_env && sh.direct_identity && sh.src_w_mod4 && sh.wo_mod4 && sh.max_wo <= 1024) {
+      const int quads = sh.max_wo / 4;
+      const int rpi = std::max(1, 256 / quads);
+      const int threads = ((rpi * quads + 31) / 32) * 32;
+      static const int RB = std::max(1, env_int("SAND_COPY_RB", 32));
+      const int nbands = (sh.max_ho + RB - 1) / RB;
+      k_copy<DT><<<(unsigned)((uint64_t)p.n_items * nbands), threads, 0, stream>>>(p, RB, nbands);
+      cudaError_t e = cudaGetLastError();
+      if (e != cudaSuccess) return cuda_error(e, "k_copy launch");
+      return SAND_OK;
+    }
+  }
   const ResampleCfg cfg = choose_resample(sh);
   if (cfg.smem > 227 * 1024) return set_error(SAND_EINVAL, "resample tile exceeds shared memory (source crop too large)");
   const int pairs = (sh.max_wo + 1) / 2;

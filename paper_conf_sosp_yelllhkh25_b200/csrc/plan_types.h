@@ -73,6 +73,8 @@ struct BatchShape {
   int32_t st_max_wo, st_max_ho, st_cols_bound;
   float st_max_scy;
   uint32_t n_direct;      // items [0, n_direct) of the batch are direct, the rest stencil items
+  int32_t direct_identity;  // every direct item has sc_x == sc_y == 1 (k_copy applies)
+  int32_t src_w_mod4;       // every source width is a multiple of 4
 };
 
 struct LaunchParams {

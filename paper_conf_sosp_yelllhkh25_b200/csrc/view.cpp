@@ -131,6 +131,8 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
   }
   for (uint64_t it = 0; it < plan->iterations; ++it) {
     BatchShape shape{};
+    shape.direct_identity = 1;
+    shape.src_w_mod4 = 1;
     shape.dtype = common_dtype;
     shape.even_wo = even_wo;
     shape.wo_mod4 = wo_mod4;
@@ -167,6 +169,8 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
           shape.st_max_scy = std::max(shape.st_max_scy, g.sc_y);
         } else {
           shape.has_direct = 1;
+          if (!(g.sc_x == 1.0f && g.sc_y == 1.0f)) shape.direct_identity = 0;
+          if (dim.width % 4u) shape.src_w_mod4 = 0;
           shape.max_wo = std::max(shape.max_wo, g.out_w);
           shape.max_ho = std::max(shape.max_ho, g.out_h);
           shape.cols_bound = std::max(shape.cols_bound, cols);

@@ -10,9 +10,9 @@ for c in slowfast twoview ray tiny; do
 done
 timeout 900 python bench.py --impl reference --steps 200 --warmup 3 > gpurun_out/bench_reference.json 2> gpurun_out/bench_reference.err; cat gpurun_out/bench_reference.json
 for c in ${NCU_CONFIGS:-k400 slowfast twoview ray}; do
-  timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"k_(stream|stencil|resample|direct)" -c 40 --csv --log-file gpurun_out/launches_$c.csv \
+  timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"k_(stream|stencil|resample|direct|copy)" -c 40 --csv --log-file gpurun_out/launches_$c.csv \
     python bench.py --config $c --steps 30 --warmup 3 --no-e2e --no-cpu > /dev/null 2> gpurun_out/ncu_launch_$c.err
-  timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_(stream|stencil|resample|direct)" -s 6 -c 2 -o gpurun_out/prof_$c -f \
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_(stream|stencil|resample|direct|copy)" -s 6 -c 2 -o gpurun_out/prof_$c -f \
     python bench.py --config $c --steps 12 --warmup 3 --no-e2e --no-cpu > /dev/null 2> gpurun_out/ncu_full_$c.err
   ncu -i gpurun_out/prof_$c.ncu-rep --page raw --csv > gpurun_out/ncu_raw_$c.csv 2>/dev/null
   ncu -i gpurun_out/prof_$c.ncu-rep --page details --csv > gpurun_out/ncu_details_$c.csv 2>/dev/null

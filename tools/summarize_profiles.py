@@ -55,7 +55,7 @@ def main():
     traffic = {}
     md = [f"# ncu summary, round {rnd}", "",
           "Captured with `scripts/gpu_round.sh` on one B200 (`ncu --set full --clock-control none`, "
-          "kernels matching `k_(stream|stencil|resample|direct)`, 2 launches after 6 skipped). Per-launch, "
+          "kernels matching `k_(stream|stencil|resample|direct|copy)`, 2 launches after 6 skipped). Per-launch, "
           "cold-cache, serialised: compare shares, not absolutes. Bench numbers come from "
           "`bench.py` (CUDA events, no profiler).", ""]
     for path in sorted(glob.glob(os.path.join(OUT, "ncu_raw_*.csv"))):
