@@ -55,6 +55,9 @@ __global__ void __launch_bounds__(256) k_copy(const LaunchParams p, int RB, int 
   const int odd = sx & 1;                                 // uniform per item (ox is a multiple of 4)
   const int nd = (int)w.n_dest;
   const uint32_t* dests = p.dests + w.dest_begin;
+  // the first two destinations in registers, advanced per row (a third and later: rare)
+  Dest dl0 = make_dest(p, dests[0], y_begin + r0, ox), dl1 = dl0;
+  if (nd > 1) dl1 = make_dest(p, dests[1], y_begin + r0, ox);
 #pragma unroll (kCopyUnroll)
   for (int oy = y_begin + r0; oy < y_end; oy += rpi) {
     const int sy = sy0 + oy;
@@ -86,13 +89,22 @@ __global__ void __launch_bounds__(256) k_copy(const LaunchParams p, int RB, int 
       cp::px(ys >> 24, k[2], c[3]);
     }
     // output column ox + j holds source pixel j (or 3 - j under flip)
-    const bool fl = g.flip != 0;
-    for (int d = 0; d < nd; ++d) {
-      const Dest e = make_dest(p, dests[d], oy, ox);
+    if (g.flip) {                                         // output column ox + j <- source pixel 3 - j
 #pragma unroll
       for (int ch = 0; ch < 3; ++ch) {
-        const uint32_t t0 = fl ? c[3][ch] : c[0][ch], t1 = fl ? c[2][ch] : c[1][ch];
-        const uint32_t t2 = fl ? c[1][ch] : c[2][ch], t3 = fl ? c[0][ch] : c[3][ch];
+        uint32_t t = c[0][ch];
+        c[0][ch] = c[3][ch];
+        c[3][ch] = t;
+        t = c[1][ch];
+        c[1][ch] = c[2][ch];
+        c[2][ch] = t;
+      }
+    }
+    for (int d = 0; d < nd; ++d) {
+      const Dest e = d == 0 ? dl0 : (d == 1 ? dl1 : make_dest(p, dests[d], oy, ox));
+#pragma unroll
+      for (int ch = 0; ch < 3; ++ch) {
+        const uint32_t t0 = c[0][ch], t1 = c[1][ch], t2 = c[2][ch], t3 = c[3][ch];
         uint8_t* o = e.row + (size_t)ch * e.cstride;
         if constexpr (DT == SAND_U8) {
           *reinterpret_cast<uint32_t*>(o) =
@@ -113,6 +125,8 @@ __global__ void __launch_bounds__(256) k_copy(const LaunchParams p, int RB, int 
         }
       }
     }
+    dl0.row += (size_t)dl0.rstride * rpi;
+    dl1.row += (size_t)dl1.rstride * rpi;
   }
 }
 
