@@ -334,7 +334,7 @@ __device__ __forceinline__ void rotate_direct(const GroupParams& g, uint32_t q2,
 #define SAND_BLUR_BX 8
 #endif
 #ifndef SAND_BLUR_BV
-#define SAND_BLUR_BV 8
+#define SAND_BLUR_BV 16
 #endif
 constexpr int kBX = SAND_BLUR_BX;   // blur: columns per thread in the horizontal pass (multiple of 4)
 constexpr int kBV = SAND_BLUR_BV;   // blur: rows per thread in the vertical pass
