@@ -1,17 +1,18 @@
 // k_stencil.cuh — fused kernel for items with rotation and/or blur (two-view config;
 // SURVEY §8(a) a4-a10).
 //
-// One CTA (512 threads, ~200 KB shared memory) per work item:
-//  Phase 1  Q2 = resample(+flip) of the clip frame for all three channels into three uint8
-//           planes in shared memory, produced band by band with the staged machinery of
-//           k_resample/k_stream: cp.async of the band's NV12 footprint, conversion to an RGBx
-//           tap grid, row walkers (4 groups of column-pair threads) writing uint8 (a4-a7, Q2).
-//  Phase 2  per channel: rotation Q2 -> Q3 (bilinear inverse map, zero outside, rint; a8, Q3)
-//           then the separable blur in row strips: horizontal pass into an fp32 strip
-//           (register-blocked along x, FFMA2 over pairs of strip rows), vertical pass
-//           (FFMA2 over column pairs read as 64-bit words), rint (Q4), normalise and store to
-//           every destination (a9, a10). The free Q2 plane of the channel, or the band/Q3
-//           region, holds the fp32 strip.
+// One CTA (512 threads, 227 KB shared memory: three uint8 Q2 planes + an 80 KB band/ring/
+// scratch region) per stencil work item:
+//  Phase 1  Q2 = resample(+flip) of the clip frame for all three channels into the planes,
+//           band by band: cp.async of the band's NV12 rows (the next band's rows load while
+//           this band is walked), conversion to an RGBx tap grid, column-pair walkers
+//           writing uint8 (a4-a7, Q2).
+//  Phase 2  rotation without blur: Q3 straight to the output (rotate_direct: rint, normalise,
+//           store; a8, a10). Rotation then blur: Q3 in place through a power-of-two ring of
+//           rows (rotate_inplace). Blur (a9), channel by channel, last to first so finished
+//           planes extend the fp32 strip scratch: horizontal pass in kBX-column register
+//           blocks over row pairs (compile-time reflect maps for the border blocks), vertical
+//           pass in kBV-row blocks over column pairs, rint (Q4), normalise, pair stores.
 // Every fp32 operation follows R#12/R#15/R#16/R#17 with IEEE rounding in the oracle's order
 // (blur taps accumulated from 0 in tap order), so outputs are bit-identical to the oracle.
 #pragma once
