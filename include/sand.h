@@ -77,8 +77,11 @@ int sand_store_add_video(sand_store* s, uint32_t video, uint32_t n_frames, uint3
  * frames are y_frame_stride / uv_frame_stride bytes apart; rows are y_pitch /
  * uv_pitch apart. src_on_device != 0: y/uv are device pointers, else host (pinned
  * host memory makes the copy asynchronous). Putting a frame again overwrites it
- * and resets its counters. Errors: ERANGE (unknown video / frame range), EINVAL,
- * ECUDA. */
+ * and resets its counters. Ordering: every put records a store event on `stream`
+ * (after waiting on the previous put's event, so puts on different streams are
+ * chained), and a later sand_view_read_batch on ANY stream waits on it before its
+ * kernels, so a read never consumes a frame whose copy has not landed. Errors: ERANGE
+ * (unknown video / frame range), EINVAL, ECUDA. */
 int sand_store_put_frames(sand_store* s, uint32_t video, uint32_t first_frame, uint32_t n_frames,
                           const uint8_t* y, uint64_t y_pitch, uint64_t y_frame_stride,
                           const uint8_t* uv, uint64_t uv_pitch, uint64_t uv_frame_stride,
@@ -95,8 +98,8 @@ int sand_store_put_frames(sand_store* s, uint32_t video, uint32_t first_frame, u
  * Stream-ordered on `stream`; the caller keeps src valid until the stream reaches the
  * copy. The call waits (host side) until the previous batch put's scatter has run, so
  * the staging buffer is never overwritten while still being read. Putting a frame again
- * overwrites it and resets its counters. Nothing is copied if any (video, frame) is
- * unknown. Errors: ERANGE (unknown video / frame), EINVAL (null pointers, frames of
+ * overwrites it and resets its counters. Ordered before later reads exactly as
+ * sand_store_put_frames. Nothing is copied if any (video, frame) is unknown. Errors: ERANGE (unknown video / frame), EINVAL (null pointers, frames of
  * different sizes, pitch/uv_offset/frame_stride too small), ECUDA. */
 int sand_store_put_frame_batch(sand_store* s, uint32_t n, const uint32_t* videos, const uint32_t* frames,
                                const uint8_t* src, uint64_t frame_stride, uint64_t pitch, uint64_t uv_offset,
@@ -115,7 +118,9 @@ int sand_store_frame_layout(const sand_store* s, uint32_t video, uint32_t frame,
                             sand_frame_layout* out);
 
 /* Mark frames as present without copying (after a producer wrote them in place via
- * sand_store_frame_layout). Errors: ERANGE. */
+ * sand_store_frame_layout). The store cannot see those writes: the caller orders them
+ * before later sand_view_read_batch calls (same stream, or an event the read stream
+ * waits on). Errors: ERANGE. */
 int sand_store_mark_present(sand_store* s, uint32_t video, uint32_t first_frame, uint32_t n_frames);
 
 /* Reuse accounting (Fig. 16 / Fig. 19): totals over the store. A

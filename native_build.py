@@ -26,6 +26,25 @@ def _run(cmd):
     subprocess.run(cmd, check=True, cwd=ROOT)
 
 
+def _run_parallel(cmds):
+    """Compile the kernel units concurrently (each nvcc is single-threaded)."""
+    from concurrent.futures import ThreadPoolExecutor
+    for c in cmds:
+        print(" ".join(c), flush=True)
+
+    def one(c):
+        r = subprocess.run(c, cwd=ROOT, capture_output=True, text=True)
+        return c, r
+
+    with ThreadPoolExecutor(max_workers=max(1, min(len(cmds), os.cpu_count() or 1))) as ex:
+        results = list(ex.map(one, cmds))
+    for c, r in results:
+        sys.stdout.write(r.stdout)
+        sys.stderr.write(r.stderr)
+        if r.returncode != 0:
+            raise subprocess.CalledProcessError(r.returncode, c)
+
+
 def _stale(target, sources):
     if not os.path.exists(target):
         return True
@@ -56,9 +75,10 @@ def build_oracle(force=False):
 
 
 PRODUCT_CPP = ["sand_api.cpp", "store.cpp", "planner.cpp", "view.cpp"]
-PRODUCT_CU = ["materialize.cu", "store_kernels.cu"]
-PRODUCT_HDR = ["internal.h", "plan_types.h", "planner.h", "k_resample.cuh", "k_stream.cuh", "k_stencil.cuh",
-               "k_direct.cuh", "k_copy.cuh"]
+PRODUCT_CU = ["materialize.cu", "store_kernels.cu", "mat_plain.cu", "mat_stream.cu", "mat_direct.cu",
+              "mat_stencil.cu"]
+PRODUCT_HDR = ["internal.h", "plan_types.h", "planner.h", "kernels.h", "kernels_common.cuh", "k_resample.cuh",
+               "k_stream.cuh", "k_plain.cuh", "k_stencil.cuh", "k_direct.cuh", "k_copy.cuh"]
 
 
 def build_product(force=False, variant=None, defines=()):
@@ -71,11 +91,14 @@ def build_product(force=False, variant=None, defines=()):
         inc = ["-I", os.path.join(ROOT, "include"), "-I", CSRC]
         for s in PRODUCT_CPP:
             objs.append(os.path.join(PKG, "build", s + ".o"))
+        jobs = []
         for s in PRODUCT_CU:
             obj = os.path.join(bdir, s + ".o")
             objs.append(obj)
-            _run([NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xptxas", "-v",
-                  "--expt-relaxed-constexpr", *["-D" + d for d in defines], *inc, "-c", os.path.join(CSRC, s), "-o", obj])
+            jobs.append([NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xptxas", "-v",
+                         "--expt-relaxed-constexpr", *["-D" + d for d in defines], *inc, "-c", os.path.join(CSRC, s),
+                         "-o", obj])
+        _run_parallel(jobs)
         _run([NVCC, *ARCH, "-shared", "-Xcompiler", "-fPIC", *objs, "-o", os.path.join(PKG, f"libsand_{variant}.so"),
               "-lcudart", "-lpthread"])
         return
@@ -91,13 +114,15 @@ def build_product(force=False, variant=None, defines=()):
             # host planner: IEEE double, no contraction (R#20 bit-exactness discipline)
             _run(["g++", "-O2", "-std=c++17", "-fPIC", "-ffp-contract=off", "-fno-fast-math", "-Wall",
                   "-I", os.path.join(CUDA_HOME, "include"), *inc, "-c", src, "-o", obj])
+    jobs = []
     for s in PRODUCT_CU:
         src = os.path.join(CSRC, s)
         obj = os.path.join(PKG, "build", s + ".o")
         objs.append(obj)
         if force or _stale(obj, [src] + hdrs):
-            _run([NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
-                  "-Xptxas", "-v", "--expt-relaxed-constexpr", *inc, "-c", src, "-o", obj])
+            jobs.append([NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
+                         "-Xptxas", "-v", "--expt-relaxed-constexpr", *inc, "-c", src, "-o", obj])
+    _run_parallel(jobs)
     so = os.path.join(PKG, "libsand.so")
     if force or _stale(so, objs):
         _run([NVCC, *ARCH, "-shared", "-Xcompiler", "-fPIC", *objs, "-o", so, "-lcudart", "-lpthread"])

@@ -100,6 +100,16 @@ def slowfast_linspace() -> Workload:
     return w
 
 
+def slowfast_hd() -> Workload:
+    """SlowFast on 1280x720 sources: short side 256 gives W' = floor(1280 * 256 / 720) = 455, a
+    real down-scaling by 2.81 on both axes (SURVEY §8(c) reading 10's variant)."""
+    w = slowfast()
+    w.name = "slowfast_hd"
+    w.n_videos, w.n_frames, w.width, w.height = 256, 300, 1280, 720
+    w.description = "SlowFast-shaped on 1280x720 NV12: short side 256 (W' = 455) -> crop 224, fast 32/2 + slow 8/8"
+    return w
+
+
 def twoview() -> Workload:
     views = [ViewSpec(clip_len=16, stride=4, spatial_group=q, rot_p=0.5, rot_max_deg=10.0, blur_p=0.5)
              for q in range(2)]
@@ -115,7 +125,8 @@ def ray() -> Workload:
                     "shared window, flip, B=16 per rank bf16")
 
 
-WORKLOADS = {"tiny": tiny, "k400": k400, "slowfast": slowfast, "twoview": twoview, "ray": ray}
+WORKLOADS = {"tiny": tiny, "k400": k400, "slowfast": slowfast, "twoview": twoview, "ray": ray,
+             "slowfast_hd": slowfast_hd, "slowfast_linspace": slowfast_linspace}
 
 
 def get(name: str) -> Workload:

@@ -65,6 +65,11 @@ struct sand_store {
   sand::PutDesc* put_desc_host = nullptr;   // pinned
   uint32_t put_desc_cap = 0;
   cudaEvent_t put_done = nullptr;
+  // ordering of puts before reads: every put records `last_put` on its stream (after waiting on
+  // the previous put's event, so puts on different streams are chained); read_batch makes its
+  // stream wait on it whenever a put happened since that stream last waited
+  cudaEvent_t last_put = nullptr;
+  uint64_t put_seq = 0;
 };
 
 namespace sand {
@@ -78,6 +83,7 @@ struct EpochPlan {
   std::vector<GroupParams> groups;            // iterations * B * n_groups
   std::vector<WorkItem> items;
   std::vector<uint32_t> dests;
+  std::vector<uint2> tasks;                   // k_plain tasks (BatchShape::task_first / n_tasks)
   std::vector<uint32_t> item_begin;           // iterations + 1
   std::vector<BatchShape> shapes;             // per iteration: launch shape
   // reuse accounting per iteration: unique (video, frame) keys and their use counts
@@ -92,11 +98,13 @@ struct EpochPlan {
   GroupParams* d_groups = nullptr;
   WorkItem* d_items = nullptr;
   uint32_t* d_dests = nullptr;
+  uint2* d_tasks = nullptr;
   bool uploaded = false;
   cudaEvent_t last_use = nullptr;              // recorded after every kernel that reads the buffer
   cudaEvent_t ready = nullptr;                 // upload complete (recorded on the view's upload stream)
   cudaStream_t ready_waited = nullptr;         // last caller stream made to wait on `ready`
   uint64_t last_touch = 0;
+  int pins = 0;                                // read_batch calls using the device copy (never evicted while > 0)
 };
 
 }  // namespace sand
@@ -137,14 +145,15 @@ struct sand_view {
   uint64_t plan_build_ns = 0, plan_wait_ns = 0, read_ns = 0;
   uint64_t plan_cpu_ns = 0, plan_buffer_wait_ns = 0, lock_wait_ns = 0, pending_waits = 0;
   size_t stencil_smem = 0;   // dynamic smem of the stencil path (0 if no view rotates/blurs)
-  uint32_t* d_sched = nullptr;   // kSchedSlots pairs of ticket counters (persistent kernels)
-  uint32_t sched_seq = 0;        // next slot pair
+  int pl_fpc = 1, pl_nq = 1;     // k_plain: frames per CTA, threads per frame (from the widest view)
   size_t n_buffers = 0;          // plan buffers allocated so far
   std::vector<cudaEvent_t> inflight;   // ring of per-batch completion events (read-ahead bound)
   // batches with both direct and stencil items: the direct kernel runs on aux_stream (forked
   // from / joined to the caller's stream) so it fills the SMs the stencil kernel's tail leaves idle
   cudaStream_t aux_stream = nullptr;
   cudaEvent_t fork_ev = nullptr, join_ev = nullptr;
+  uint64_t put_seq_seen = 0;              // store->put_seq the last read_batch stream waited for
+  cudaStream_t put_stream_seen = nullptr;
 };
 
 namespace sand {
@@ -158,7 +167,7 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
 size_t stencil_smem_bytes(int max_h, int max_w, int max_r);
 int configure_kernels(size_t stencil_smem);
 // aux/fork/join may be null (then the kernels run back to back on `stream`)
-int launch_materialize(const LaunchParams& p, const BatchShape& shape, size_t stencil_smem, cudaStream_t stream,
-                       cudaStream_t aux, cudaEvent_t fork, cudaEvent_t join, int* n_launched);
+int launch_materialize(const LaunchParams& p, const BatchShape& shape, size_t stencil_smem, int pl_fpc, int pl_nq,
+                       cudaStream_t stream, cudaStream_t aux, cudaEvent_t fork, cudaEvent_t join, int* n_launched);
 
 }  // namespace sand

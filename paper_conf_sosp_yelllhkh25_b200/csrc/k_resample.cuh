@@ -1,65 +1,19 @@
-// k_resample.cuh — fused resample kernel for items without rotation/blur
-// (DESIGN.md §7).
-//
-// One CTA = one work item (clip slot, source frame, group) x one band of R output rows.
-//  1. Separable tap tables: output column j -> (x0, x1, lambda_x); band row -> (y0, y1,
-//     lambda_y) with the exact fp32 rule of R#12.
-//  2. Source -> shared memory, two modes chosen per batch by the host:
-//     RAW    (scale <= ~2, Kinetics/SlowFast): the band's NV12 footprint (Y rows + UV rows,
-//            16 B aligned column span) is copied with cp.async (LDGSTS, all requests in
-//            flight at once), then converted in shared memory to packed RGBx, two pixels
-//            per thread sharing one chroma sample (a4, a5, Q1).
-//     GATHER (heavy down-scaling, 1080p Ray trials): only the tapped source columns and
-//            rows are touched: bitmaps + popcount prefix give a compact tap grid, whose
-//            pixels are gathered from HBM with 4 independent loads in flight per thread
-//            and converted (a4, a5).
-//  3. Two row-walker groups; each thread owns two adjacent output columns, walks down its
-//     half of the band and keeps the horizontal lerps of the two current source rows in
-//     registers, so each (source row, column) lerp is computed once (a6). Flip is the
-//     column mirror (a7). Vertical lerp, rint, normalise and packing run as FFMA2/FADD2
-//     pairs (sm_100a packed fp32), then one 4-byte store per (row, channel, destination)
-//     through per-destination pointers computed once (a10); every destination view of the
-//     group is written from the same registers (a11, node merging P:L277).
-// Every fp32 operation is the R#12/R#17 op sequence with IEEE rounding, so results are
-// bit-identical to the oracle (byte->float via the 2^23 exponent trick and rint via
-// +1.5*2^23 are exact for values in [0, 256)).
+// k_resample.cuh — shared device helpers of the resample kernels (k_plain, k_stream, k_direct,
+// k_copy, k_stencil2): the R#12 tap rule, packed fp32
+// pair arithmetic (sm_100a FFMA2/FADD2), horizontal lerps of RGBx words, destinations and the
+// vertical lerp / rint / normalise / store sequence (R#12, R#17). Every fp32 operation is the
+// oracle's op sequence with IEEE rounding (byte->float via the 2^23 exponent trick and rint via
+// +1.5*2^23 are exact for values in [0, 256)), so results are bit-identical to the oracle.
 #pragma once
 
 namespace sand {
 namespace rs {
 
-constexpr int kColWords = 128;             // GATHER: source column span <= 4096
-constexpr int kRowWords = 32;              // GATHER: band source row span <= 1024
 constexpr int kInlineDests = 2;            // destinations kept in registers
 constexpr float kBias = 8388608.0f;        // 2^23
 constexpr float kRound = 12582912.0f;      // 1.5 * 2^23
 
 __host__ __device__ inline size_t a16(size_t x) { return (x + 15) & ~size_t(15); }
-
-// --- shared layout: [tables][mode data] -----------------------------------------------
-struct Tables {
-  uint2* ctab;        // per output column j: (x0 | x1 << 16 grid-relative, bits of lambda_x)
-  uint2* rtab;        // per band row: (y0 | y1 << 16 grid-relative, bits of lambda_y)
-  int* misc;          // GATHER: [0] tapped columns, [1] tapped rows
-};
-
-__host__ __device__ inline size_t tables_bytes(int maxWo, int R) {
-  return a16((size_t)maxWo * 8) + a16((size_t)R * 8) + 16;
-}
-
-__device__ inline Tables carve_tables(uint8_t*& p, int maxWo, int R) {
-  Tables t;
-  t.ctab = reinterpret_cast<uint2*>(p); p += a16((size_t)maxWo * 8);
-  t.rtab = reinterpret_cast<uint2*>(p); p += a16((size_t)R * 8);
-  t.misc = reinterpret_cast<int*>(p); p += 16;
-  return t;
-}
-
-// GATHER-mode bookkeeping
-__host__ __device__ inline size_t gather_meta_bytes(int maxWo, int R) {
-  return a16(kColWords * 4) + a16(kRowWords * 4) + a16(kColWords * 2) + a16(kRowWords * 2) +
-         a16((size_t)2 * maxWo * 2) + a16((size_t)2 * R * 2);
-}
 
 // source tap of output index o (R#12): s = max(sc*((float)(off+o)+0.5f)-0.5f, 0)
 __device__ __forceinline__ void tap(float sc, int off, int o, int lim, int org, int& i0, int& i1, float& lam) {
@@ -254,325 +208,6 @@ __device__ __forceinline__ void emit(const Row3& top, const Row3& bot, float l, 
   }
 }
 
-// Walk band rows [rr_lo, rr_hi) for the output column pair (ox, ox+1). ND: destinations in
-// registers (1, or 2 plus a loop over the rest). Horizontal lerps of source rows live in two
-// register slots indexed by row parity: y1 = y0 + 1 (or y0 at the clamp), so the two rows an
-// output row needs are always in different slots and each source row's lerp is computed
-// once, with no register copies between rows (the branches on parity are warp-uniform).
-template <int DT, int ND, bool VEC>
-__device__ __forceinline__ void walk_rows(const LaunchParams& p, const uint32_t* __restrict__ dests, int nd,
-                                          const uint2* __restrict__ rtab, const uint32_t* __restrict__ grid,
-                                          int gw, int oy0, int rr_lo, int rr_hi, int ox, uint32_t ca, uint32_t cb,
-                                          uint64_t lx, bool vec, bool has_b) {
-  Dest dl[ND];
-  int dt[ND];
-#pragma unroll
-  for (int d = 0; d < ND; ++d) {
-    dl[d] = make_dest(p, dests[d], oy0 + rr_lo, ox);
-    dt[d] = DT >= 0 ? DT : p.views[dests[d] >> 24].dtype;
-  }
-  int have0 = -1, have1 = -1;      // source row held in slot 0 (even rows) / slot 1 (odd rows)
-  Row3 S0, S1;
-  for (int rr = rr_lo; rr < rr_hi; ++rr) {
-    const uint2 rt = rtab[rr];
-    const int r0 = (int)(rt.x & 0xffffu), r1 = (int)(rt.x >> 16);
-    const float l = __uint_as_float(rt.y);
-    if (r0 & 1) {
-      if (have1 != r0) { hrow(S1, grid + (size_t)r0 * gw, ca, cb, lx); have1 = r0; }
-      if (r1 != r0) {
-        if (have0 != r1) { hrow(S0, grid + (size_t)r1 * gw, ca, cb, lx); have0 = r1; }
-        emit<DT, ND, VEC>(S1, S0, l, dl, dt, p, dests, nd, oy0 + rr, ox, vec, has_b);
-      } else {
-        emit<DT, ND, VEC>(S1, S1, l, dl, dt, p, dests, nd, oy0 + rr, ox, vec, has_b);
-      }
-    } else {
-      if (have0 != r0) { hrow(S0, grid + (size_t)r0 * gw, ca, cb, lx); have0 = r0; }
-      if (r1 != r0) {
-        if (have1 != r1) { hrow(S1, grid + (size_t)r1 * gw, ca, cb, lx); have1 = r1; }
-        emit<DT, ND, VEC>(S0, S1, l, dl, dt, p, dests, nd, oy0 + rr, ox, vec, has_b);
-      } else {
-        emit<DT, ND, VEC>(S0, S0, l, dl, dt, p, dests, nd, oy0 + rr, ox, vec, has_b);
-      }
-    }
-  }
-}
-
-// The row walk (step 3), shared by both modes. grid: RGBx rows of gw words.
-template <int DT, bool VEC>
-__device__ __forceinline__ void walk(const LaunchParams& p, const WorkItem& w, const GroupParams& g,
-                                     const Tables& t, const uint32_t* __restrict__ grid, int gw, int oy_lo,
-                                     int nrows) {
-  const int Wo = g.out_w;
-  const int pairs = (Wo + 1) >> 1;
-  const int P = blockDim.x >> 1;                       // threads per walker
-  const int walker = threadIdx.x >= P ? 1 : 0;
-  const int half = (nrows + 1) >> 1;
-  const int rr_lo = walker * half, rr_hi = min(nrows, rr_lo + half);
-  const int nd = (int)w.n_dest;
-  const uint32_t* dests = p.dests + w.dest_begin;
-  const uint2* rtab = reinterpret_cast<const uint2*>(t.rtab);
-  for (int pair = threadIdx.x - walker * P; pair < pairs; pair += P) {
-    const int ox = 2 * pair;
-    const bool has_b = ox + 1 < Wo;
-    const bool vec = has_b && !(Wo & 1);
-    const int ja = g.flip ? Wo - 1 - ox : ox;
-    const int jb = has_b ? (g.flip ? Wo - 2 - ox : ox + 1) : ja;
-    const uint2 ta = t.ctab[ja], tb = t.ctab[jb];
-    const uint64_t lx = f2::pack(ta.y, tb.y);
-    if (nd == 1)
-      walk_rows<DT, 1, VEC>(p, dests, nd, rtab, grid, gw, oy_lo, rr_lo, rr_hi, ox, ta.x, tb.x, lx, vec, has_b);
-    else
-      walk_rows<DT, kInlineDests, VEC>(p, dests, nd, rtab, grid, gw, oy_lo, rr_lo, rr_hi, ox, ta.x, tb.x, lx, vec,
-                                  has_b);
-  }
-}
-
 }  // namespace rs
-
-// RAW mode: p launch params; R band rows; nbands; maxWo table sizing.
-template <int DT, bool VEC>
-__global__ void __launch_bounds__(224, 3) k_resample_raw(const LaunchParams p, int R, int nbands, int maxWo) {
-  extern __shared__ __align__(16) uint8_t smem_raw[];
-  using namespace rs;
-  const int item_idx = blockIdx.x / nbands;
-  const int band = blockIdx.x - item_idx * nbands;
-  const WorkItem w = p.items[item_idx];
-  if (w.flags & 1u) return;
-  const GroupParams& g = p.groups[w.gp];
-  const int Wo = g.out_w, Ho = g.out_h;
-  const int oy_lo = band * R;
-  if (oy_lo >= Ho) return;
-  const int nrows = min(R, Ho - oy_lo);
-  uint8_t* sp = smem_raw;
-  const Tables t = carve_tables(sp, maxWo, R);
-  const int tid = threadIdx.x, nthr = blockDim.x;
-
-  // footprint: monotone taps -> first/last output column and row bound it
-  const int x_lo = tap0(g.sc_x, g.off_x, 0, g.org_x);
-  int x_hi, y_lo, y_hi, dmy;
-  float fl;
-  tap(g.sc_x, g.off_x, Wo - 1, g.lim_x, g.org_x, dmy, x_hi, fl);
-  y_lo = tap0(g.sc_y, g.off_y, oy_lo, g.org_y);
-  tap(g.sc_y, g.off_y, oy_lo + nrows - 1, g.lim_y, g.org_y, dmy, y_hi, fl);
-  const int x16 = x_lo & ~15;
-  const int gw = ((x_hi + 16) & ~15) - x16;        // grid / raw row width (bytes of Y, words of RGBx)
-  const int ny = y_hi - y_lo + 1;
-  const int uv_lo = y_lo >> 1;
-  const int nuv = (y_hi >> 1) - uv_lo + 1;
-  uint8_t* rawY = sp;
-  uint8_t* rawUV = rawY + (size_t)ny * gw;
-  uint32_t* grid = reinterpret_cast<uint32_t*>(rawUV + a16((size_t)nuv * gw));
-
-  // 1. async copy of the NV12 footprint (16 B requests)
-  const uint8_t* Yp = p.slab + w.y_off;
-  const uint8_t* UVp = Yp + (size_t)w.pitch * w.src_h;
-  const int chunks = gw >> 4;
-  {
-    // thread -> (row slot, chunk): rows advance by nthr / chunks per pass, no division in the loop
-    const int rows_per_pass = max(1, nthr / chunks);
-    const int k = tid % chunks, r0 = tid / chunks;
-    if (r0 < rows_per_pass)
-      for (int r = r0; r < ny + nuv; r += rows_per_pass) {
-        if (r < ny)
-          cp_async16(rawY + (size_t)r * gw + k * 16, Yp + (size_t)(y_lo + r) * w.pitch + x16 + k * 16);
-        else
-          cp_async16(rawUV + (size_t)(r - ny) * gw + k * 16, UVp + (size_t)(uv_lo + r - ny) * w.pitch + x16 + k * 16);
-      }
-    for (int kk = k + nthr; kk < chunks; kk += nthr)     // only if a row has more chunks than threads
-      for (int r = 0; r < ny + nuv; ++r) {
-        if (r < ny)
-          cp_async16(rawY + (size_t)r * gw + kk * 16, Yp + (size_t)(y_lo + r) * w.pitch + x16 + kk * 16);
-        else
-          cp_async16(rawUV + (size_t)(r - ny) * gw + kk * 16, UVp + (size_t)(uv_lo + r - ny) * w.pitch + x16 + kk * 16);
-      }
-  }
-  // 2. tap tables, grid-relative (overlaps the copy)
-  for (int j = tid; j < Wo; j += nthr) {
-    int x0, x1;
-    float lx;
-    tap(g.sc_x, g.off_x, j, g.lim_x, g.org_x, x0, x1, lx);
-    t.ctab[j] = make_uint2((uint32_t)(x0 - x16) | ((uint32_t)(x1 - x16) << 16), __float_as_uint(lx));
-  }
-  for (int r = tid; r < nrows; r += nthr) {
-    int y0, y1;
-    float ly;
-    tap(g.sc_y, g.off_y, oy_lo + r, g.lim_y, g.org_y, y0, y1, ly);
-    t.rtab[r] = make_uint2((uint32_t)(y0 - y_lo) | ((uint32_t)(y1 - y_lo) << 16), __float_as_uint(ly));
-  }
-  cp_async_wait_all();
-  __syncthreads();
-
-  // 3. NV12 -> RGBx in shared memory: a thread takes one chroma sample and the (up to) 2x2
-  //    luma pixels that share it; warps walk chroma rows, lanes walk chroma columns
-  const int hp = gw >> 1;
-  const int nwarps = nthr >> 5, lane = tid & 31;
-  for (int u = tid >> 5; u < nuv; u += nwarps) {
-    const int ytop = 2 * (uv_lo + u) - y_lo;      // grid rows ytop, ytop+1 (may fall outside)
-    const bool top = ytop >= 0, bot = ytop + 1 < ny;
-    const uint8_t* uvrow = rawUV + (size_t)u * gw;
-    for (int k = lane; k < hp; k += 32) {
-      const Chroma ch = chroma(*reinterpret_cast<const uint16_t*>(uvrow + 2 * k));
-      if (top) {
-        const uint32_t yp = *reinterpret_cast<const uint16_t*>(rawY + (size_t)ytop * gw + 2 * k);
-        *reinterpret_cast<uint2*>(grid + (size_t)ytop * gw + 2 * k) =
-            make_uint2(rgbx((int)(yp & 0xffu), ch), rgbx((int)(yp >> 8), ch));
-      }
-      if (bot) {
-        const uint32_t yp = *reinterpret_cast<const uint16_t*>(rawY + (size_t)(ytop + 1) * gw + 2 * k);
-        *reinterpret_cast<uint2*>(grid + (size_t)(ytop + 1) * gw + 2 * k) =
-            make_uint2(rgbx((int)(yp & 0xffu), ch), rgbx((int)(yp >> 8), ch));
-      }
-    }
-  }
-  __syncthreads();
-
-  // 4. row walk
-  walk<DT, VEC>(p, w, g, t, grid, gw, oy_lo, nrows);
-}
-
-// GATHER mode (heavy down-scaling): compact tap grid gathered from HBM.
-template <int DT, bool VEC>
-__global__ void __launch_bounds__(224, 3) k_resample_gather(const LaunchParams p, int R, int nbands, int maxWo) {
-  extern __shared__ __align__(16) uint8_t smem_raw[];
-  using namespace rs;
-  const int item_idx = blockIdx.x / nbands;
-  const int band = blockIdx.x - item_idx * nbands;
-  const WorkItem w = p.items[item_idx];
-  if (w.flags & 1u) return;
-  const GroupParams& g = p.groups[w.gp];
-  const int Wo = g.out_w, Ho = g.out_h;
-  const int oy_lo = band * R;
-  if (oy_lo >= Ho) return;
-  const int nrows = min(R, Ho - oy_lo);
-  uint8_t* sp = smem_raw;
-  const Tables t = carve_tables(sp, maxWo, R);
-  uint32_t* colbits = reinterpret_cast<uint32_t*>(sp); sp += a16(kColWords * 4);
-  uint32_t* rowbits = reinterpret_cast<uint32_t*>(sp); sp += a16(kRowWords * 4);
-  uint16_t* colpref = reinterpret_cast<uint16_t*>(sp); sp += a16(kColWords * 2);
-  uint16_t* rowpref = reinterpret_cast<uint16_t*>(sp); sp += a16(kRowWords * 2);
-  uint16_t* xs = reinterpret_cast<uint16_t*>(sp); sp += a16((size_t)2 * maxWo * 2);
-  uint16_t* ys = reinterpret_cast<uint16_t*>(sp); sp += a16((size_t)2 * R * 2);
-  uint32_t* grid = reinterpret_cast<uint32_t*>(sp);
-  const int tid = threadIdx.x, nthr = blockDim.x;
-  const int warp = tid >> 5, lane = tid & 31;
-
-  for (int i = tid; i < kColWords + kRowWords; i += nthr) {
-    if (i < kColWords) colbits[i] = 0u;
-    else rowbits[i - kColWords] = 0u;
-  }
-  const int cbase = tap0(g.sc_x, g.off_x, 0, g.org_x);
-  const int rbase = tap0(g.sc_y, g.off_y, oy_lo, g.org_y);
-  __syncthreads();
-  for (int j = tid; j < Wo; j += nthr) {
-    int x0, x1;
-    float lx;
-    tap(g.sc_x, g.off_x, j, g.lim_x, g.org_x, x0, x1, lx);
-    const int r0 = x0 - cbase, r1 = x1 - cbase;
-    t.ctab[j] = make_uint2((uint32_t)r0 | ((uint32_t)r1 << 16), __float_as_uint(lx));
-    atomicOr(&colbits[r0 >> 5], 1u << (r0 & 31));
-    atomicOr(&colbits[r1 >> 5], 1u << (r1 & 31));
-  }
-  for (int r = tid; r < nrows; r += nthr) {
-    int y0, y1;
-    float ly;
-    tap(g.sc_y, g.off_y, oy_lo + r, g.lim_y, g.org_y, y0, y1, ly);
-    const int r0 = y0 - rbase, r1 = y1 - rbase;
-    t.rtab[r] = make_uint2((uint32_t)r0 | ((uint32_t)r1 << 16), __float_as_uint(ly));
-    atomicOr(&rowbits[r0 >> 5], 1u << (r0 & 31));
-    atomicOr(&rowbits[r1 >> 5], 1u << (r1 & 31));
-  }
-  __syncthreads();
-  if (warp == 0) {   // exclusive popcount prefix of the column bitmap
-    uint32_t c[kColWords / 32];
-    uint32_t sum = 0;
-#pragma unroll
-    for (int k = 0; k < kColWords / 32; ++k) {
-      c[k] = __popc(colbits[lane * (kColWords / 32) + k]);
-      sum += c[k];
-    }
-    uint32_t incl = sum;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const uint32_t o = __shfl_up_sync(0xffffffffu, incl, d);
-      if (lane >= d) incl += o;
-    }
-    uint32_t run = incl - sum;
-#pragma unroll
-    for (int k = 0; k < kColWords / 32; ++k) {
-      colpref[lane * (kColWords / 32) + k] = (uint16_t)run;
-      run += c[k];
-    }
-    if (lane == 31) t.misc[0] = (int)incl;
-  }
-  if (warp == (nthr > 32 ? 1 : 0)) {   // ... and of the row bitmap
-    const uint32_t c = __popc(rowbits[lane]);
-    uint32_t incl = c;
-#pragma unroll
-    for (int d = 1; d < 32; d <<= 1) {
-      const uint32_t o = __shfl_up_sync(0xffffffffu, incl, d);
-      if (lane >= d) incl += o;
-    }
-    rowpref[lane] = (uint16_t)(incl - c);
-    if (lane == 31) t.misc[1] = (int)incl;
-  }
-  __syncthreads();
-  for (int wd = tid; wd < kColWords + kRowWords; wd += nthr) {
-    const bool col = wd < kColWords;
-    const int k0 = col ? wd : wd - kColWords;
-    uint32_t b = col ? colbits[k0] : rowbits[k0];
-    int k = col ? colpref[k0] : rowpref[k0];
-    const int base = (col ? cbase : rbase) + k0 * 32;
-    uint16_t* dst = col ? xs : ys;
-    while (b) {
-      const int bit = __ffs(b) - 1;
-      b &= b - 1;
-      dst[k++] = (uint16_t)(base + bit);
-    }
-  }
-  auto cidx = [&](const uint32_t* bits, const uint16_t* pref, int r) -> uint32_t {
-    return pref[r >> 5] + __popc(bits[r >> 5] & ((1u << (r & 31)) - 1u));
-  };
-  for (int j = tid; j < Wo; j += nthr) {
-    const uint32_t v = t.ctab[j].x;
-    t.ctab[j].x = cidx(colbits, colpref, (int)(v & 0xffffu)) | (cidx(colbits, colpref, (int)(v >> 16)) << 16);
-  }
-  for (int r = tid; r < nrows; r += nthr) {
-    const uint32_t v = t.rtab[r].x;
-    t.rtab[r].x = cidx(rowbits, rowpref, (int)(v & 0xffffu)) | (cidx(rowbits, rowpref, (int)(v >> 16)) << 16);
-  }
-  __syncthreads();
-
-  // gather-convert with 4 independent loads in flight per thread
-  const int nX = t.misc[0], nY = t.misc[1];
-  const uint8_t* Yp = p.slab + w.y_off;
-  const uint8_t* UVp = Yp + (size_t)w.pitch * w.src_h;
-  const int nwarps = nthr >> 5;
-  for (int i = warp; i < nY; i += nwarps) {
-    const int y = ys[i];
-    const uint8_t* yrow = Yp + (size_t)y * w.pitch;
-    const uint8_t* uvrow = UVp + (size_t)(y >> 1) * w.pitch;
-    uint32_t* grow = grid + (size_t)i * nX;
-    for (int j0 = lane; j0 < nX; j0 += 128) {
-      int yv[4];
-      uint32_t uvv[4];
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const int jj = j0 + 32 * u;
-        if (jj < nX) {
-          const int x = xs[jj];
-          yv[u] = __ldg(yrow + x);
-          uvv[u] = __ldg(reinterpret_cast<const uint16_t*>(uvrow + (x & ~1)));
-        }
-      }
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const int jj = j0 + 32 * u;
-        if (jj < nX) grow[jj] = rgbx(yv[u], chroma(uvv[u]));
-      }
-    }
-  }
-  __syncthreads();
-  walk<DT, VEC>(p, w, g, t, grid, nX, oy_lo, nrows);
-}
 
 }  // namespace sand

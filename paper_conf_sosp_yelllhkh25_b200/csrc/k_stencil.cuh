@@ -28,7 +28,6 @@ struct Shape {
   int grid_rows;    // grid / raw capacity in rows per band
   size_t plane;     // bytes of one uint8 plane (Ho*Wo, 16-aligned)
   size_t ubytes;    // bytes of the shared band/Q3 region
-  int skip;         // profiling only (SAND_STENCIL_SKIP): bit0 rotation, bit1 blur, bit2 Q2 walk
 };
 
 __host__ __device__ inline size_t band_bytes(int maxWo, int R, int grid_rows, int gw) {
@@ -621,7 +620,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
       band(oy_lo + sh.R, nr1, ylo1, yhi1);
       st::stage_rows_cp(s_rawb, Yp + x16, UVp + x16, w.pitch, gw, ylo1, yhi1, warp, nwarps, lane);
     }
-    if (grp < groups && pr < pairs && !(sh.skip & 4)) {
+    if (grp < groups && pr < pairs) {
       const int ox = 2 * pr;
       const bool has_b = ox + 1 < Wo;
       const bool even_w = !(Wo & 1);
@@ -683,7 +682,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
   const int r = g.blur_on ? g.blur_r : 0;
   const float cxo = (float)(Wo - 1) * 0.5f, cyo = (float)(Ho - 1) * 0.5f;
   if constexpr (DT >= 0) {
-    if (g.rot_on && !g.blur_on && nd == 1 && !(sh.skip & 1)) {   // a8 + a10 straight to the output
+    if (g.rot_on && !g.blur_on && nd == 1) {   // a8 + a10 straight to the output
       uint8_t* ob[3];
       float na[3], nb[3];
 #pragma unroll
@@ -699,7 +698,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
   }
   // a8 in place for all three channels when its ring fits the band/Q3 region; else per channel
   bool rotated = false;
-  if (g.rot_on && !(sh.skip & 1)) {
+  if (g.rot_on) {
     const float bound = fabsf(g.rot_s) * cxo + (1.f - g.rot_c) * cyo;
     const int D = (int)ceilf(bound) + 2;
     int ring_rows = 1;
@@ -721,7 +720,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
     uint32_t src = q2 + (uint32_t)(c * sh.plane);
     uint32_t scratch = q2 + (uint32_t)((c + 1) * sh.plane);
     size_t scratch_bytes = (size_t)(2 - c) * sh.plane + sh.ubytes;
-    if (g.rot_on && !rotated && !(sh.skip & 1)) {              // a8: Q3 = rotate(Q2) (R#15), one channel
+    if (g.rot_on && !rotated) {              // a8: Q3 = rotate(Q2) (R#15), one channel
       const uint32_t q3 = ureg;
       const float rc = g.rot_c, rsn = g.rot_s, nrs = -g.rot_s;
       for (int oy = warp; oy < Ho; oy += nwarps) {
@@ -764,7 +763,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
       scratch = q2 + (uint32_t)(c * sh.plane);   // this channel's Q2 plane (and the done ones) are free now
       scratch_bytes = (size_t)(3 - c) * sh.plane;
     }
-    if (g.blur_on && !(sh.skip & 2)) {         // a9: separable Gaussian in strips (R#16)
+    if (g.blur_on) {         // a9: separable Gaussian in strips (R#16)
       switch (r) {
         case 0: blur_plane<DT, VEC, 0>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;
         case 1: blur_plane<DT, VEC, 1>(p, g, cd, src, scratch, scratch_bytes, Wo, Ho, tid, nthr); break;

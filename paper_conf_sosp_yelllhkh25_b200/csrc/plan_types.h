@@ -7,6 +7,7 @@
 // the same (b, f) are adjacent so the groups of one frame share its lines in L2.
 #pragma once
 #include <stdint.h>
+#include <vector_types.h>   // uint2 (LaunchParams::tasks)
 
 #if defined(__CUDACC__)
 #define SAND_HD __host__ __device__
@@ -73,9 +74,36 @@ struct BatchShape {
   int32_t st_max_wo, st_max_ho, st_cols_bound;
   float st_max_scy;
   uint32_t n_direct;      // items [0, n_direct) of the batch are direct, the rest stencil items
-  int32_t direct_identity;  // every direct item has sc_x == sc_y == 1 (k_copy applies)
+  int32_t direct_identity;  // every mild direct item has sc_x == sc_y == 1 (k_copy applies)
   int32_t src_w_mod4;       // every source width is a multiple of 4
+  // item classes (per item, not per batch): direct items [0, n_mild) have a source step <= 2
+  // on both axes (k_plain / k_copy), [n_mild, n_direct) heavier down-scaling (k_direct)
+  uint32_t n_mild;
+  int32_t max_dests;        // largest destination count of a direct item
+  int32_t heavy_max_wo, heavy_max_ho;
+  // k_plain: the batch's task slice and exact shared-memory bounds over its tasks
+  uint32_t task_first, n_tasks;
+  int32_t pl_gw, pl_ring, pl_raw, pl_rb;
 };
+
+// k_plain task granularity (view.cpp builds the tasks, k_plain.cuh consumes them)
+constexpr int kPlainS = 4;         // output rows per sub-band
+constexpr int kPlainRB = 32;       // output rows per band
+constexpr int kPlainRBTail = 8;    // band of the tasks that make up the last part of the work
+constexpr double kPlainTailFrac = 0.25;
+
+// k_plain task word: frames | band rows << 8 | first output row << 20
+SAND_HD inline uint32_t pl_task_y(uint32_t nfr, uint32_t nr, uint32_t y0) { return nfr | (nr << 8) | (y0 << 20); }
+
+// exact fp32 tap of output index o (R#12), the same op sequence as the kernels' tap()
+SAND_HD inline void tap_ref(float sc, int off, int o, int lim, int org, int* i0, int* i1, float* lam) {
+  float s = sc * ((float)(off + o) + 0.5f) - 0.5f;
+  s = s > 0.f ? s : 0.f;
+  const int i = (int)s;
+  *lam = s - (float)i;
+  *i0 = org + i;
+  *i1 = org + (i + 1 < lim - 1 ? i + 1 : lim - 1);
+}
 
 struct LaunchParams {
   const uint8_t* slab;
@@ -87,10 +115,7 @@ struct LaunchParams {
   ViewConst views[kMaxViews];
   uint32_t n_views;
   uint32_t batch;          // B
-  uint32_t* sched;         // ticket counters of persistent kernels: [2 * slot] next task, [2 * slot + 1] CTAs done
-  uint32_t sched_slot;     // slot of this launch (counters are zero between launches)
+  const uint2* tasks;      // k_plain tasks of this batch (view.cpp)
 };
-
-constexpr int kSchedSlots = 64;
 
 }  // namespace sand

@@ -70,6 +70,26 @@ extern "C" int sand_store_add_video(sand_store* s, uint32_t video, uint32_t n_fr
   return SAND_OK;
 }
 
+namespace {
+// order a put on `st` after the previous put (any stream); call before enqueuing its copies
+int put_begin(sand_store* s, cudaStream_t st) {
+  if (!s->last_put) {
+    cudaError_t e = cudaEventCreateWithFlags(&s->last_put, cudaEventDisableTiming);
+    if (e != cudaSuccess) return sand::cuda_error(e, "cudaEventCreate(last_put)");
+  } else if (s->put_seq > 0) {
+    cudaError_t e = cudaStreamWaitEvent(st, s->last_put, 0);
+    if (e != cudaSuccess) return sand::cuda_error(e, "cudaStreamWaitEvent(last_put)");
+  }
+  return SAND_OK;
+}
+int put_end(sand_store* s, cudaStream_t st) {
+  cudaError_t e = cudaEventRecord(s->last_put, st);
+  if (e != cudaSuccess) return sand::cuda_error(e, "cudaEventRecord(last_put)");
+  s->put_seq++;
+  return SAND_OK;
+}
+}  // namespace
+
 extern "C" int sand_store_put_frames(sand_store* s, uint32_t video, uint32_t first_frame, uint32_t n_frames,
                                      const uint8_t* y, uint64_t y_pitch, uint64_t y_frame_stride,
                                      const uint8_t* uv, uint64_t uv_pitch, uint64_t uv_frame_stride,
@@ -86,6 +106,8 @@ extern "C" int sand_store_put_frames(sand_store* s, uint32_t video, uint32_t fir
   if (e != cudaSuccess) return sand::cuda_error(e, "cudaSetDevice");
   const cudaMemcpyKind kind = src_on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
   auto st = static_cast<cudaStream_t>(stream);
+  int rc = put_begin(s, st);
+  if (rc != SAND_OK) return rc;
   for (uint32_t f = 0; f < n_frames; ++f) {
     uint8_t* dst = s->slab + v.offset + v.frame_stride * (first_frame + f);
     e = cudaMemcpy2DAsync(dst, v.pitch, y + y_frame_stride * f, y_pitch, v.width, v.height, kind, st);
@@ -97,7 +119,7 @@ extern "C" int sand_store_put_frames(sand_store* s, uint32_t video, uint32_t fir
     v.fetches[first_frame + f] = 0;
     v.uses[first_frame + f] = 0;
   }
-  return SAND_OK;
+  return put_end(s, st);
 }
 
 extern "C" int sand_store_put_frame_batch(sand_store* s, uint32_t n, const uint32_t* videos, const uint32_t* frames,
@@ -132,6 +154,10 @@ extern "C" int sand_store_put_frame_batch(sand_store* s, uint32_t n, const uint3
   // the staging buffers of the previous call are reusable once its scatter has run
   e = cudaEventSynchronize(s->put_done);
   if (e != cudaSuccess) return sand::cuda_error(e, "cudaEventSynchronize(put_done)");
+  {
+    const int prc = put_begin(s, st);
+    if (prc != SAND_OK) return prc;
+  }
   if (s->put_desc_cap < n) {
     cudaFree(s->put_desc);
     cudaFreeHost(s->put_desc_host);
@@ -181,7 +207,7 @@ extern "C" int sand_store_put_frame_batch(sand_store* s, uint32_t n, const uint3
   if (rc != SAND_OK) return rc;
   e = cudaEventRecord(s->put_done, st);
   if (e != cudaSuccess) return sand::cuda_error(e, "cudaEventRecord(put_done)");
-  return SAND_OK;
+  return put_end(s, st);
 }
 
 extern "C" int sand_store_frame_layout(const sand_store* s, uint32_t video, uint32_t frame,
@@ -260,6 +286,7 @@ extern "C" int sand_store_destroy(sand_store* s) {
   cudaFree(s->put_desc);
   cudaFreeHost(s->put_desc_host);
   if (s->put_done) cudaEventDestroy(s->put_done);
+  if (s->last_put) cudaEventDestroy(s->last_put);
   delete s;
   return SAND_OK;
 }

@@ -34,11 +34,6 @@ uint64_t now_ns() {
       std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now().time_since_epoch()).count());
 }
 
-int env_int(const char* name, int dflt, int lo, int hi) {
-  const char* e = std::getenv(name);
-  const int x = e ? std::atoi(e) : dflt;
-  return std::min(hi, std::max(lo, x));
-}
 
 GroupParams group_params(const sand_view_desc& d, const sand_clip_meta& m, uint32_t q, uint32_t W, uint32_t H) {
   GroupParams g{};
@@ -84,6 +79,115 @@ GroupParams group_params(const sand_view_desc& d, const sand_clip_meta& m, uint3
   return g;
 }
 
+// staged column span of a group (16-aligned pixels the kernels copy per source row): from the
+// first column's i0 to the last column's i1 (taps are monotone; the same set under flip)
+int span16(const GroupParams& g) {
+  int lo, hi, d;
+  float l;
+  tap_ref(g.sc_x, g.off_x, 0, g.lim_x, g.org_x, &lo, &d, &l);
+  tap_ref(g.sc_x, g.off_x, g.out_w - 1, g.lim_x, g.org_x, &d, &hi, &l);
+  return ((hi + 16) & ~15) - (lo & ~15);
+}
+
+int row_tap0(const GroupParams& g, int o) {
+  int a, b;
+  float l;
+  tap_ref(g.sc_y, g.off_y, o, g.lim_y, g.org_y, &a, &b, &l);
+  return a;
+}
+int row_tap1(const GroupParams& g, int o) {
+  int a, b;
+  float l;
+  tap_ref(g.sc_y, g.off_y, o, g.lim_y, g.org_y, &a, &b, &l);
+  return b;
+}
+
+// k_plain shared-memory needs of one band [y0, y0 + nr) of a group, walked in sub-bands of
+// kPlainS rows exactly as the kernel does: ring rows live at once and staged rows per sub-band
+void plain_band_bounds(const GroupParams& g, int y0, int nr, int* ring, int* raw, int* conv_rows) {
+  *ring = 0;
+  *raw = 0;
+  int ya = row_tap0(g, y0), yb = -1;
+  const int first = ya;
+  for (int k = 0; k * kPlainS < nr; ++k) {
+    const int r_lo = k * kPlainS, r_hi = std::min(nr, r_lo + kPlainS) - 1;
+    const int last = row_tap1(g, y0 + r_hi);
+    *ring = std::max(*ring, last - row_tap0(g, y0 + r_lo) + 1);
+    const int na = k == 0 ? ya : yb + 1;
+    if (last >= na) *raw = std::max(*raw, (last - na + 1) + ((last >> 1) - (na >> 1) + 1));
+    yb = std::max(yb, last);
+  }
+  *conv_rows = yb - first + 1;
+}
+
+// k_plain tasks of one batch's mild items [0, n) (ordered by clip slot, group, frame): runs of
+// one (clip slot, group) in chunks of `fpc` frames x bands of kPlainRB rows; the costliest first
+// (the block scheduler then approximates longest-processing-time order), and the cheapest
+// quarter of the work split into kPlainRBTail-row bands so the grid's last wave is short.
+// Also returns the exact shared-memory bounds over the tasks.
+void plain_tasks(const std::vector<WorkItem>& items, size_t first, size_t n, const std::vector<GroupParams>& groups,
+                 int fpc, std::vector<uint2>* out, BatchShape* shape) {
+  struct T {
+    uint32_t item, nfr, y0, nr;
+    double cost;
+  };
+  std::vector<T> ts;
+  auto cost_of = [&](const GroupParams& g, uint32_t nfr, int y0, int nr) {
+    int ring, raw, conv;
+    plain_band_bounds(g, y0, nr, &ring, &raw, &conv);
+    // lane instructions: ~4.4 per converted channel value, ~8 per output value
+    return (double)nfr * (4.4 * 3.0 * conv * span16(g) + 8.0 * 3.0 * nr * g.out_w);
+  };
+  for (size_t i = 0; i < n;) {
+    size_t j = i;
+    while (j < n && items[first + j].clip_slot == items[first + i].clip_slot &&
+           items[first + j].group == items[first + i].group)
+      ++j;
+    const GroupParams& g = groups[items[first + i].gp];
+    for (size_t f0 = i; f0 < j; f0 += fpc) {
+      const uint32_t nfr = (uint32_t)std::min<size_t>(fpc, j - f0);
+      for (int y0 = 0; y0 < g.out_h; y0 += kPlainRB) {
+        const int nr = std::min(kPlainRB, g.out_h - y0);
+        ts.push_back({(uint32_t)f0, nfr, (uint32_t)y0, (uint32_t)nr, cost_of(g, nfr, y0, nr)});
+      }
+    }
+    i = j;
+  }
+  std::stable_sort(ts.begin(), ts.end(), [](const T& a, const T& b) { return a.cost > b.cost; });
+  double total = 0.0;
+  for (const T& t : ts) total += t.cost;
+  std::vector<T> big, tail;
+  double acc = 0.0;
+  for (auto it = ts.rbegin(); it != ts.rend(); ++it) {   // cheapest first
+    acc += it->cost;
+    if (acc <= kPlainTailFrac * total && (int)it->nr > kPlainRBTail) {
+      const GroupParams& g = groups[items[first + it->item].gp];
+      for (uint32_t y = it->y0; y < it->y0 + it->nr; y += kPlainRBTail) {
+        const uint32_t nr = std::min<uint32_t>(kPlainRBTail, it->y0 + it->nr - y);
+        tail.push_back({it->item, it->nfr, y, nr, cost_of(g, it->nfr, (int)y, (int)nr)});
+      }
+    } else {
+      big.push_back(*it);
+    }
+  }
+  std::reverse(big.begin(), big.end());
+  std::stable_sort(tail.begin(), tail.end(), [](const T& a, const T& b) { return a.cost > b.cost; });
+  shape->task_first = (uint32_t)out->size();
+  shape->pl_gw = shape->pl_ring = shape->pl_raw = shape->pl_rb = 0;
+  for (const auto* v : {&big, &tail})
+    for (const T& t : *v) {
+      const GroupParams& g = groups[items[first + t.item].gp];
+      int ring, raw, conv;
+      plain_band_bounds(g, (int)t.y0, (int)t.nr, &ring, &raw, &conv);
+      shape->pl_ring = std::max(shape->pl_ring, ring);
+      shape->pl_raw = std::max(shape->pl_raw, raw);
+      shape->pl_gw = std::max(shape->pl_gw, span16(g));
+      shape->pl_rb = std::max(shape->pl_rb, (int)t.nr);
+      out->push_back(make_uint2(t.item, pl_task_y(t.nfr, t.nr, t.y0)));
+    }
+  shape->n_tasks = (uint32_t)out->size() - shape->task_first;
+}
+
 }  // namespace
 
 std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32_t rank,
@@ -99,6 +203,7 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
   plan->last_touch = 0;
   plan->items.clear();
   plan->dests.clear();
+  plan->tasks.clear();
   plan->item_begin.clear();
   plan->shapes.clear();
   plan->fetch_begin.clear();
@@ -159,15 +264,18 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
       uint32_t gflags[SAND_MAX_GROUPS];
       for (uint32_t gi = 0; gi < nG; ++gi) {
         const GroupParams& g = plan->groups[slot * nG + gi];
-        gflags[gi] = (g.rot_on || g.blur_on) ? 1u : 0u;
-        const int cols = std::min(2 * g.out_w, static_cast<int>(std::ceil(static_cast<double>(g.sc_x) * g.out_w)) + 3);
-        if (gflags[gi]) {
+        // the exact staged span (16-aligned; an estimate capped at 2 * out_w let a
+        // wide crop overrun the staging kernels' shared memory)
+        const int cols = span16(g);
+        const bool mild = g.sc_x <= 2.0f && g.sc_y <= 2.0f;
+        gflags[gi] = (g.rot_on || g.blur_on) ? 1u : (mild ? 0u : 2u);
+        if (gflags[gi] & 1u) {
           shape.has_stencil = 1;
           shape.st_max_wo = std::max(shape.st_max_wo, g.out_w);
           shape.st_max_ho = std::max(shape.st_max_ho, g.out_h);
           shape.st_cols_bound = std::max(shape.st_cols_bound, cols);
           shape.st_max_scy = std::max(shape.st_max_scy, g.sc_y);
-        } else {
+        } else if (mild) {
           shape.has_direct = 1;
           if (!(g.sc_x == 1.0f && g.sc_y == 1.0f)) shape.direct_identity = 0;
           if (dim.width % 4u) shape.src_w_mod4 = 0;
@@ -175,6 +283,10 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
           shape.max_ho = std::max(shape.max_ho, g.out_h);
           shape.cols_bound = std::max(shape.cols_bound, cols);
           shape.max_scy = std::max(shape.max_scy, g.sc_y);
+        } else {
+          shape.has_direct = 1;
+          shape.heavy_max_wo = std::max(shape.heavy_max_wo, g.out_w);
+          shape.heavy_max_ho = std::max(shape.heavy_max_ho, g.out_h);
         }
       }
       // (frame, view, t) uses of the clip sorted by frame: one pass groups the destinations of
@@ -200,6 +312,7 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
           }
           w.n_dest = static_cast<uint32_t>(plan->dests.size()) - w.dest_begin;
           if (w.n_dest == 0) continue;
+          if (!(gflags[gi] & 1u)) shape.max_dests = std::max<int32_t>(shape.max_dests, static_cast<int32_t>(w.n_dest));
           uses += w.n_dest;
           w.y_off = ent->offset + ent->frame_stride * f;
           w.pitch = ent->pitch;
@@ -237,6 +350,15 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
       auto first = plan->items.begin() + plan->item_begin.back();
       auto mid = std::stable_partition(first, plan->items.end(), [](const sand::WorkItem& w) { return !(w.flags & 1u); });
       shape.n_direct = static_cast<uint32_t>(mid - first);
+      // direct items: mild (k_plain) before heavy (k_direct); mild ones in (clip slot, group,
+      // frame) order so the frames of one clip group are adjacent (a k_plain task)
+      auto hv = std::stable_partition(first, mid, [](const sand::WorkItem& w) { return !(w.flags & 2u); });
+      shape.n_mild = static_cast<uint32_t>(hv - first);
+      std::stable_sort(first, hv, [](const sand::WorkItem& a, const sand::WorkItem& b) {
+        return a.clip_slot != b.clip_slot ? a.clip_slot < b.clip_slot : a.group < b.group;
+      });
+      plain_tasks(plan->items, static_cast<size_t>(plan->item_begin.back()), shape.n_mild, plan->groups, v.pl_fpc,
+                  &plan->tasks, &shape);
       // stencil items longest first (one CTA per item, dispatched in order): the grid's last
       // wave then holds the cheapest items. Cost model in lane instructions per output value
       // (ncu): resample ~15, rotation ~28, blur ~10 + 3 r.
@@ -291,7 +413,7 @@ void free_pool(sand_view* v) {
 }
 
 struct PlanLayout {
-  size_t gb, ib, db, off_i, off_d, total;
+  size_t gb, ib, db, tb, off_i, off_d, off_t, total;
 };
 
 PlanLayout plan_layout(const EpochPlan& p) {
@@ -299,9 +421,11 @@ PlanLayout plan_layout(const EpochPlan& p) {
   L.gb = p.groups.size() * sizeof(GroupParams);
   L.ib = p.items.size() * sizeof(WorkItem);
   L.db = p.dests.size() * sizeof(uint32_t);
+  L.tb = p.tasks.size() * sizeof(uint2);
   L.off_i = (L.gb + 255) / 256 * 256;
   L.off_d = L.off_i + (L.ib + 255) / 256 * 256;
-  L.total = std::max<size_t>(L.off_d + L.db, 256);
+  L.off_t = L.off_d + (L.db + 255) / 256 * 256;
+  L.total = std::max<size_t>(L.off_t + L.tb, 256);
   return L;
 }
 
@@ -383,6 +507,7 @@ int upload_plan(sand_view* v, EpochPlan& p, PlanBuffer* buf) {
   if (L.gb) std::memcpy(h, p.groups.data(), L.gb);
   if (L.ib) std::memcpy(h + L.off_i, p.items.data(), L.ib);
   if (L.db) std::memcpy(h + L.off_d, p.dests.data(), L.db);
+  if (L.tb) std::memcpy(h + L.off_t, p.tasks.data(), L.tb);
   e = cudaMemcpyAsync(buf->d, buf->h, L.total, cudaMemcpyHostToDevice, v->upload_stream);
   if (e != cudaSuccess) return cuda_error(e, "cudaMemcpyAsync(plan)");
   e = cudaEventRecord(buf->ready, v->upload_stream);
@@ -397,6 +522,7 @@ int upload_plan(sand_view* v, EpochPlan& p, PlanBuffer* buf) {
   p.d_groups = reinterpret_cast<GroupParams*>(d);
   p.d_items = reinterpret_cast<WorkItem*>(d + L.off_i);
   p.d_dests = reinterpret_cast<uint32_t*>(d + L.off_d);
+  p.d_tasks = reinterpret_cast<uint2*>(d + L.off_t);
   p.uploaded = true;
   return SAND_OK;
 }
@@ -449,11 +575,13 @@ std::shared_ptr<EpochPlan> get_plan(sand_view* v, std::unique_lock<std::mutex>& 
   v->plans_built++;
   plan->last_touch = ++v->touch;
   v->plans[key] = plan;
-  while (v->plans.size() > kPlanCache) {   // evict the least recently used plan
-    auto victim = v->plans.begin();
+  while (v->plans.size() > kPlanCache) {   // evict the least recently used unpinned plan
+    auto victim = v->plans.end();
     for (auto i = v->plans.begin(); i != v->plans.end(); ++i)
-      if (i->second->last_touch < victim->second->last_touch) victim = i;
-    if (victim->first == key) break;
+      if (i->first != key && i->second->pins == 0 &&
+          (victim == v->plans.end() || i->second->last_touch < victim->second->last_touch))
+        victim = i;
+    if (victim == v->plans.end()) break;
     release_plan_device(v, *victim->second);
     if (victim->second.use_count() == 1) v->spare_plans.push_back(std::move(victim->second));
     v->plans.erase(victim);
@@ -543,6 +671,12 @@ extern "C" int sand_view_create(sand_store* s, const sand_view_spec* spec, sand_
     return sand::cuda_error(e, "cudaSetDevice");
   }
   v->stencil_smem = stencil ? sand::stencil_smem_bytes(max_h, max_w, max_r) : 0;
+  {   // k_plain CTA: frames of one clip group side by side, NQ = column quads of the widest view
+    uint32_t wmax = 4;
+    for (uint32_t k = 0; k < spec->n_views; ++k) wmax = std::max(wmax, spec->views[k].out_w);
+    v->pl_nq = static_cast<int>((wmax + 3) / 4);
+    v->pl_fpc = std::max(1, std::min(8, 224 / v->pl_nq));   // <= 224 threads (k_plain launch bounds)
+  }
   rc = sand::configure_kernels(v->stencil_smem);
   if (rc != SAND_OK) {
     delete v;
@@ -553,19 +687,8 @@ extern "C" int sand_view_create(sand_store* s, const sand_view_spec* spec, sand_
     delete v;
     return sand::cuda_error(e, "cudaStreamCreate(upload)");
   }
-  // ticket counters of the persistent kernels: zero between launches (each launch's last CTA
-  // clears its slot); successive launches rotate through the slots
-  e = cudaMalloc(&v->d_sched, 2 * sand::kSchedSlots * sizeof(uint32_t));
-  if (e == cudaSuccess) e = cudaMemset(v->d_sched, 0, 2 * sand::kSchedSlots * sizeof(uint32_t));
-  if (e == cudaSuccess) e = cudaDeviceSynchronize();
-  if (e != cudaSuccess) {
-    if (v->d_sched) cudaFree(v->d_sched);
-    cudaStreamDestroy(v->upload_stream);
-    delete v;
-    return sand::cuda_error(e, "cudaMalloc(scheduler counters)");
-  }
   s->live_views++;
-  const int n_workers = sand::env_int("SAND_PLAN_THREADS", 2, 1, 16);
+  const int n_workers = 2;   // plan builders: the current epoch's and the next one's
   for (int i = 0; i < n_workers; ++i) v->workers.emplace_back(sand::worker_loop, v);
   *out = v;
   return SAND_OK;
@@ -653,6 +776,13 @@ extern "C" int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank,
                                                 std::to_string(key.first) + " is not in the store");
       }
     }
+    // frames put since this stream last waited: order the kernel after their copies
+    if (st->put_seq > 0 && (st->put_seq != v->put_seq_seen || stream != v->put_stream_seen)) {
+      e = cudaStreamWaitEvent(stream, st->last_put, 0);
+      if (e != cudaSuccess) return sand::cuda_error(e, "cudaStreamWaitEvent(last_put)");
+      v->put_seq_seen = st->put_seq;
+      v->put_stream_seen = stream;
+    }
   }
   // bound the read-ahead: at most kInflight batches of this view are queued on the GPU. An
   // unbounded run-ahead keeps many epoch plans alive at once (more plan buffers, allocations
@@ -666,10 +796,15 @@ extern "C" int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank,
     }
   }
   if (v->batches >= sand::kInflight) {
+    // the plan is pinned while the lock is dropped: a builder thread cannot evict it and
+    // recycle its device buffer before the kernel below has been launched
+    plan->pins++;
     lk.unlock();
     e = cudaEventSynchronize(v->inflight[slot]);
     lk.lock();
+    plan->pins--;
     if (e != cudaSuccess) return sand::cuda_error(e, "cudaEventSynchronize(inflight)");
+    if (!plan->uploaded) return sand::set_error(SAND_ECUDA, "plan lost its device copy");
   }
   sand::LaunchParams lp{};
   lp.slab = st->slab;
@@ -679,23 +814,22 @@ extern "C" int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank,
   lp.dests = plan->d_dests;
   lp.n_views = s.n_views;
   lp.batch = s.batch_size;
-  lp.sched = v->d_sched;
-  lp.sched_slot = v->sched_seq;   // launch_materialize uses slots sched_slot and sched_slot + 1
-  v->sched_seq = (v->sched_seq + 2) % sand::kSchedSlots;
+  lp.tasks = plan->d_tasks;
   for (uint32_t k = 0; k < s.n_views; ++k) {
     lp.out[k] = out->data[k];
     lp.views[k] = v->vconst[k];
   }
   int launched = 0;
   const sand::BatchShape& bshape = plan->shapes[it];
-  if (bshape.has_direct && bshape.has_stencil && !v->aux_stream && getenv("SAND_NO_FORK") == nullptr) {
+  const int classes = (bshape.n_mild > 0) + (bshape.n_direct > bshape.n_mild) + (lp.n_items > bshape.n_direct);
+  if (classes > 1 && !v->aux_stream) {
     e = cudaStreamCreateWithFlags(&v->aux_stream, cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&v->fork_ev, cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&v->join_ev, cudaEventDisableTiming);
     if (e != cudaSuccess) return sand::cuda_error(e, "aux stream for the direct kernel");
   }
-  int rc = sand::launch_materialize(lp, bshape, v->stencil_smem, stream, v->aux_stream, v->fork_ev, v->join_ev,
-                                    &launched);
+  int rc = sand::launch_materialize(lp, bshape, v->stencil_smem, v->pl_fpc, v->pl_nq, stream, v->aux_stream, v->fork_ev,
+                                    v->join_ev, &launched);
   if (rc != SAND_OK) return rc;
   e = cudaEventRecord(plan->last_use, stream);
   if (e == cudaSuccess) e = cudaEventRecord(v->inflight[slot], stream);
@@ -826,7 +960,6 @@ extern "C" int sand_view_destroy(sand_view* v) {
   if (v->aux_stream) cudaStreamDestroy(v->aux_stream);
   if (v->fork_ev) cudaEventDestroy(v->fork_ev);
   if (v->join_ev) cudaEventDestroy(v->join_ev);
-  if (v->d_sched) cudaFree(v->d_sched);
   for (auto& ev : v->inflight)
     if (ev) cudaEventDestroy(ev);
   v->store->live_views--;

@@ -107,3 +107,35 @@ def test_host_plan_linspace_slow_pathway_matches_oracle():
     bad.views[0].subsample_of = 1            # a sub-sample of a sub-sample
     with pytest.raises(sand.SandError):
         sand.plan_clip(bad, vids, 0, 0)
+
+
+def _plan_equal(spec, vids, epochs, clips):
+    ospec = to_oracle(spec)
+    ods = oracle.make_dataset(vids)
+    for epoch in epochs:
+        for clip in clips:
+            got = sand.plan_clip(spec, vids, epoch, clip)
+            ref = oracle.ClipMeta()
+            oracle.lib().oracle_plan_clip(oracle.ctypes.byref(ospec), ods, epoch, clip, oracle.ctypes.byref(ref))
+            assert meta_fields(spec, got) == meta_fields(spec, ref), (epoch, clip)
+            yield got
+
+
+def test_host_plan_short_video_clamp_matches_oracle():
+    """Videos shorter than the shared pool (F < P, R#4): start 0 and indices clamped to F - 1."""
+    w = configs.slowfast()
+    vids = [(1000 + i, 20 + 7 * i, 340, 256) for i in range(6)]     # F in 20..55 < P = 63
+    for got in _plan_equal(w.spec, vids, (0, 3), range(6)):
+        F = vids[got.clip][1]
+        assert got.pool_start == 0 and max(got.frames[0][:32]) == F - 1
+
+
+def test_host_plan_rrc_central_fallback_matches_oracle():
+    """An RRC range no attempt satisfies takes torchvision's central fallback (R#8), in both
+    directions of the ratio clamp."""
+    for ratio, box in (((2.5, 3.0), [0, 60, 340, 136]), ((0.2, 0.25), [138, 0, 64, 256])):
+        spec = configs.Spec(batch_size=1, views=[configs.ViewSpec(clip_len=4, stride=2, scale=(0.95, 1.0),
+                                                                  ratio=ratio)])
+        vids = [(1000 + i, 30, 340, 256) for i in range(4)]
+        for got in _plan_equal(spec, vids, (0, 1, 5), range(4)):
+            assert list(got.box[0]) == box
