@@ -26,7 +26,7 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-DEFAULT_STEPS = {"tiny": 2000, "k400": 3000, "slowfast": 3000, "twoview": 1000, "ray": 1000}
+DEFAULT_STEPS = {"tiny": 2000, "k400": 3000, "slowfast": 3000, "twoview": 1000, "ray": 1000, "slowfast_hd": 1000}
 
 
 def log(*a):
@@ -102,10 +102,9 @@ def measured_peaks():
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-# the kernel that dominates each config's step (the roofline's subject; `achieved` divides the
-# step's algorithmic bytes by the summed duration of every kernel read_batch launched)
-DOMINANT_KERNEL = {"tiny": "k_stream", "k400": "k_stream", "slowfast": "k_copy",
-                   "twoview": "k_stencil2 (with k_stream for the plain items)", "ray": "k_direct"}
+# kernel of each item class (SAND_N_CLASSES: mild plain, heavy plain, rotation/blur); the roofline's
+# subject is the class with the most kernel time, its bytes / its own event-timed duration
+CLASS_KERNELS = {"slowfast": ("k_copy", "k_direct", "k_stencil2")}
 
 
 def ncu_traffic(config: str):
@@ -257,9 +256,16 @@ def run_sand(args):
     rank, world, local = dist_env()
     if world != args.gpus:
         log(f"warning: --gpus {args.gpus} but WORLD_SIZE={world}; using WORLD_SIZE")
+    # one process per GPU over NCCL; --backend gloo (tests) lets several ranks share a device
+    if args.backend == "gloo":
+        local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group("gloo")
+    coll_dev = f"cuda:{local}" if args.backend == "nccl" else "cpu"
     w = configs.get(args.config)
     spec = w.spec
     spec.world_size = world
@@ -353,21 +359,53 @@ def run_sand(args):
     slow = [(i, round(x, 3)) for i, x in enumerate(kraw) if x > 2 * kt[len(kt) // 2]]
     host["slow_steps"] = {"n": len(slow), "ms_total": round(sum(x for _, x in slow), 3),
                           "first": [(first_timed + i, x) for i, x in slow[:8]], "iters_per_epoch": iters}
-    elapsed_ms, kernel_ms_max = max_over_ranks([elapsed_ms, kernel_ms], world, f"cuda:{local}")
+    elapsed_ms, kernel_ms_max = max_over_ranks([elapsed_ms, kernel_ms], world, coll_dev)
     ms_per_step = elapsed_ms / args.steps
     value = fps * args.steps * world / (elapsed_ms / 1000.0)
 
-    # reuse counters: the only collective (NCCL all_gather of a few integers)
+    # reuse counters of the warm-up + timed batches: the only collective (an all_gather of a few
+    # integers over NCCL)
     c = store.counters()
-    totals, _ = gather_counters([c.fetches, c.uses, c.batches], world, f"cuda:{local}")
+    totals, per_rank = gather_counters([c.fetches, c.uses, c.batches], world, coll_dev)
+
+    # per-kernel roofline: each item class is its own kernel; time each class with
+    # CUDA events recorded by the library around its launch, on the stream it runs on, over a
+    # separate pass of the same batches (so the timed loop above carries no timing events)
+    cls_names = CLASS_KERNELS.get(args.config, ("k_plain", "k_direct", "k_stencil2"))
+    view.set_timing(True)
+    n_cls_steps = min(args.steps, 200)
+    s_cls = first_timed
+    for _ in range(n_cls_steps):
+        e, it = step_id(s_cls)
+        view.read_batch(e, rank, it, outs_a if s_cls % 2 == 0 else outs_b, stream.cuda_stream)
+        s_cls += 1
+    cls_ms, cls_n = view.class_times()
+    view.set_timing(False)
+    cls_bytes = [[0.0, 0.0] for _ in range(3)]
+    for e, it in sample:
+        for c in range(3):
+            b = view.batch_bytes_class(e, rank, it, c)
+            cls_bytes[c][0] += b.src_bytes / len(sample)
+            cls_bytes[c][1] += b.out_bytes / len(sample)
+    per_class = {}
+    for c in range(3):
+        if cls_n[c]:
+            ms_each = cls_ms[c] / cls_n[c]
+            per_class[cls_names[c]] = {"ms_per_launch": ms_each, "launches": int(cls_n[c]),
+                                       "alg_bytes_per_launch": {"read": cls_bytes[c][0], "write": cls_bytes[c][1]},
+                                       "achieved_gbs": (cls_bytes[c][0] + cls_bytes[c][1]) / (ms_each / 1e3) / 1e9}
+    dom = max(per_class, key=lambda k: per_class[k]["ms_per_launch"] * per_class[k]["launches"]) if per_class else None
+
+
 
     # ---- e2e through the C-ABI with HOST buffers
     e2e = None
     if not args.no_e2e:
-        e2e = run_e2e(args, w, spec, view, store, stream, rank, iters, s, world)
+        e2e = run_e2e(args, w, spec, view, store, stream, rank, iters, s, world, coll_dev)
 
     peak, peak_src = measured_peaks()
-    achieved = (alg_read + alg_write) / (kernel_ms / 1000.0) / 1e9
+    step_achieved = (alg_read + alg_write) / (kernel_ms / 1000.0) / 1e9
+    achieved = per_class[dom]["achieved_gbs"] if dom else step_achieved
     line = {
         "metric": "output frames/s", "value": value, "unit": "frames/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
@@ -376,14 +414,20 @@ def run_sand(args):
         "batches_per_s": value / fps,
         "per_gpu_frames_per_s": value / world,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                     "traffic": ncu_traffic(args.config), "kernel": DOMINANT_KERNEL.get(args.config, "k_stream"),
-                     "alg_bytes_per_launch": {"read": alg_read, "write": alg_write},
-                     "kernel_ms_per_step": kernel_ms, "peak_source": peak_src,
-                     "frac_of_8tbs_spec": achieved / 8000.0},
+                     "traffic": ncu_traffic(args.config), "kernel": dom,
+                     "alg_bytes_per_launch": (per_class[dom]["alg_bytes_per_launch"] if dom else
+                                              {"read": alg_read, "write": alg_write}),
+                     "ms_per_launch": per_class[dom]["ms_per_launch"] if dom else kernel_ms,
+                     "per_kernel": per_class,
+                     "step": {"achieved": step_achieved, "frac": step_achieved / peak, "kernel_ms_per_step": kernel_ms,
+                              "alg_bytes": {"read": alg_read, "write": alg_write}},
+                     "peak_source": peak_src, "frac_of_8tbs_spec": achieved / 8000.0},
         "gpu_launches": int(launches),
         "host": host,
         "clocks": clk,
-        "reuse": {"fetches": totals[0], "uses": totals[1], "batches": totals[2]},
+        "reuse": {"fetches": totals[0], "uses": totals[1], "batches": totals[2], "per_rank": per_rank},
+        "collectives": {"backend": args.backend if world > 1 else None,
+                        "timing": "max over ranks of CUDA-event times", "counters": "all_gather"},
     }
     if e2e is not None:
         line["e2e"] = e2e
@@ -398,7 +442,7 @@ def run_sand(args):
     return 0
 
 
-def run_e2e(args, w, spec, view, store, stream, rank, iters, s0, world):
+def run_e2e(args, w, spec, view, store, stream, rank, iters, s0, world, coll_dev):
     """Same metric end to end through the public API: every step copies its input frames
     from pinned host memory into the store (one sand_store_put_frame_batch: one H2D copy of
     the packed frames + one scatter kernel), reads the batch, and copies the batch back to
@@ -454,18 +498,93 @@ def run_e2e(args, w, spec, view, store, stream, rank, iters, s0, world):
     stream.wait_stream(copy_stream)
     end.record(stream)
     torch.cuda.synchronize()
-    ms = max_over_ranks([start.elapsed_time(end)], world, f"cuda:{torch.cuda.current_device()}")[0]
+    ms = max_over_ranks([start.elapsed_time(end)], world, coll_dev)[0]
     return {"value": frames_per_step(spec) * n * world / (ms / 1000.0), "unit": "frames/s",
             "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h), "steps": n,
             "ms_per_step": ms / n, "api": "sand_store_put_frame_batch + sand_view_read_batch, D2H overlapped"}
 
 
-def cpu_baseline(w, spec, vids, args):
+def cpu_model() -> str:
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for ln in out.splitlines():
+            if ln.startswith("Model name:"):
+                return ln.split(":", 1)[1].strip()
+    except (OSError, subprocess.SubprocessError):
+        pass
+    return "unknown"
+
+
+def _oracle_worker(config, cpu, index, procs, seconds, q):
+    """One pinned oracle process: renders output frames index, index + procs, ... of the
+    workload's batches (disjoint across processes) for `seconds` (the box-level
+    CPU rate, P = os.cpu_count() pinned processes over disjoint clips)."""
+    try:
+        os.sched_setaffinity(0, {cpu})
+    except (AttributeError, OSError):
+        pass
+    import oracle
     import synth
-    done, el = oracle_frames_per_second(w, spec, vids, None, args.cpu_seconds, synth.UNIFORM, 1234, warmup=1)
-    return {"value": done / el, "unit": "frames/s", "cores": 1, "kind": "oracle",
-            "sample": f"{done} output frames of batch (epoch 0, rank 0, it 0) rendered one by one by the "
-                      f"single-threaded C oracle in {el:.1f}s (source-frame generation excluded)"}
+    from paper_conf_sosp_yelllhkh25_b200 import configs
+    w = configs.get(config)
+    spec = w.spec
+    spec.world_size = 1
+    vids = [(1000 + i, w.n_frames, w.width, w.height) for i in range(w.n_videos)]
+    ospec = _oracle_spec(spec)
+    ods = oracle.make_dataset(vids)
+    order = []
+    it = 0
+    while len(order) < 4 * procs and it < oracle.iterations(ospec, len(vids)):
+        metas = oracle.plan_batch(ospec, ods, len(vids), 0, 0, it)
+        order += [(metas[b], k) + (metas[b].frames[k][t],) for b in range(spec.batch_size)
+                  for k, v in enumerate(spec.views) for t in range(v.clip_len)]
+        it += 1
+    mine = order[index::procs][:64]
+    src = {}
+    for m, k, f in mine:           # source frames generated before the clock starts
+        if (m.video, f) not in src:
+            y, uv = synth.frames(synth.UNIFORM, 1234, m.video, f, 1, w.width, w.height)
+            src[(m.video, f)] = (y[0], uv[0])
+    done, t0 = 0, time.perf_counter()
+    while time.perf_counter() - t0 < seconds:
+        m, k, f = mine[done % len(mine)]
+        y, uv = src[(m.video, f)]
+        oracle.render_frame(ospec, m, k, y, uv)
+        done += 1
+    q.put((done, time.perf_counter() - t0))
+
+
+def cpu_baseline(w, spec, vids, args):
+    """The oracle as it stands on the box's host cores: one pinned process per core over
+    disjoint output frames (box rate), the single-core rate, the CPU model and the paper's
+    12-cores-per-GPU provisioning as context."""
+    import multiprocessing as mp
+    import synth
+    done1, el1 = oracle_frames_per_second(w, spec, vids, None, min(args.cpu_seconds, 6.0), synth.UNIFORM, 1234,
+                                          warmup=1)
+    try:
+        cpus = sorted(os.sched_getaffinity(0))
+    except AttributeError:
+        cpus = list(range(os.cpu_count() or 1))
+    procs = len(cpus)
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    ps = [ctx.Process(target=_oracle_worker, args=(args.config, cpus[i], i, procs, args.cpu_seconds, q))
+          for i in range(procs)]
+    for p in ps:
+        p.start()
+    res = [q.get(timeout=600) for _ in ps]
+    for p in ps:
+        p.join()
+    box = sum(d / e for d, e in res)
+    return {"value": box, "unit": "frames/s", "cores": procs, "kind": "oracle",
+            "cpu_model": cpu_model(),
+            "sample": f"{procs} pinned processes (one per host core), each rendering disjoint output frames of the "
+                      f"workload's first batches one by one with the single-threaded C oracle for "
+                      f"{args.cpu_seconds:.0f}s (source-frame generation excluded); box rate = sum of per-process rates",
+            "single_core": {"value": done1 / el1, "frames": done1, "seconds": round(el1, 2)},
+            "per_12_cores": box * 12.0 / procs,
+            "per_12_cores_note": "the paper provisions 12 CPU cores per GPU (P:L120, P:L414): box rate x 12 / cores"}
 
 
 def main():
@@ -473,13 +592,15 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=None)
     ap.add_argument("--warmup", type=int, default=20)
-    ap.add_argument("--config", default="k400", choices=["tiny", "k400", "slowfast", "twoview", "ray"])
+    ap.add_argument("--config", default="k400", choices=["tiny", "k400", "slowfast", "twoview", "ray", "slowfast_hd"])
     ap.add_argument("--impl", default="sand", choices=["sand", "reference"])
     ap.add_argument("--videos", type=int, default=None, help="override the store size (videos per GPU)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=16)
-    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process-group backend (gloo: test mode, ranks may share one GPU)")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0)
     args = ap.parse_args()
     if args.steps is None:
         args.steps = DEFAULT_STEPS[args.config] if args.impl == "sand" else 200

@@ -207,6 +207,24 @@ typedef struct {
  * ERANGE (iteration), ENOENT (a planned frame is absent), ECUDA (launch failure). */
 int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank, const sand_batch_out* out);
 
+/* Pre-materialisation (§5.4). sand_view_prematerialize runs the
+ * kernels of batch (epoch, rank, iteration) AHEAD of its read, into a library-owned device
+ * buffer, on the view's own low-priority stream, so they overlap whatever the caller's
+ * streams are doing (the training step); it returns immediately. A later read of that batch
+ * is served from the buffer: sand_view_read_batch makes out->stream wait for the batch and
+ * copies it into out->data (device to device); or sand_view_acquire_batch hands the buffer
+ * itself to the caller (data_out[k] = device pointer of view k, valid until
+ * sand_view_release_batch; no copy). Results are bit-identical to a direct read.
+ * sand_view_set_prematerialize(v, slots) allocates `slots` batch buffers (0 frees them; the
+ * call waits for outstanding work). Errors: EINVAL (no slots configured, null pointers),
+ * EBUSY (every slot holds a batch not yet read / released), ERANGE (acquire/release of a batch
+ * that is not pre-materialised), plus read_batch's. */
+int sand_view_set_prematerialize(sand_view* v, uint32_t slots);
+int sand_view_prematerialize(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration);
+int sand_view_acquire_batch(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration, sand_stream_t stream,
+                            void* data_out[SAND_MAX_VIEWS]);
+int sand_view_release_batch(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration, sand_stream_t stream);
+
 /* Plan an epoch ahead of time on a background host thread (the plan analogue of
  * the paper's pre-materialisation threads). Returns immediately. */
 int sand_view_prefetch_epoch(sand_view* v, uint64_t epoch, uint32_t rank);
@@ -233,6 +251,25 @@ typedef struct {
 } sand_batch_bytes;
 int sand_view_batch_bytes(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration,
                           sand_batch_bytes* out);
+
+/* Item classes of a batch (each launched as its own kernel): 0 = plain items with a source
+ * step <= 2 on both axes (k_plain / k_copy / k_stream), 1 = plain items with heavier
+ * down-scaling (k_direct), 2 = items with rotation and/or blur (k_stencil2). */
+#define SAND_N_CLASSES 3
+
+/* sand_view_batch_bytes restricted to the items of class `cls`: the sectors the class's own
+ * taps touch (deduplicated within the class), the bytes its items write, its fetches and uses.
+ * The per-kernel roofline numerator of the measurement. Errors: EINVAL, ERANGE. */
+int sand_view_batch_bytes_class(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration, uint32_t cls,
+                                sand_batch_bytes* out);
+
+/* Per-class kernel timing (measurement only): with sand_view_set_timing(v, 1) every
+ * read_batch records CUDA events around each class's kernel on the stream it is launched on;
+ * sand_view_class_times waits for the recorded events and returns, per class, the summed
+ * milliseconds and launch count since the previous call (then resets them). Timing is off by
+ * default (read_batch records nothing). Errors: EINVAL, ECUDA. */
+int sand_view_set_timing(sand_view* v, int on);
+int sand_view_class_times(sand_view* v, double ms[SAND_N_CLASSES], uint64_t launches[SAND_N_CLASSES]);
 
 /* Host-only planning (no store, no device): the same planner read_batch uses.
  * sand_plan_rank_clips writes the global clip ids of (epoch, rank) in DistributedSampler

@@ -208,6 +208,40 @@ class View:
               "sand_view_batch_bytes")
         return out
 
+    def batch_bytes_class(self, epoch: int, rank: int, iteration: int, cls: int) -> _abi.sand_batch_bytes:
+        out = _abi.sand_batch_bytes()
+        check(lib().sand_view_batch_bytes_class(self._h, epoch, rank, iteration, cls, ctypes.byref(out)),
+              "sand_view_batch_bytes_class")
+        return out
+
+    def set_prematerialize(self, slots: int) -> None:
+        check(lib().sand_view_set_prematerialize(self._h, slots), "sand_view_set_prematerialize")
+
+    def prematerialize(self, epoch: int, rank: int, iteration: int) -> None:
+        check(lib().sand_view_prematerialize(self._h, epoch, rank, iteration), "sand_view_prematerialize")
+
+    def acquire_batch(self, epoch: int, rank: int, iteration: int, stream=None):
+        """Device pointers of a pre-materialised batch (one per view), valid until release."""
+        ptrs = (ctypes.c_void_p * _abi.MAX_VIEWS)()
+        check(lib().sand_view_acquire_batch(self._h, epoch, rank, iteration, _stream(stream), ptrs),
+              "sand_view_acquire_batch")
+        return [ptrs[k] for k in range(len(self.spec.views))]
+
+    def release_batch(self, epoch: int, rank: int, iteration: int, stream=None) -> None:
+        check(lib().sand_view_release_batch(self._h, epoch, rank, iteration, _stream(stream)),
+              "sand_view_release_batch")
+
+    def set_timing(self, on: bool) -> None:
+        check(lib().sand_view_set_timing(self._h, int(bool(on))), "sand_view_set_timing")
+
+    def class_times(self):
+        """(milliseconds, launches) per item class since the previous call (0 mild plain,
+        1 heavy plain, 2 rotation/blur)."""
+        ms = (ctypes.c_double * 3)()
+        n = (ctypes.c_uint64 * 3)()
+        check(lib().sand_view_class_times(self._h, ms, n), "sand_view_class_times")
+        return list(ms), list(n)
+
     def stats(self) -> _abi.sand_view_stats:
         out = _abi.sand_view_stats()
         check(lib().sand_view_get_stats(self._h, ctypes.byref(out)), "sand_view_get_stats")

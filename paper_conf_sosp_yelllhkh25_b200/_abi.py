@@ -102,6 +102,13 @@ SIGNATURES = {
     "sand_view_get_meta": (ctypes.c_int, [vp, u64, u32, u64, P(sand_clip_meta)]),
     "sand_view_batch_bytes": (ctypes.c_int, [vp, u64, u32, u64, P(sand_batch_bytes)]),
     "sand_view_get_stats": (ctypes.c_int, [vp, P(sand_view_stats)]),
+    "sand_view_batch_bytes_class": (ctypes.c_int, [vp, u64, u32, u64, u32, P(sand_batch_bytes)]),
+    "sand_view_set_timing": (ctypes.c_int, [vp, ctypes.c_int]),
+    "sand_view_set_prematerialize": (ctypes.c_int, [vp, u32]),
+    "sand_view_prematerialize": (ctypes.c_int, [vp, u64, u32, u64]),
+    "sand_view_acquire_batch": (ctypes.c_int, [vp, u64, u32, u64, vp, P(vp)]),
+    "sand_view_release_batch": (ctypes.c_int, [vp, u64, u32, u64, vp]),
+    "sand_view_class_times": (ctypes.c_int, [vp, P(ctypes.c_double), P(u64)]),
     "sand_view_destroy": (ctypes.c_int, [vp]),
     "sand_last_error": (ctypes.c_char_p, []),
     "sand_version": (ctypes.c_char_p, []),

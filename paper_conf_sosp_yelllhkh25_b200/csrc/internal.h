@@ -152,6 +152,29 @@ struct sand_view {
   // from / joined to the caller's stream) so it fills the SMs the stencil kernel's tail leaves idle
   cudaStream_t aux_stream = nullptr;
   cudaEvent_t fork_ev = nullptr, join_ev = nullptr;
+  // per-class kernel timing (sand_view_set_timing): event pairs recorded by read_batch
+  bool timing = false;
+  struct TimedLaunch {
+    int cls;
+    cudaEvent_t start, end;
+  };
+  std::vector<TimedLaunch> timed;                 // recorded, not yet collected
+  std::vector<cudaEvent_t> free_events;
+  double class_ms[3] = {0, 0, 0};
+  uint64_t class_launches[3] = {0, 0, 0};
+  // pre-materialisation (sand_view_prematerialize): batch buffers filled on a low-priority stream
+  struct PreSlot {
+    bool busy = false, acquired = false, consumed_pending = false;
+    uint64_t epoch = 0, iteration = 0;
+    uint32_t rank = 0;
+    uint8_t* buf = nullptr;
+    cudaEvent_t done = nullptr, consumed = nullptr;
+  };
+  std::vector<PreSlot> pre;
+  size_t pre_view_off[sand::kMaxViews] = {};
+  size_t pre_view_bytes[sand::kMaxViews] = {};
+  cudaStream_t pre_stream = nullptr;
+  uint64_t pre_made = 0, pre_served = 0;
   uint64_t put_seq_seen = 0;              // store->put_seq the last read_batch stream waited for
   cudaStream_t put_stream_seen = nullptr;
 };
@@ -167,7 +190,13 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
 size_t stencil_smem_bytes(int max_h, int max_w, int max_r);
 int configure_kernels(size_t stencil_smem);
 // aux/fork/join may be null (then the kernels run back to back on `stream`)
+// optional per-class event pairs recorded around each class's launch (null: no timing)
+struct ClassEvents {
+  cudaEvent_t start[3], end[3];
+  bool used[3];
+};
 int launch_materialize(const LaunchParams& p, const BatchShape& shape, size_t stencil_smem, int pl_fpc, int pl_nq,
-                       cudaStream_t stream, cudaStream_t aux, cudaEvent_t fork, cudaEvent_t join, int* n_launched);
+                       cudaStream_t stream, cudaStream_t aux, cudaEvent_t fork, cudaEvent_t join, int* n_launched,
+                       ClassEvents* ev = nullptr);
 
 }  // namespace sand

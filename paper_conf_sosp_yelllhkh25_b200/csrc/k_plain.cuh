@@ -5,59 +5,76 @@
 //
 // A TASK is (run of up to FPC items of ONE (clip slot, spatial group), band of output rows).
 // Spatial parameters are per clip and group (R#7), so the FPC frames of a task share every tap,
-// table and branch: the CTA holds FPC x NQ threads (NQ = output column quads per row; 4 x 56 =
-// 224 for 224-wide outputs, no idle lanes) whose control flow is identical, each frame with its
-// own source rows in shared memory. Per band, sub-bands of S output rows are processed as
-//   * the NV12 rows a sub-band adds are copied HBM -> shared memory by the TMA engine
-//     (cp.async.bulk, one copy per row per frame, completion counted on one mbarrier), issued
-//     while the previous sub-band is walked (a4);
-//   * they are converted once into a per-frame ring of RGBx rows (R#11, the DPX formulation of
-//     k_stream.cuh; a5): warps take (frame, UV row) pairs, lanes take 4-pixel groups;
-//   * each thread owns four adjacent output columns of its frame for the whole band, keeps the
-//     horizontal lerps of the two current source rows in registers (parity-indexed slots, R#12,
-//     a6), mirrored for flip (a7), and emits vertical lerp, rint, normalise and 8-byte (bf16)
+// table and branch: the CTA holds FPC x NQ threads (NQ = output columns per row / (2 NP), NP
+// column pairs per thread; 4 x 112 = 448 for 224-wide outputs at NP = 1, no idle lanes) whose
+// control flow is identical, each frame with its
+// own source rows in shared memory. The band's source rows [y_first, y_last] are walked in
+// CHUNKS of CR rows (chunk boundaries at even rows, so a UV row never straddles two chunks),
+// double-buffered, with one CTA barrier per chunk:
+//   * the NV12 rows of chunk j + 2 are copied HBM -> shared memory by the TMA engine
+//     (cp.async.bulk, one copy per row per frame, completion counted on the staging buffer's
+//     mbarrier) while chunk j is walked (a4);
+//   * chunk j + 1 is converted once into RGBx rows (R#11, the DPX formulation of k_stream.cuh;
+//     a5) while chunk j is walked: each thread owns fixed (frame, 4-pixel group) slots and converts
+//     their UV rows; odd warps walk before converting, so the two phases overlap across warps;
+//   * the walk is SOURCE-ROW major: each thread owns 2 NP adjacent output columns of its frame,
+//     computes the horizontal lerps of each source row once (R#12, a6; flip mirrors the column
+//     taps, a7) into one of two register sets whose roles alternate with the row's parity
+//     (static in the unrolled code: no register copies), and emits every output row whose top
+//     tap is the previous source row: vertical lerp, rint, normalise and 4 NP-byte (bf16)
 //     stores per channel to every destination view of the item (a10, a11).
-// Row taps, ring offsets and walker actions come from a per-band table in shared memory (one
-// LDS.128 broadcast per row). Every fp32 operation is the R#12/R#17 op sequence with IEEE
-// rounding: bit-identical to the oracle. Tasks and the exact shared-memory bounds (span, ring
-// and staging rows) are computed on the host from the same fp32 tap rule (view.cpp).
+// Every fp32 operation is the R#12/R#17 op sequence with IEEE rounding: bit-identical to the
+// oracle. Tasks and the exact staged span are computed on the host from the same fp32 tap rule
+// (view.cpp).
 #pragma once
 
 namespace sand {
 namespace pl {
 
+#ifndef SAND_PLAIN_SB
+#define SAND_PLAIN_SB 0               // 1: single-buffered chunks (A/B variant)
+#endif
+constexpr int kCR = SAND_PLAIN_SB ? 8 : 6;    // source rows per chunk (even)
+constexpr int kRawRows = kCR + kCR / 2 + 1;   // staging rows per chunk: Y rows + their UV rows
+constexpr int kConvBufs = SAND_PLAIN_SB ? 1 : 2;   // conversion buffers per frame
+
 struct Shape {        // host-chosen launch shape of one batch's plain items
   int fpc;            // frames (items of one run) per CTA
-  int nq;             // threads per frame = output column quads of the widest view
-  int S;              // output rows per sub-band
+  int nq;             // threads per frame = output columns of the widest view / (2 NP)
   int rb;             // largest band (rows of the row table)
-  int ring;           // ring capacity in source rows (>= rows any sub-band spans)
-  int raw_rows;       // staging capacity in rows (Y + UV rows any sub-band adds)
   int gw;             // row capacity in pixels (multiple of 16, >= every item's staged span)
-  uint32_t ring_magic;   // floor(2^32 / ring) + 1
 };
 
-__host__ __device__ inline size_t frame_bytes(const Shape& s) {
-  return (size_t)s.ring * s.gw * 4 + rs::a16((size_t)s.raw_rows * s.gw);
-}
+// per frame: two converted-row buffers (chunks j and j + 1) then two staging buffers
+__host__ __device__ inline size_t conv_bytes(const Shape& s) { return (size_t)kCR * s.gw * 4; }
+__host__ __device__ inline size_t raw_bytes(const Shape& s) { return rs::a16((size_t)kRawRows * s.gw); }
+__host__ __device__ inline size_t frame_bytes(const Shape& s) { return kConvBufs * conv_bytes(s) + 2 * raw_bytes(s); }
 __host__ __device__ inline size_t smem_bytes(const Shape& s) {
-  return rs::a16((size_t)s.rb * 16) + 16 + (size_t)s.fpc * frame_bytes(s);
+  return rs::a16((size_t)s.rb * 8) + 16 + (size_t)s.fpc * frame_bytes(s);
 }
 
 // task encoding (uint2, built by view.cpp): x = first item (index into the launch's items),
 // y = pl_task_y(frames, band rows, first output row) (plan_types.h)
 
-// exact quotient of small non-negative integers r / n via a float reciprocal (r < 2^16, n < 2^8)
+// exact quotient of small non-negative integers r / n via a float reciprocal (r < 2^16, n < 2^12)
 __device__ __forceinline__ int small_div(int r, float inv_n) { return (int)(((float)r + 0.5f) * inv_n); }
 
 }  // namespace pl
 
-template <int DT, int ND>
-__global__ void __launch_bounds__(224, 2) k_plain(const LaunchParams p, const uint2* __restrict__ tasks, pl::Shape sh) {
+// NP column pairs per thread (1: 2 columns, 448-thread CTAs of 14 warps; 2: 4 columns)
+template <int NP>
+struct PlainBounds {
+  static constexpr int kThreads = NP == 1 ? 448 : 224;
+  static constexpr int kMinBlocks = 2;
+};
+
+template <int DT, int ND, int NP>
+__global__ void __launch_bounds__(PlainBounds<NP>::kThreads, PlainBounds<NP>::kMinBlocks) k_plain(const LaunchParams p, const uint2* __restrict__ tasks, pl::Shape sh) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   using namespace rs;
+  using pl::kCR;
   const int tid = threadIdx.x, nthr = blockDim.x;
-  const int warp = tid >> 5, lane = tid & 31, nwarps = nthr >> 5;
+  const int warp = tid >> 5, lane = tid & 31;
   const uint2 tk = tasks[blockIdx.x];
   const int item0 = (int)tk.x;
   const int nfr = (int)(tk.y & 0xffu), nr = (int)((tk.y >> 8) & 0xfffu), Y0 = (int)(tk.y >> 20);
@@ -70,12 +87,14 @@ __global__ void __launch_bounds__(224, 2) k_plain(const LaunchParams p, const ui
 
   uint32_t s_base = (uint32_t)__cvta_generic_to_shared(smem_raw);
   asm volatile("" : "+r"(s_base));
-  const uint32_t s_tab = s_base;                                   // rb x 16 B row table
-  const uint32_t s_bar = s_tab + (uint32_t)a16((size_t)sh.rb * 16);
+  const uint32_t s_tab = s_base;                                   // rb x 8 B row table
+  const uint32_t s_bar = s_tab + (uint32_t)a16((size_t)sh.rb * 8);  // two mbarriers (staging buffers)
   const uint32_t s_fr = s_bar + 16;                                // frame f at s_fr + f * fbytes
   const uint32_t fbytes = (uint32_t)pl::frame_bytes(sh);
-  const uint32_t ring_b = (uint32_t)sh.ring * (uint32_t)sh.gw * 4u;   // raw staging after the ring
-  const uint32_t rowbytes = (uint32_t)sh.gw * 4u;                  // ring row stride
+  const uint32_t rowbytes = (uint32_t)sh.gw * 4u;                  // converted row stride
+  const uint32_t convb = (uint32_t)pl::conv_bytes(sh);             // conv buffer b at b * convb
+  const uint32_t raw_off = (uint32_t)pl::kConvBufs * convb;        // staging buffer b at raw_off + b * rawb
+  const uint32_t rawb = (uint32_t)pl::raw_bytes(sh);
   const uint32_t rawpitch = (uint32_t)sh.gw;                       // staging row stride
 
   // staged column span (monotone taps): [x16, x16 + gwi)
@@ -85,71 +104,69 @@ __global__ void __launch_bounds__(224, 2) k_plain(const LaunchParams p, const ui
   tap(sc_x, off_x, Wo - 1, lim_x, org_x, dmy, x_hi, fl);
   const int x16 = x_lo & ~15;
   const int gwi = ((x_hi + 16) & ~15) - x16;
-  const int y_first = tap0(sc_y, off_y, Y0, org_y);
   if (gwi > sh.gw) __trap();                                       // host bound violated (never)
+  // source rows of the band: y0 of its first row .. y1 of its last row (monotone taps)
+  const int y_first = tap0(sc_y, off_y, Y0, org_y);
+  int y_last;
+  tap(sc_y, off_y, Y0 + nr - 1, lim_y, org_y, dmy, y_last, fl);
+  const int ybase = y_first & ~1;                                  // chunk j: [ybase + j CR, + CR)
+  const int nchunks = (y_last - ybase) / kCR + 1;
 
   if (tid == 0) {
     st::mbar_init(s_bar, 1);
+    st::mbar_init(s_bar + 8, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
 
-  // sub-band k covers band rows [k S, min((k + 1) S, nr)); it adds source rows
-  // (y1(last row of k - 1), y1(last row of k)]
-  auto last_src = [&](int k) {
-    int a, b;
-    float l;
-    tap(sc_y, off_y, Y0 + min((k + 1) * sh.S, nr) - 1, lim_y, org_y, a, b, l);
-    return b;
-  };
-  // NV12 rows [ya, yb] (Y) and their UV rows of every frame -> staging, one bulk copy per row
-  auto stage = [&](int ya, int yb) {
+  auto chunk_lo = [&](int j) { return max(y_first, ybase + j * kCR); };
+  auto chunk_hi = [&](int j) { return min(y_last, ybase + j * kCR + kCR - 1); };
+  // chunk j's NV12 rows (Y rows, then their UV rows) of every frame -> staging buffer j & 1, one
+  // bulk copy per row, completion counted on that buffer's mbarrier (warp 0)
+  auto stage = [&](int j) {
+    const int ya = chunk_lo(j), yb = chunk_hi(j);
     const int ny = yb - ya + 1, u0 = ya >> 1, nuv = (yb >> 1) - u0 + 1, per = ny + nuv;
-    if (lane == 0) st::mbar_arrive_expect_tx(s_bar, (uint32_t)(nfr * per * gwi));
+    const uint32_t bar = s_bar + 8u * (uint32_t)(j & 1);
+    const uint32_t dst0 = s_fr + raw_off + (uint32_t)(j & 1) * rawb;
+    if (lane == 0) st::mbar_arrive_expect_tx(bar, (uint32_t)(nfr * per * gwi));
     const float inv = 1.0f / (float)per;
     for (int c = lane; c < nfr * per; c += 32) {
       const int f = pl::small_div(c, inv), r = c - f * per;
       const WorkItem& w = p.items[item0 + f];
       const uint8_t* src = p.slab + w.y_off + x16 +
                            (r < ny ? (size_t)(ya + r) * w.pitch : (size_t)w.pitch * (w.src_h + u0 + r - ny));
-      st::bulk_g2s(s_fr + (uint32_t)f * fbytes + ring_b + (uint32_t)r * rawpitch, src, (uint32_t)gwi, s_bar);
+      st::bulk_g2s(dst0 + (uint32_t)f * fbytes + (uint32_t)r * rawpitch, src, (uint32_t)gwi, bar);
     }
   };
-  const int nsub = (nr + sh.S - 1) / sh.S;
-  int ya = y_first, yb = last_src(0);
-  if (warp == 0) stage(ya, yb);
+  if (warp == 0) {
+    stage(0);
+    if (nchunks > 1) stage(1);
+  }
 
-  // row table: ring byte offsets of (y0, y1), walker action and lambda_y per band row
+  // row table: (y0 of the output row, lambda_y); lambda 0 at the bottom clamp (y1 == y0), where
+  // the row is emitted from (H(y0), H(y0)): fmaf(0, h - h, h) == h (R#12 unchanged)
   for (int r = tid; r < nr; r += nthr) {
     int y0, y1;
     float ly;
     tap(sc_y, off_y, Y0 + r, lim_y, org_y, y0, y1, ly);
-    const uint32_t s0 = st::ring_mod((uint32_t)(y0 - y_first), (uint32_t)sh.ring, sh.ring_magic);
-    const uint32_t s1 = st::ring_mod((uint32_t)(y1 - y_first), (uint32_t)sh.ring, sh.ring_magic);
-    uint32_t act = st::kActTop | st::kActBot;
-    if (r > 0) {
-      const int yp = tap0(sc_y, off_y, Y0 + r - 1, org_y);
-      act = y0 == yp ? 0u : (y0 == yp + 1 ? st::kActFlip | st::kActBot : act);
-    }
-    if (y1 == y0) {            // bottom clamp: lambda 0, the bottom set is never read
-      act &= ~st::kActBot;
-      ly = 0.f;
-    }
-    st::sts128(s_tab + 16u * (uint32_t)r, make_uint4(s0 * rowbytes, s1 * rowbytes, act, __float_as_uint(ly)));
+    if (y1 == y0) ly = 0.f;
+    asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(s_tab + 8u * (uint32_t)r), "r"((uint32_t)y0),
+                 "r"(__float_as_uint(ly))
+                 : "memory");
   }
 
-  // walker: frame f, output columns [ox, ox + 4)
+  // walker: frame f, output columns [ox, ox + 2 NP)
   const int f = tid / sh.nq;
   const int qd = tid - f * sh.nq;
-  const int ox = 4 * qd;
+  const int ox = 2 * NP * qd;
   int active = (f < nfr && ox < Wo) ? 1 : 0;
   asm volatile("" : "+r"(active));
   const int fa = min(f, nfr - 1);
-  const uint32_t ringf = s_fr + (uint32_t)fa * fbytes;
-  uint32_t ca0[2], ca1[2], cb0[2], cb1[2];
-  uint64_t lx[2];
+  const uint32_t rowsf = s_fr + (uint32_t)fa * fbytes;             // this frame's conversion buffers
+  uint32_t ca0[NP], ca1[NP], cb0[NP], cb1[NP];
+  uint64_t lx[NP];
 #pragma unroll
-  for (int j = 0; j < 2; ++j) {
+  for (int j = 0; j < NP; ++j) {
     const int oj = min(ox + 2 * j, Wo - 2);
     const int ja = flip ? Wo - 1 - oj : oj;
     const int jb = flip ? Wo - 2 - oj : oj + 1;
@@ -157,10 +174,12 @@ __global__ void __launch_bounds__(224, 2) k_plain(const LaunchParams p, const ui
     float la, lb;
     tap(sc_x, off_x, ja, lim_x, org_x, a0, a1, la);
     tap(sc_x, off_x, jb, lim_x, org_x, b0, b1, lb);
-    ca0[j] = 4u * (uint32_t)(a0 - x16);
-    ca1[j] = 4u * (uint32_t)(a1 - x16);
-    cb0[j] = 4u * (uint32_t)(b0 - x16);
-    cb1[j] = 4u * (uint32_t)(b1 - x16);
+    // shared addresses of the four taps in this frame's conversion buffer 0, row slot 0; a row
+    // is then one offset common to the whole CTA (uniform)
+    ca0[j] = rowsf + 4u * (uint32_t)(a0 - x16);
+    ca1[j] = rowsf + 4u * (uint32_t)(a1 - x16);
+    cb0[j] = rowsf + 4u * (uint32_t)(b0 - x16);
+    cb1[j] = rowsf + 4u * (uint32_t)(b1 - x16);
     lx[j] = f2::pack(__float_as_uint(la), __float_as_uint(lb));
   }
   const WorkItem wf = p.items[item0 + fa];
@@ -169,87 +188,125 @@ __global__ void __launch_bounds__(224, 2) k_plain(const LaunchParams p, const ui
   Dest dl[ND];
 #pragma unroll
   for (int d = 0; d < ND; ++d) dl[d] = make_dest(p, dests[d < nd ? d : 0], Y0, ox);
-  Row3 X[2], Y[2];
+  Row3 X[NP], Y[NP];
 #pragma unroll
-  for (int j = 0; j < 2; ++j)
+  for (int j = 0; j < NP; ++j)
 #pragma unroll
     for (int c = 0; c < 3; ++c) X[j].h[c] = Y[j].h[c] = 0ull;
-  int top = 0;
-  auto hrows = [&](Row3 (&R)[2], uint32_t rowaddr) {
+  auto hrows = [&](Row3 (&R)[NP], uint32_t rowoff) {
 #pragma unroll
-    for (int j = 0; j < 2; ++j) st::hrow_s(R[j], rowaddr, ca0[j], ca1[j], cb0[j], cb1[j], lx[j]);
+    for (int j = 0; j < NP; ++j) st::hrow_s(R[j], rowoff, ca0[j], ca1[j], cb0[j], cb1[j], lx[j]);
+  };
+  int r = 0;                               // next output row to emit
+  uint2 rt = make_uint2(0xffffffffu, 0u);  // its table entry (y0, lambda)
+  // emit every output row whose y0 is `y` from the lerps of rows y (T) and y + 1 (B)
+  auto emit_rows = [&](const Row3 (&T)[NP], const Row3 (&B)[NP], int y) {
+    while ((int)rt.x == y) {
+      if (active) st::emit_np<DT, ND, NP>(T, B, __uint_as_float(rt.y), dl, p, dests, nd, Y0 + r, ox);
+      ++r;
+      rt.x = 0xffffffffu;
+      if (r < nr) asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(rt.x), "=r"(rt.y) : "r"(s_tab + 8u * (uint32_t)r));
+    }
   };
 
-  uint32_t phase = 0;
-  bool staged = true;
-  for (int k = 0; k < nsub; ++k) {
-    if (staged) {
-      st::mbar_wait(s_bar, phase);
-      phase ^= 1u;
-    }
-    __syncthreads();                       // walk(k - 1) done: its ring rows may be overwritten
-    if (staged) {                          // convert rows [ya, yb] of every frame into the rings
-      const int ny = yb - ya + 1, u0 = ya >> 1, nuv = (yb >> 1) - u0 + 1;
-      const int q4 = gwi >> 2;
-      const float inv = 1.0f / (float)nuv;
-      for (int rr = warp; rr < nfr * nuv; rr += nwarps) {
-        const int fr = pl::small_div(rr, inv), u = rr - fr * nuv;
-        const uint32_t fbase = s_fr + (uint32_t)fr * fbytes;
-        const uint32_t raw = fbase + ring_b;
-        const int yt = 2 * (u0 + u);
-        const bool ptop = yt >= ya, pbot = yt + 1 <= yb;
-        const uint32_t st_ = st::ring_mod((uint32_t)(yt - y_first + sh.ring), (uint32_t)sh.ring, sh.ring_magic);
-        const uint32_t sb_ = st_ + 1 == (uint32_t)sh.ring ? 0u : st_ + 1;
-        const uint32_t yrow_t = raw + (uint32_t)(yt - ya) * rawpitch;
-        const uint32_t uvrow = raw + (uint32_t)(ny + u) * rawpitch;
-        const uint32_t out_t = fbase + st_ * rowbytes, out_b = fbase + sb_ * rowbytes;
-        for (int q = lane; q < q4; q += 32) {
-          const uint32_t uv = st::lds32(uvrow + 4u * q);
-          const st::Chroma3 c0 = st::chroma_at<0>(uv), c1 = st::chroma_at<16>(uv);
-          if (ptop) {
-            const uint32_t yw = st::lds32(yrow_t + 4u * q);
-            st::sts128(out_t + 16u * q, make_uint4(st::rgbx_dpx(st::byte_of<0>(yw), c0), st::rgbx_dpx(st::byte_of<1>(yw), c0),
-                                                   st::rgbx_dpx(st::byte_of<2>(yw), c1), st::rgbx_dpx(st::byte_of<3>(yw), c1)));
-          }
-          if (pbot) {
-            const uint32_t yw = st::lds32(yrow_t + rawpitch + 4u * q);
-            st::sts128(out_b + 16u * q, make_uint4(st::rgbx_dpx(st::byte_of<0>(yw), c0), st::rgbx_dpx(st::byte_of<1>(yw), c0),
-                                                   st::rgbx_dpx(st::byte_of<2>(yw), c1), st::rgbx_dpx(st::byte_of<3>(yw), c1)));
-          }
+  // conversion slots: (frame, 4-pixel group) pairs, fixed per thread for the whole task (thread t
+  // owns slots t, t + nthr, ...); a chunk converts every UV row of every slot
+  const int q4 = gwi >> 2;
+  const int n_slots = nfr * q4;
+  // chunk j: staged rows -> RGBx rows of conversion buffer j & 1, after waiting for its staging buffer
+  auto convert = [&](int j) {
+    const int ya = chunk_lo(j), yb = chunk_hi(j);
+    st::mbar_wait(s_bar + 8u * (uint32_t)(j & 1), (uint32_t)(j >> 1) & 1u);
+    const int ny = yb - ya + 1, u0 = ya >> 1, nuv = (yb >> 1) - u0 + 1;
+    const uint32_t slot0 = (uint32_t)(ybase + j * kCR);            // absolute row of slot 0
+    const uint8_t* rawb0 = smem_raw + (s_fr - s_base) + raw_off + (uint32_t)(j & 1) * rawb;
+    uint8_t* convb0 = smem_raw + (s_fr - s_base) + (uint32_t)(j & (pl::kConvBufs - 1)) * convb;
+    for (int sl = tid; sl < n_slots; sl += nthr) {
+      const int fr = sl / q4, q = sl - fr * q4;
+      const uint8_t* raw = rawb0 + (uint32_t)fr * fbytes + 4u * q;
+      uint8_t* conv = convb0 + (uint32_t)fr * fbytes + 16u * q;
+      for (int u = 0; u < nuv; ++u) {
+        const int yt = 2 * (u0 + u);                       // top Y row of this UV row
+        const uint32_t uv = *reinterpret_cast<const uint32_t*>(raw + (uint32_t)(ny + u) * rawpitch);
+        const st::Chroma3 c0 = st::chroma_at<0>(uv), c1 = st::chroma_at<16>(uv);
+        uint8_t* out = conv + ((uint32_t)yt - slot0) * rowbytes;   // row yt
+        if (yt >= ya) {
+          const uint32_t yw = *reinterpret_cast<const uint32_t*>(raw + (uint32_t)(yt - ya) * rawpitch);
+          *reinterpret_cast<uint4*>(out) = make_uint4(st::rgbx_dpx(st::byte_of<0>(yw), c0), st::rgbx_dpx(st::byte_of<1>(yw), c0),
+                                                      st::rgbx_dpx(st::byte_of<2>(yw), c1), st::rgbx_dpx(st::byte_of<3>(yw), c1));
+        }
+        if (yt + 1 <= yb) {
+          const uint32_t yw = *reinterpret_cast<const uint32_t*>(raw + (uint32_t)(yt + 1 - ya) * rawpitch);
+          *reinterpret_cast<uint4*>(out + rowbytes) =
+              make_uint4(st::rgbx_dpx(st::byte_of<0>(yw), c0), st::rgbx_dpx(st::byte_of<1>(yw), c0),
+                         st::rgbx_dpx(st::byte_of<2>(yw), c1), st::rgbx_dpx(st::byte_of<3>(yw), c1));
         }
       }
     }
-    staged = false;
-    __syncthreads();                       // rings hold every row of sub-band k; staging drained
-    if (k + 1 < nsub) {                    // stage the next sub-band's new rows
-      const int na = yb + 1, nb = last_src(k + 1);
-      if (nb >= na) {
-        if (warp == 0) {
-          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-          stage(na, nb);
-        }
-        staged = true;
-      }
-      ya = na;
-      yb = max(nb, yb);
+  };
+  // walk of chunk j: source row y's lerps go to X when (y - y_first) is even, else to Y; the
+  // output rows whose top tap is y - 1 are emitted as soon as y's lerps exist
+  auto walk = [&](int j) {
+    const int ya = chunk_lo(j), yb = chunk_hi(j);
+    uint32_t row = (uint32_t)(j & (pl::kConvBufs - 1)) * convb + (uint32_t)(ya - ybase - j * kCR) * rowbytes;   // row ya
+    int y = ya;
+    if ((y - y_first) & 1) {
+      hrows(Y, row);
+      emit_rows(X, Y, y - 1);
+      ++y;
+      row += rowbytes;
     }
-    const int r_lo = k * sh.S, r_hi = min(r_lo + sh.S, nr);
-    for (int rr = r_lo; rr < r_hi; ++rr) {
-      const uint4 rt = st::lds128(s_tab + 16u * (uint32_t)rr);
-      const uint32_t act = rt.z;
-      const float l = __uint_as_float(rt.w);
-      top ^= (act & st::kActFlip) ? 1 : 0;
-      if (top == 0) {
-        if (act & st::kActTop) hrows(X, ringf + rt.x);
-        if (act & st::kActBot) hrows(Y, ringf + rt.y);
-        if (active) st::emit_np<DT, ND, 2>(X, Y, l, dl, p, dests, nd, Y0 + rr, ox);
-      } else {
-        if (act & st::kActTop) hrows(Y, ringf + rt.x);
-        if (act & st::kActBot) hrows(X, ringf + rt.y);
-        if (active) st::emit_np<DT, ND, 2>(Y, X, l, dl, p, dests, nd, Y0 + rr, ox);
-      }
+    for (; y + 1 <= yb; y += 2) {
+      hrows(X, row);
+      emit_rows(Y, X, y - 1);
+      hrows(Y, row + rowbytes);
+      emit_rows(X, Y, y);
+      row += 2 * rowbytes;
     }
+    if (y <= yb) {
+      hrows(X, row);
+      emit_rows(Y, X, y - 1);
+    }
+  };
+
+#if SAND_PLAIN_SB
+  // single-buffered chunks: convert chunk j, barrier, stage chunk j + 1, walk chunk j
+  for (int j = 0; j < nchunks; ++j) {
+    __syncthreads();                       // walk of chunk j - 1 done: conversion buffer free
+    convert(j);
+    __syncthreads();                       // chunk j converted, its staging buffer drained
+    if (j == 0) asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(rt.x), "=r"(rt.y) : "r"(s_tab));
+    if (j + 2 < nchunks && warp == 0) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      stage(j + 2);
+    }
+    walk(j);
   }
+#else
+  convert(0);
+  __syncthreads();                         // chunk 0 converted, its staging buffer drained; table visible
+  asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(rt.x), "=r"(rt.y) : "r"(s_tab));
+  for (int j = 0; j < nchunks; ++j) {
+    // staging buffer j & 1 was drained by convert(j) before the last barrier: chunk j + 2 may land
+    if (j + 2 < nchunks && warp == 0) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      stage(j + 2);
+    }
+    // convert chunk j + 1 (buffer (j + 1) & 1, last read by the walk of chunk j - 1 before the
+    // barrier) and walk chunk j; odd warps walk first, so the CTA's warps overlap the two phases
+    for (int ph = 0; ph < 2; ++ph) {
+      if (((ph ^ warp) & 1) == 0) {
+        if (j + 1 < nchunks) convert(j + 1);
+      } else {
+        walk(j);
+      }
+    }
+    __syncthreads();
+  }
+#endif
+  // rows at the bottom clamp (y0 == y1 == y_last, lambda 0): emitted from H(y_last) twice
+  if ((y_last - y_first) & 1) emit_rows(Y, Y, y_last);
+  else emit_rows(X, X, y_last);
 }
 
 }  // namespace sand

@@ -238,13 +238,15 @@ constexpr uint32_t kActFlip = 4;   // y0 = previous y0 + 1: the old bottom set b
 // At the bottom edge (y1 == y0) the bottom set is not computed and lambda_y is stored as 0:
 // fmaf(0, b - h0, h0) == h0 == fmaf(lambda, h0 - h0, h0) for any finite b (R#12 unchanged).
 
-// Vertical lerp + rint + stores of one output row for NP column pairs (R#12, R#17), NP = 2:
-// four adjacent columns, one 8 B (bf16) / 16 B (f32) / 4 B (u8) store per channel and
-// destination. Requires out_w % 4 == 0 for every view (host-checked), so the stores are aligned.
+// Vertical lerp + rint + stores of one output row for NP (1 or 2) column pairs (R#12, R#17):
+// 2 NP adjacent columns, one 4 NP-byte (bf16) / 8 NP-byte (f32) / 2 NP-byte (u8) store per
+// channel and destination. Requires out_w % (2 NP) == 0 for every view (host-checked), so the
+// stores are aligned.
 template <int DT, int ND, int NP>
 __device__ __forceinline__ void emit_np(const rs::Row3 (&top)[NP], const rs::Row3 (&bot)[NP], float l,
                                         rs::Dest (&dl)[ND], const LaunchParams& p, const uint32_t* __restrict__ dests,
                                         int nd, int oy, int ox) {
+  static_assert(NP == 1 || NP == 2, "one or two column pairs");
   using namespace rs;
   const uint64_t ly = f2::splat(l);
   uint64_t q[NP][3], tq[NP][3];
@@ -262,18 +264,28 @@ __device__ __forceinline__ void emit_np(const rs::Row3 (&top)[NP], const rs::Row
       uint8_t* o = d.row + (size_t)c * d.cstride;
       if (DT == SAND_U8) {
         const uint32_t p0 = __byte_perm(f2::lo(tq[0][c]), f2::hi(tq[0][c]), 0x0040);
-        const uint32_t p1 = __byte_perm(f2::lo(tq[1][c]), f2::hi(tq[1][c]), 0x0040);
-        *reinterpret_cast<uint32_t*>(o) = __byte_perm(p0, p1, 0x5410);
+        if constexpr (NP == 2) {
+          const uint32_t p1 = __byte_perm(f2::lo(tq[1][c]), f2::hi(tq[1][c]), 0x0040);
+          *reinterpret_cast<uint32_t*>(o) = __byte_perm(p0, p1, 0x5410);
+        } else {
+          *reinterpret_cast<uint16_t*>(o) = (uint16_t)p0;
+        }
       } else {
         const uint64_t a = f2::splat(d.a[c]), b = f2::splat(d.b[c]);
-        const uint64_t y0 = f2::fma(q[0][c], a, b), y1 = f2::fma(q[1][c], a, b);   // fmaf(q, a_c, b_c)
-        if (DT == SAND_BF16) {
-          const __nv_bfloat162 v0 = __floats2bfloat162_rn(f2::lof(y0), f2::hif(y0));
-          const __nv_bfloat162 v1 = __floats2bfloat162_rn(f2::lof(y1), f2::hif(y1));
-          *reinterpret_cast<uint2*>(o) =
-              make_uint2(*reinterpret_cast<const uint32_t*>(&v0), *reinterpret_cast<const uint32_t*>(&v1));
+        const uint64_t y0 = f2::fma(q[0][c], a, b);                               // fmaf(q, a_c, b_c)
+        if constexpr (NP == 2) {
+          const uint64_t y1 = f2::fma(q[1][c], a, b);
+          if (DT == SAND_BF16) {
+            const __nv_bfloat162 v0 = __floats2bfloat162_rn(f2::lof(y0), f2::hif(y0));
+            const __nv_bfloat162 v1 = __floats2bfloat162_rn(f2::lof(y1), f2::hif(y1));
+            *reinterpret_cast<uint2*>(o) =
+                make_uint2(*reinterpret_cast<const uint32_t*>(&v0), *reinterpret_cast<const uint32_t*>(&v1));
+          } else {
+            *reinterpret_cast<uint4*>(o) = make_uint4(f2::lo(y0), f2::hi(y0), f2::lo(y1), f2::hi(y1));
+          }
         } else {
-          *reinterpret_cast<uint4*>(o) = make_uint4(f2::lo(y0), f2::hi(y0), f2::lo(y1), f2::hi(y1));
+          if (DT == SAND_BF16) *reinterpret_cast<__nv_bfloat162*>(o) = __floats2bfloat162_rn(f2::lof(y0), f2::hif(y0));
+          else *reinterpret_cast<uint64_t*>(o) = y0;
         }
       }
     }

@@ -26,6 +26,9 @@ int configure_stencil();
 // SAND_OK with *launched = false when the batch does not fit k_plain (mixed dtypes, widths not a
 // multiple of 4, shared memory); the caller then takes the generic kernel.
 int launch_plain(const LaunchParams& p, const BatchShape& sh, int fpc, int nq, cudaStream_t stream, bool* launched);
+// k_plain's output columns per thread and largest CTA (the view sizes its tasks from them)
+int plain_cols_per_thread();
+int plain_max_threads();
 
 // mat_stream.cu — identity-scale copy kernel (k_copy; *launched = false if not applicable) and
 // the generic streaming kernel (k_stream, any dtype mix / width) over mild items p.items[0, n)

@@ -4,44 +4,48 @@
 
 namespace sand {
 
+#ifndef SAND_PLAIN_NP
+#define SAND_PLAIN_NP 2       // column pairs per thread (k_plain.cuh)
+#endif
+constexpr int kNP = SAND_PLAIN_NP;
+
+int plain_cols_per_thread() { return 2 * kNP; }
+int plain_max_threads() { return PlainBounds<kNP>::kThreads; }
+
 int configure_plain() {
-  for (cudaError_t e : {allow_smem(k_plain<SAND_U8, 1>), allow_smem(k_plain<SAND_BF16, 1>),
-                        allow_smem(k_plain<SAND_F32, 1>), allow_smem(k_plain<SAND_U8, 2>),
-                        allow_smem(k_plain<SAND_BF16, 2>), allow_smem(k_plain<SAND_F32, 2>)})
+  for (cudaError_t e : {allow_smem(k_plain<SAND_U8, 1, kNP>), allow_smem(k_plain<SAND_BF16, 1, kNP>),
+                        allow_smem(k_plain<SAND_F32, 1, kNP>), allow_smem(k_plain<SAND_U8, 2, kNP>),
+                        allow_smem(k_plain<SAND_BF16, 2, kNP>), allow_smem(k_plain<SAND_F32, 2, kNP>)})
     if (e != cudaSuccess) return cuda_error(e, "cudaFuncSetAttribute(k_plain)");
   return SAND_OK;
 }
 
 int launch_plain(const LaunchParams& p, const BatchShape& sh, int fpc, int nq, cudaStream_t stream, bool* launched) {
   *launched = false;
-  if (sh.n_tasks == 0 || !sh.wo_mod4 || sh.dtype < 0) return SAND_OK;
+  if (sh.n_tasks == 0 || sh.dtype < 0 || (kNP == 2 ? !sh.wo_mod4 : !sh.even_wo)) return SAND_OK;
   pl::Shape s;
   s.fpc = fpc;
   s.nq = nq;
-  s.S = kPlainS;
   s.rb = sh.pl_rb;
-  s.ring = sh.pl_ring;
-  s.raw_rows = sh.pl_raw;
   s.gw = sh.pl_gw;
-  s.ring_magic = (uint32_t)((1ull << 32) / (uint64_t)s.ring + 1);
   const size_t smem = pl::smem_bytes(s);
-  if (smem > 200 * 1024 || s.ring > 255) return SAND_OK;       // pathological shapes: generic kernel
+  if (smem > 200 * 1024) return SAND_OK;                         // pathological widths: generic kernel
   const unsigned threads = (unsigned)((fpc * nq + 31) / 32 * 32);
-  if (threads > 224) return SAND_OK;                             // outputs wider than 896: generic kernel
+  if (threads > (unsigned)PlainBounds<kNP>::kThreads) return SAND_OK;   // very wide outputs: generic kernel
   const uint2* tasks = p.tasks + sh.task_first;
   const bool nd1 = sh.max_dests <= 1;
   switch (sh.dtype) {
     case SAND_U8:
-      if (nd1) k_plain<SAND_U8, 1><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
-      else k_plain<SAND_U8, 2><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
+      if (nd1) k_plain<SAND_U8, 1, kNP><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
+      else k_plain<SAND_U8, 2, kNP><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
       break;
     case SAND_BF16:
-      if (nd1) k_plain<SAND_BF16, 1><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
-      else k_plain<SAND_BF16, 2><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
+      if (nd1) k_plain<SAND_BF16, 1, kNP><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
+      else k_plain<SAND_BF16, 2, kNP><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
       break;
     default:
-      if (nd1) k_plain<SAND_F32, 1><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
-      else k_plain<SAND_F32, 2><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
+      if (nd1) k_plain<SAND_F32, 1, kNP><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
+      else k_plain<SAND_F32, 2, kNP><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
       break;
   }
   cudaError_t e = cudaGetLastError();

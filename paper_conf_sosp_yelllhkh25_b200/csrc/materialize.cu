@@ -24,7 +24,13 @@ int configure_kernels(size_t stencil_smem) {
 }
 
 int launch_materialize(const LaunchParams& p, const BatchShape& shape, size_t stencil_smem, int pl_fpc, int pl_nq,
-                       cudaStream_t stream, cudaStream_t aux, cudaEvent_t fork, cudaEvent_t join, int* n_launched) {
+                       cudaStream_t stream, cudaStream_t aux, cudaEvent_t fork, cudaEvent_t join, int* n_launched,
+                       ClassEvents* ev) {
+  auto mark = [&](int cls, bool end, cudaStream_t s) {
+    if (!ev) return cudaSuccess;
+    if (end) ev->used[cls] = true;
+    return cudaEventRecord(end ? ev->end[cls] : ev->start[cls], s);
+  };
   *n_launched = 0;
   if (p.n_items == 0) return SAND_OK;
   const uint32_t n_mild = shape.n_mild, n_heavy = shape.n_direct - shape.n_mild;
@@ -43,16 +49,21 @@ int launch_materialize(const LaunchParams& p, const BatchShape& shape, size_t st
     LaunchParams ps = p;
     ps.items = p.items + shape.n_direct;
     ps.n_items = n_stencil;
+    mark(2, false, stream);
     const int rc = launch_stencil(ps, shape, stencil_smem, stream);
     if (rc != SAND_OK) return rc;
+    mark(2, true, stream);
     ++*n_launched;
   }
   if (n_heavy > 0) {
     LaunchParams ph = p;
     ph.items = p.items + n_mild;
     ph.n_items = n_heavy;
-    const int rc = launch_direct(ph, shape, n_stencil > 0 ? side : stream);
+    cudaStream_t s = n_stencil > 0 ? side : stream;
+    mark(1, false, s);
+    const int rc = launch_direct(ph, shape, s);
     if (rc != SAND_OK) return rc;
+    mark(1, true, s);
     ++*n_launched;
   }
   if (n_mild > 0) {
@@ -60,10 +71,12 @@ int launch_materialize(const LaunchParams& p, const BatchShape& shape, size_t st
     pm.n_items = n_mild;
     cudaStream_t s = (n_stencil > 0 || n_heavy > 0) ? side : stream;
     bool done = false;
+    mark(0, false, s);
     int rc = launch_copy(pm, shape, s, &done);
     if (rc == SAND_OK && !done) rc = launch_plain(pm, shape, pl_fpc, pl_nq, s, &done);
     if (rc == SAND_OK && !done) rc = launch_stream_generic(pm, shape, s);
     if (rc != SAND_OK) return rc;
+    mark(0, true, s);
     ++*n_launched;
   }
   if (fork_ok) {

@@ -81,13 +81,12 @@ struct BatchShape {
   uint32_t n_mild;
   int32_t max_dests;        // largest destination count of a direct item
   int32_t heavy_max_wo, heavy_max_ho;
-  // k_plain: the batch's task slice and exact shared-memory bounds over its tasks
+  // k_plain: the batch's task slice, the widest staged span (pixels) and the longest band
   uint32_t task_first, n_tasks;
-  int32_t pl_gw, pl_ring, pl_raw, pl_rb;
+  int32_t pl_gw, pl_rb;
 };
 
 // k_plain task granularity (view.cpp builds the tasks, k_plain.cuh consumes them)
-constexpr int kPlainS = 4;         // output rows per sub-band
 constexpr int kPlainRB = 32;       // output rows per band
 constexpr int kPlainRBTail = 8;    // band of the tasks that make up the last part of the work
 constexpr double kPlainTailFrac = 0.25;

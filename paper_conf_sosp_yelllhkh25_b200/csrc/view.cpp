@@ -16,6 +16,7 @@
 #include <cstring>
 
 #include "internal.h"
+#include "kernels.h"
 
 namespace sand {
 namespace {
@@ -102,29 +103,14 @@ int row_tap1(const GroupParams& g, int o) {
   return b;
 }
 
-// k_plain shared-memory needs of one band [y0, y0 + nr) of a group, walked in sub-bands of
-// kPlainS rows exactly as the kernel does: ring rows live at once and staged rows per sub-band
-void plain_band_bounds(const GroupParams& g, int y0, int nr, int* ring, int* raw, int* conv_rows) {
-  *ring = 0;
-  *raw = 0;
-  int ya = row_tap0(g, y0), yb = -1;
-  const int first = ya;
-  for (int k = 0; k * kPlainS < nr; ++k) {
-    const int r_lo = k * kPlainS, r_hi = std::min(nr, r_lo + kPlainS) - 1;
-    const int last = row_tap1(g, y0 + r_hi);
-    *ring = std::max(*ring, last - row_tap0(g, y0 + r_lo) + 1);
-    const int na = k == 0 ? ya : yb + 1;
-    if (last >= na) *raw = std::max(*raw, (last - na + 1) + ((last >> 1) - (na >> 1) + 1));
-    yb = std::max(yb, last);
-  }
-  *conv_rows = yb - first + 1;
-}
+// source rows a k_plain band [y0, y0 + nr) of a group converts (its cost model)
+int plain_band_rows(const GroupParams& g, int y0, int nr) { return row_tap1(g, y0 + nr - 1) - row_tap0(g, y0) + 1; }
 
 // k_plain tasks of one batch's mild items [0, n) (ordered by clip slot, group, frame): runs of
 // one (clip slot, group) in chunks of `fpc` frames x bands of kPlainRB rows; the costliest first
 // (the block scheduler then approximates longest-processing-time order), and the cheapest
 // quarter of the work split into kPlainRBTail-row bands so the grid's last wave is short.
-// Also returns the exact shared-memory bounds over the tasks.
+// Also returns the widest staged span and the longest band over the tasks.
 void plain_tasks(const std::vector<WorkItem>& items, size_t first, size_t n, const std::vector<GroupParams>& groups,
                  int fpc, std::vector<uint2>* out, BatchShape* shape) {
   struct T {
@@ -133,8 +119,7 @@ void plain_tasks(const std::vector<WorkItem>& items, size_t first, size_t n, con
   };
   std::vector<T> ts;
   auto cost_of = [&](const GroupParams& g, uint32_t nfr, int y0, int nr) {
-    int ring, raw, conv;
-    plain_band_bounds(g, y0, nr, &ring, &raw, &conv);
+    const int conv = plain_band_rows(g, y0, nr);
     // lane instructions: ~4.4 per converted channel value, ~8 per output value
     return (double)nfr * (4.4 * 3.0 * conv * span16(g) + 8.0 * 3.0 * nr * g.out_w);
   };
@@ -173,14 +158,10 @@ void plain_tasks(const std::vector<WorkItem>& items, size_t first, size_t n, con
   std::reverse(big.begin(), big.end());
   std::stable_sort(tail.begin(), tail.end(), [](const T& a, const T& b) { return a.cost > b.cost; });
   shape->task_first = (uint32_t)out->size();
-  shape->pl_gw = shape->pl_ring = shape->pl_raw = shape->pl_rb = 0;
+  shape->pl_gw = shape->pl_rb = 0;
   for (const auto* v : {&big, &tail})
     for (const T& t : *v) {
       const GroupParams& g = groups[items[first + t.item].gp];
-      int ring, raw, conv;
-      plain_band_bounds(g, (int)t.y0, (int)t.nr, &ring, &raw, &conv);
-      shape->pl_ring = std::max(shape->pl_ring, ring);
-      shape->pl_raw = std::max(shape->pl_raw, raw);
       shape->pl_gw = std::max(shape->pl_gw, span16(g));
       shape->pl_rb = std::max(shape->pl_rb, (int)t.nr);
       out->push_back(make_uint2(t.item, pl_task_y(t.nfr, t.nr, t.y0)));
@@ -671,11 +652,12 @@ extern "C" int sand_view_create(sand_store* s, const sand_view_spec* spec, sand_
     return sand::cuda_error(e, "cudaSetDevice");
   }
   v->stencil_smem = stencil ? sand::stencil_smem_bytes(max_h, max_w, max_r) : 0;
-  {   // k_plain CTA: frames of one clip group side by side, NQ = column quads of the widest view
+  {   // k_plain CTA: frames of one clip group side by side, NQ threads per frame row
     uint32_t wmax = 4;
     for (uint32_t k = 0; k < spec->n_views; ++k) wmax = std::max(wmax, spec->views[k].out_w);
-    v->pl_nq = static_cast<int>((wmax + 3) / 4);
-    v->pl_fpc = std::max(1, std::min(8, 224 / v->pl_nq));   // <= 224 threads (k_plain launch bounds)
+    const int cpt = sand::plain_cols_per_thread();
+    v->pl_nq = static_cast<int>((wmax + cpt - 1) / cpt);
+    v->pl_fpc = std::max(1, std::min(8, sand::plain_max_threads() / v->pl_nq));
   }
   rc = sand::configure_kernels(v->stencil_smem);
   if (rc != SAND_OK) {
@@ -726,7 +708,171 @@ extern "C" int sand_view_prefetch_epoch(sand_view* v, uint64_t epoch, uint32_t r
   return SAND_OK;
 }
 
+static int read_batch_direct(sand_view* v, uint64_t epoch, uint32_t rank, const sand_batch_out* out);
+
+namespace sand {
+namespace {
+// the pre-materialised slot holding (epoch, rank, iteration), or -1 (caller holds v->mu)
+int find_slot(const sand_view* v, uint64_t epoch, uint32_t rank, uint64_t it) {
+  for (size_t i = 0; i < v->pre.size(); ++i) {
+    const auto& sl = v->pre[i];
+    if (sl.busy && sl.epoch == epoch && sl.rank == rank && sl.iteration == it) return static_cast<int>(i);
+  }
+  return -1;
+}
+void free_slots(sand_view* v) {
+  for (auto& sl : v->pre) {
+    if (sl.done) {
+      cudaEventSynchronize(sl.done);
+      cudaEventDestroy(sl.done);
+    }
+    if (sl.consumed) {
+      cudaEventSynchronize(sl.consumed);
+      cudaEventDestroy(sl.consumed);
+    }
+    cudaFree(sl.buf);
+  }
+  v->pre.clear();
+}
+}  // namespace
+}  // namespace sand
+
+extern "C" int sand_view_set_prematerialize(sand_view* v, uint32_t slots) {
+  if (!v) return sand::set_error(SAND_EINVAL, "null argument");
+  std::lock_guard<std::mutex> lk(v->mu);
+  cudaError_t e = cudaSetDevice(v->store->device);
+  if (e != cudaSuccess) return sand::cuda_error(e, "cudaSetDevice");
+  sand::free_slots(v);
+  if (slots == 0) return SAND_OK;
+  if (!v->pre_stream) {
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);   // lo = least priority
+    e = cudaStreamCreateWithPriority(&v->pre_stream, cudaStreamNonBlocking, lo);
+    if (e != cudaSuccess) return sand::cuda_error(e, "cudaStreamCreateWithPriority(prematerialize)");
+  }
+  size_t total = 0;
+  for (uint32_t k = 0; k < v->info.spec.n_views; ++k) {
+    sand_tensor_desc td;
+    sand_view_output_desc(v, k, &td);
+    v->pre_view_off[k] = total;
+    v->pre_view_bytes[k] = td.bytes;
+    total += (td.bytes + 255) / 256 * 256;
+  }
+  v->pre.resize(slots);
+  for (auto& sl : v->pre) {
+    e = cudaMalloc(&sl.buf, total);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&sl.done, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&sl.consumed, cudaEventDisableTiming);
+    if (e != cudaSuccess) {
+      sand::free_slots(v);
+      return sand::cuda_error(e, "pre-materialisation buffers");
+    }
+  }
+  return SAND_OK;
+}
+
+extern "C" int sand_view_prematerialize(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration) {
+  if (!v) return sand::set_error(SAND_EINVAL, "null argument");
+  sand_batch_out out{};
+  int slot = -1;
+  {
+    std::lock_guard<std::mutex> lk(v->mu);
+    if (v->pre.empty()) return sand::set_error(SAND_EINVAL, "pre-materialisation not configured");
+    if (sand::find_slot(v, epoch, rank, iteration) >= 0) return SAND_OK;   // already under way
+    for (size_t i = 0; i < v->pre.size(); ++i)
+      if (!v->pre[i].busy) {
+        slot = static_cast<int>(i);
+        break;
+      }
+    if (slot < 0) return sand::set_error(SAND_EBUSY, "every pre-materialisation slot holds an unread batch");
+    auto& sl = v->pre[slot];
+    // the slot's previous batch may still be being copied out / used by its reader
+    if (sl.consumed_pending) {
+      cudaError_t e = cudaStreamWaitEvent(v->pre_stream, sl.consumed, 0);
+      if (e != cudaSuccess) return sand::cuda_error(e, "cudaStreamWaitEvent(slot consumed)");
+      sl.consumed_pending = false;
+    }
+    out.iteration = iteration;
+    out.stream = v->pre_stream;
+    for (uint32_t k = 0; k < v->info.spec.n_views; ++k) out.data[k] = sl.buf + v->pre_view_off[k];
+    sl.busy = true;   // reserved while the kernels are enqueued
+    sl.epoch = epoch;
+    sl.rank = rank;
+    sl.iteration = iteration;
+  }
+  const int rc = read_batch_direct(v, epoch, rank, &out);
+  std::lock_guard<std::mutex> lk(v->mu);
+  auto& sl = v->pre[slot];
+  if (rc != SAND_OK) {
+    sl.busy = false;
+    return rc;
+  }
+  cudaError_t e = cudaEventRecord(sl.done, v->pre_stream);
+  if (e != cudaSuccess) {
+    sl.busy = false;
+    return sand::cuda_error(e, "cudaEventRecord(prematerialized)");
+  }
+  v->pre_made++;
+  return SAND_OK;
+}
+
+extern "C" int sand_view_acquire_batch(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration,
+                                       sand_stream_t stream, void* data_out[SAND_MAX_VIEWS]) {
+  if (!v || !data_out) return sand::set_error(SAND_EINVAL, "null argument");
+  std::lock_guard<std::mutex> lk(v->mu);
+  const int i = sand::find_slot(v, epoch, rank, iteration);
+  if (i < 0 || v->pre[i].acquired) return sand::set_error(SAND_ERANGE, "batch is not pre-materialised");
+  auto& sl = v->pre[i];
+  cudaError_t e = cudaStreamWaitEvent(static_cast<cudaStream_t>(stream), sl.done, 0);
+  if (e != cudaSuccess) return sand::cuda_error(e, "cudaStreamWaitEvent(prematerialized)");
+  for (uint32_t k = 0; k < SAND_MAX_VIEWS; ++k)
+    data_out[k] = k < v->info.spec.n_views ? static_cast<void*>(sl.buf + v->pre_view_off[k]) : nullptr;
+  sl.acquired = true;
+  v->pre_served++;
+  return SAND_OK;
+}
+
+extern "C" int sand_view_release_batch(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration,
+                                       sand_stream_t stream) {
+  if (!v) return sand::set_error(SAND_EINVAL, "null argument");
+  std::lock_guard<std::mutex> lk(v->mu);
+  const int i = sand::find_slot(v, epoch, rank, iteration);
+  if (i < 0 || !v->pre[i].acquired) return sand::set_error(SAND_ERANGE, "batch was not acquired");
+  auto& sl = v->pre[i];
+  cudaError_t e = cudaEventRecord(sl.consumed, static_cast<cudaStream_t>(stream));
+  if (e != cudaSuccess) return sand::cuda_error(e, "cudaEventRecord(slot consumed)");
+  sl.consumed_pending = true;
+  sl.acquired = false;
+  sl.busy = false;
+  return SAND_OK;
+}
+
 extern "C" int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank, const sand_batch_out* out) {
+  if (!v || !out) return sand::set_error(SAND_EINVAL, "null argument");
+  {   // a pre-materialised batch: wait for it and copy it out (stream-ordered)
+    std::lock_guard<std::mutex> lk(v->mu);
+    const int i = v->pre.empty() ? -1 : sand::find_slot(v, epoch, rank, out->iteration);
+    if (i >= 0 && !v->pre[i].acquired) {
+      auto& sl = v->pre[i];
+      auto stream = static_cast<cudaStream_t>(out->stream);
+      cudaError_t e = cudaStreamWaitEvent(stream, sl.done, 0);
+      for (uint32_t k = 0; k < v->info.spec.n_views && e == cudaSuccess; ++k) {
+        if (!out->data[k]) return sand::set_error(SAND_EINVAL, "null output pointer");
+        e = cudaMemcpyAsync(out->data[k], sl.buf + v->pre_view_off[k], v->pre_view_bytes[k], cudaMemcpyDeviceToDevice,
+                            stream);
+      }
+      if (e == cudaSuccess) e = cudaEventRecord(sl.consumed, stream);
+      if (e != cudaSuccess) return sand::cuda_error(e, "serving a pre-materialised batch");
+      sl.consumed_pending = true;
+      sl.busy = false;
+      v->pre_served++;
+      return SAND_OK;
+    }
+  }
+  return read_batch_direct(v, epoch, rank, out);
+}
+
+static int read_batch_direct(sand_view* v, uint64_t epoch, uint32_t rank, const sand_batch_out* out) {
   if (!v || !out) return sand::set_error(SAND_EINVAL, "null argument");
   const sand_view_spec& s = v->info.spec;
   if (rank >= s.world_size) return sand::set_error(SAND_EINVAL, "rank >= world_size");
@@ -828,8 +974,30 @@ extern "C" int sand_view_read_batch(sand_view* v, uint64_t epoch, uint32_t rank,
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&v->join_ev, cudaEventDisableTiming);
     if (e != cudaSuccess) return sand::cuda_error(e, "aux stream for the direct kernel");
   }
+  sand::ClassEvents cev{};
+  if (v->timing) {   // measurement only: an event pair per class from the view's pool
+    for (int c = 0; c < 3; ++c)
+      for (cudaEvent_t* ev : {&cev.start[c], &cev.end[c]}) {
+        if (v->free_events.empty()) {
+          e = cudaEventCreate(ev);
+          if (e != cudaSuccess) return sand::cuda_error(e, "cudaEventCreate(timing)");
+        } else {
+          *ev = v->free_events.back();
+          v->free_events.pop_back();
+        }
+      }
+  }
   int rc = sand::launch_materialize(lp, bshape, v->stencil_smem, v->pl_fpc, v->pl_nq, stream, v->aux_stream, v->fork_ev,
-                                    v->join_ev, &launched);
+                                    v->join_ev, &launched, v->timing ? &cev : nullptr);
+  if (v->timing)
+    for (int c = 0; c < 3; ++c) {
+      if (cev.used[c] && rc == SAND_OK) {
+        v->timed.push_back({c, cev.start[c], cev.end[c]});
+      } else {
+        v->free_events.push_back(cev.start[c]);
+        v->free_events.push_back(cev.end[c]);
+      }
+    }
   if (rc != SAND_OK) return rc;
   e = cudaEventRecord(plan->last_use, stream);
   if (e == cudaSuccess) e = cudaEventRecord(v->inflight[slot], stream);
@@ -866,25 +1034,36 @@ extern "C" int sand_view_get_meta(sand_view* v, uint64_t epoch, uint32_t rank, u
 // source rows touched by any bilinear tap, deduplicated across views, groups and
 // clips that share a (video, frame); rows assumed 32 B aligned (the store's pitch
 // is a multiple of 64 B). Taps follow the same fp32 coordinate rule as the kernel.
-extern "C" int sand_view_batch_bytes(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration,
-                                     sand_batch_bytes* out) {
+// cls < 0: every item; else only the items of that class (SAND_N_CLASSES).
+static int batch_bytes_impl(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration, int cls,
+                            sand_batch_bytes* out) {
   if (!v || !out) return sand::set_error(SAND_EINVAL, "null argument");
   if (rank >= v->info.spec.world_size) return sand::set_error(SAND_EINVAL, "rank >= world_size");
+  if (cls >= SAND_N_CLASSES) return sand::set_error(SAND_EINVAL, "class out of range");
   std::unique_lock<std::mutex> lk(v->mu);
   auto plan = sand::get_plan(v, lk, epoch, rank);
   lk.unlock();
   if (iteration >= plan->iterations) return sand::set_error(SAND_ERANGE, "iteration out of range");
   const sand_view_spec& s = v->info.spec;
   std::memset(out, 0, sizeof(*out));
-  for (uint32_t k = 0; k < s.n_views; ++k) {
-    sand_tensor_desc td;
-    sand_view_output_desc(v, k, &td);
-    out->out_bytes += td.bytes;
-  }
-  // group items by source frame
+  const uint32_t ib = plan->item_begin[iteration], ie = plan->item_begin[iteration + 1];
+  const sand::BatchShape& shape = plan->shapes[iteration];
+  auto class_of = [&](uint32_t i) {
+    const uint32_t r = i - ib;
+    return r < shape.n_mild ? 0 : (r < shape.n_direct ? 1 : 2);
+  };
+  // group the selected items by source frame; output bytes and uses from their destinations
   std::map<uint64_t, std::vector<uint32_t>> by_frame;
-  for (uint32_t i = plan->item_begin[iteration]; i < plan->item_begin[iteration + 1]; ++i)
-    by_frame[plan->items[i].y_off].push_back(i);
+  for (uint32_t i = ib; i < ie; ++i) {
+    if (cls >= 0 && class_of(i) != cls) continue;
+    const sand::WorkItem& w = plan->items[i];
+    by_frame[w.y_off].push_back(i);
+    for (uint32_t d = 0; d < w.n_dest; ++d) {
+      const sand_view_desc& vd = s.views[plan->dests[w.dest_begin + d] >> 24];
+      out->out_bytes += 3ull * vd.out_h * vd.out_w * sand::dtype_bytes(vd.out_dtype);
+    }
+    out->uses += w.n_dest;
+  }
   for (auto& kv : by_frame) {
     const sand::WorkItem& w0 = plan->items[kv.second[0]];
     const uint32_t W = w0.src_w, H = w0.src_h, nsec = (W + 31) / 32;
@@ -893,11 +1072,11 @@ extern "C" int sand_view_batch_bytes(sand_view* v, uint64_t epoch, uint32_t rank
       const sand::GroupParams& g = plan->groups[plan->items[i].gp];
       auto taps = [](float sc, int off, int n_out, int lim, int org, std::vector<uint8_t>& mark) {
         for (int o = 0; o < n_out; ++o) {
-          const float sv = std::max(sc * (static_cast<float>(off + o) + 0.5f) - 0.5f, 0.0f);
-          const int i0 = static_cast<int>(sv);
-          const int i1 = std::min(i0 + 1, lim - 1);
-          mark[org + i0] = 1;
-          mark[org + i1] = 1;
+          int i0, i1;
+          float l;
+          sand::tap_ref(sc, off, o, lim, org, &i0, &i1, &l);
+          mark[i0] = 1;
+          mark[i1] = 1;
         }
       };
       std::vector<uint8_t> cols(W, 0), rows(H, 0);
@@ -921,9 +1100,55 @@ extern "C" int sand_view_batch_bytes(sand_view* v, uint64_t epoch, uint32_t rank
     for (uint8_t b : uvsec) out->src_sectors += b;
   }
   out->src_bytes = out->src_sectors * 32;
-  for (uint32_t i = plan->fetch_begin[iteration]; i < plan->fetch_begin[iteration + 1]; ++i) {
-    out->fetches += 1;
-    out->uses += plan->fetch_uses[i];
+  if (cls < 0) {
+    for (uint32_t i = plan->fetch_begin[iteration]; i < plan->fetch_begin[iteration + 1]; ++i) out->fetches += 1;
+  } else {
+    std::map<uint64_t, int> frames;
+    for (const auto& kv : by_frame) frames[kv.first] = 1;
+    out->fetches = frames.size();
+  }
+  return SAND_OK;
+}
+
+extern "C" int sand_view_batch_bytes(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration,
+                                     sand_batch_bytes* out) {
+  return batch_bytes_impl(v, epoch, rank, iteration, -1, out);
+}
+
+extern "C" int sand_view_batch_bytes_class(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration, uint32_t cls,
+                                           sand_batch_bytes* out) {
+  if (cls >= SAND_N_CLASSES) return sand::set_error(SAND_EINVAL, "class out of range");
+  return batch_bytes_impl(v, epoch, rank, iteration, static_cast<int>(cls), out);
+}
+
+extern "C" int sand_view_set_timing(sand_view* v, int on) {
+  if (!v) return sand::set_error(SAND_EINVAL, "null argument");
+  std::lock_guard<std::mutex> lk(v->mu);
+  v->timing = on != 0;
+  return SAND_OK;
+}
+
+extern "C" int sand_view_class_times(sand_view* v, double ms[SAND_N_CLASSES], uint64_t launches[SAND_N_CLASSES]) {
+  if (!v || !ms || !launches) return sand::set_error(SAND_EINVAL, "null argument");
+  std::lock_guard<std::mutex> lk(v->mu);
+  cudaError_t e = cudaSetDevice(v->store->device);
+  if (e != cudaSuccess) return sand::cuda_error(e, "cudaSetDevice");
+  for (const auto& t : v->timed) {
+    e = cudaEventSynchronize(t.end);
+    float x = 0.f;
+    if (e == cudaSuccess) e = cudaEventElapsedTime(&x, t.start, t.end);
+    if (e != cudaSuccess) return sand::cuda_error(e, "class timing events");
+    v->class_ms[t.cls] += x;
+    v->class_launches[t.cls] += 1;
+    v->free_events.push_back(t.start);
+    v->free_events.push_back(t.end);
+  }
+  v->timed.clear();
+  for (int c = 0; c < SAND_N_CLASSES; ++c) {
+    ms[c] = v->class_ms[c];
+    launches[c] = v->class_launches[c];
+    v->class_ms[c] = 0;
+    v->class_launches[c] = 0;
   }
   return SAND_OK;
 }
@@ -962,6 +1187,13 @@ extern "C" int sand_view_destroy(sand_view* v) {
   if (v->join_ev) cudaEventDestroy(v->join_ev);
   for (auto& ev : v->inflight)
     if (ev) cudaEventDestroy(ev);
+  for (auto& t : v->timed) {
+    cudaEventDestroy(t.start);
+    cudaEventDestroy(t.end);
+  }
+  for (auto& ev : v->free_events) cudaEventDestroy(ev);
+  sand::free_slots(v);
+  if (v->pre_stream) cudaStreamDestroy(v->pre_stream);
   v->store->live_views--;
   delete v;
   return SAND_OK;

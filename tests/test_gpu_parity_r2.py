@@ -125,3 +125,76 @@ def test_rrc_central_fallback():
     for m in metas:                          # central, full width, height = round(340 / 2.5)
         assert list(m.box[0]) == [0, (256 - 136) // 2, 340, 136]
     _run(w, None, epochs=(0, 1))
+
+
+def test_bench_two_ranks_on_one_gpu():
+    """bench.py's multi-rank path with real read_batch calls: two ranks (torchrun, gloo for the
+    collectives, both on cuda:0) each read their DistributedSampler share; the barrier, the
+    max-over-ranks timing and the counter all-gather run, and the counters add up to one
+    epoch's clips exactly once."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr=127.0.0.1", "--master-port=29531", "bench.py", "--gpus", "2", "--config", "k400",
+           "--videos", "64", "--steps", "2", "--warmup", "3", "--no-cpu", "--no-e2e", "--backend", "gloo"]
+    out = subprocess.run(cmd, cwd=root, capture_output=True, text=True, timeout=600)
+    assert out.returncode == 0, out.stderr[-2000:]
+    lines = [ln for ln in out.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, out.stdout
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["value"] > 0 and d["collectives"]["backend"] == "gloo"
+    per = d["reuse"]["per_rank"]
+    assert len(per) == 2 and all(p[2] == 5 for p in per)          # 3 warm-up + 2 timed batches each
+    # 64 clips, B = 32, two ranks: one batch per rank per epoch -> 5 epochs, each clip once per epoch
+    assert d["reuse"]["batches"] == 10 and d["reuse"]["uses"] == 10 * 32 * 16
+
+
+def test_prematerialized_batches_equal_direct_reads():
+    """f1 pre-materialisation: batches materialised ahead on the view's own
+    low-priority stream, then served by read_batch (device copy) or acquire_batch (zero copy),
+    are bit-identical to direct reads; slots are reused once released."""
+    w = configs.k400()
+    w.spec.batch_size = 4
+    store, view, ospec, ods, vids = _setup(w, 16)
+    ref_view = sand.View(store, w.spec, [v[0] for v in vids])
+    try:
+        view.set_prematerialize(2)
+        for e in (0, 1):
+            n_it = view.iterations(e, 0)
+            for it in range(n_it):
+                ref = ref_view.alloc_outputs()
+                ref_view.read_batch(e, 0, it, ref)
+                view.prematerialize(e, 0, it)
+                if it % 2 == 0:                      # served by read_batch (copy out)
+                    got = view.alloc_outputs()
+                    view.read_batch(e, 0, it, got)
+                    torch.cuda.synchronize()
+                    for a, b in zip(got, ref):
+                        assert torch.equal(a.view(torch.int16), b.view(torch.int16))
+                else:                                # zero-copy hand-over
+                    ptrs = view.acquire_batch(e, 0, it)
+                    torch.cuda.synchronize()
+                    for p_, b in zip(ptrs, ref):
+                        nbytes = b.numel() * b.element_size()
+
+                        class _Dev:               # the library's buffer, wrapped without a copy
+                            __cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1",
+                                                        "data": (p_, True), "version": 3}
+                        buf = torch.as_tensor(_Dev(), device="cuda")
+                        assert torch.equal(buf, b.reshape(-1).view(torch.uint8))
+                    view.release_batch(e, 0, it)
+        # two slots: a third outstanding batch is refused
+        view.prematerialize(2, 0, 0)
+        view.prematerialize(2, 0, 1)
+        with pytest.raises(sand.SandError) as ex:
+            view.prematerialize(2, 0, 2)
+        assert ex.value.code == sand._abi.EBUSY
+        with pytest.raises(sand.SandError):
+            view.acquire_batch(2, 0, 3)
+    finally:
+        ref_view.close()
+        view.close()
+        store.close()
