@@ -269,6 +269,8 @@ def run_sand(args):
     w = configs.get(args.config)
     spec = w.spec
     spec.world_size = world
+    if args.pool_epochs:
+        spec.pool_epochs = args.pool_epochs
     n_videos = w.n_videos if args.videos is None else args.videos
     vids = [(1000 + i, w.n_frames, w.width, w.height) for i in range(n_videos)]
     pitch = (w.width + 63) // 64 * 64
@@ -282,6 +284,8 @@ def run_sand(args):
     stream.synchronize()
     log(f"[rank {rank}] store filled: {n_videos} videos, {cap / 1e9:.1f} GB in {time.time() - t0:.1f}s")
     view = sand.View(store, spec, [v[0] for v in vids])
+    if args.object_budget_gb:         # f2: HBM-budgeted cache of resized frames (R#27)
+        view.set_object_budget(int(args.object_budget_gb * 1e9))
     iters = view.iterations(0, rank)
     outs_a = view.alloc_outputs()
     outs_b = view.alloc_outputs()
@@ -423,6 +427,9 @@ def run_sand(args):
                               "alg_bytes": {"read": alg_read, "write": alg_write}},
                      "peak_source": peak_src, "frac_of_8tbs_spec": achieved / 8000.0},
         "gpu_launches": int(launches),
+        "object_cache": (None if not args.object_budget_gb else
+                         {k: int(getattr(view.object_stats(), k)) for k in
+                          ("hits", "fills", "misses", "evictions", "objects", "bytes_used", "bytes_budget")}),
         "host": host,
         "clocks": clk,
         "reuse": {"fetches": totals[0], "uses": totals[1], "batches": totals[2], "per_rank": per_rank},
@@ -598,6 +605,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=16)
+    ap.add_argument("--pool-epochs", type=int, default=0, help="k-epoch shared frame pool (f1, R#25)")
+    ap.add_argument("--object-budget-gb", type=float, default=0.0, help="HBM object cache (f2, R#27)")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend (gloo: test mode, ranks may share one GPU)")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)

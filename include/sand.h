@@ -225,6 +225,29 @@ int sand_view_acquire_batch(sand_view* v, uint64_t epoch, uint32_t rank, uint64_
                             void* data_out[SAND_MAX_VIEWS]);
 int sand_view_release_batch(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration, sand_stream_t stream);
 
+/* HBM-budgeted object reuse (§5.3 Alg. 1, §6; DESIGN.md
+ * R#27). The cached object is the RESIZED FRAME of a short-side view (R#10): the whole frame
+ * resized to W' x H' (uint8 R, G, B planes), keyed by (video, frame). Any crop of it is a copy
+ * plus normalisation, bit-identical to resampling the crop from the NV12 frame. read_batch
+ * decides per item of a group whose leader view is SHORTSIDE_CROP without rotation/blur, in
+ * batch order: HIT (cached: copied from the object), FILL (not cached, used again in a later
+ * epoch of the k-epoch chunk — Alg. 1: caching the parent instead of its >= 2 leaves saves
+ * space — and a slot is free after eviction: the resized frame is materialised into the cache,
+ * then copied from), MISS (otherwise: resampled from the NV12 frame as usual). Eviction (§6),
+ * down to 75 % of the budget when a fill finds no free slot (keeping the objects of the batch
+ * being decided) and after each batch: first objects not needed again in the current chunk
+ * (least recently used first), then the latest next use. One object size per view
+ * (the first eligible item's W' x H'; others MISS). `bytes` = 0 disables the cache (default);
+ * set it before the view plans or reads (EBUSY otherwise). Reads of a view with a cache must be
+ * ordered among themselves (one stream, or the caller orders them). Errors: EINVAL (8 views,
+ * mixed dtypes), EBUSY, ECUDA. */
+int sand_view_set_object_budget(sand_view* v, uint64_t bytes);
+typedef struct {
+  uint64_t hits, fills, misses, evictions;   /* eligible items served by each path; objects evicted */
+  uint64_t objects, bytes_used, bytes_budget;
+} sand_object_stats;
+int sand_view_object_stats(const sand_view* v, sand_object_stats* out);
+
 /* Plan an epoch ahead of time on a background host thread (the plan analogue of
  * the paper's pre-materialisation threads). Returns immediately. */
 int sand_view_prefetch_epoch(sand_view* v, uint64_t epoch, uint32_t rank);

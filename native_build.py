@@ -74,11 +74,11 @@ def build_oracle(force=False):
               src, "-o", so, "-lm"])
 
 
-PRODUCT_CPP = ["sand_api.cpp", "store.cpp", "planner.cpp", "view.cpp"]
+PRODUCT_CPP = ["sand_api.cpp", "store.cpp", "planner.cpp", "view.cpp", "objcache.cpp"]
 PRODUCT_CU = ["materialize.cu", "store_kernels.cu", "mat_plain.cu", "mat_stream.cu", "mat_direct.cu",
-              "mat_stencil.cu"]
+              "mat_stencil.cu", "mat_crop.cu"]
 PRODUCT_HDR = ["internal.h", "plan_types.h", "planner.h", "kernels.h", "kernels_common.cuh", "k_resample.cuh",
-               "k_stream.cuh", "k_plain.cuh", "k_stencil.cuh", "k_direct.cuh", "k_copy.cuh"]
+               "k_stream.cuh", "k_plain.cuh", "k_stencil.cuh", "k_direct.cuh", "k_copy.cuh", "k_crop.cuh"]
 
 
 def build_product(force=False, variant=None, defines=()):

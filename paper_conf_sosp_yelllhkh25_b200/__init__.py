@@ -65,6 +65,14 @@ def make_spec(spec: Spec, videos) -> tuple[_abi.sand_view_spec, object]:
     return s, arr
 
 
+def _stream(stream):
+    """cudaStream_t of `stream` (a raw handle, a torch.cuda.Stream, or None = torch's current)."""
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    return getattr(stream, "cuda_stream", stream)
+
+
 def plan_rank_clips(spec: Spec, videos, epoch: int, rank: int) -> list[int]:
     """Global clip ids of (epoch, rank) in DistributedSampler order (host-only planner)."""
     s, keep = make_spec(spec, list(videos))
@@ -212,6 +220,14 @@ class View:
         out = _abi.sand_batch_bytes()
         check(lib().sand_view_batch_bytes_class(self._h, epoch, rank, iteration, cls, ctypes.byref(out)),
               "sand_view_batch_bytes_class")
+        return out
+
+    def set_object_budget(self, nbytes: int) -> None:
+        check(lib().sand_view_set_object_budget(self._h, nbytes), "sand_view_set_object_budget")
+
+    def object_stats(self) -> _abi.sand_object_stats:
+        out = _abi.sand_object_stats()
+        check(lib().sand_view_object_stats(self._h, ctypes.byref(out)), "sand_view_object_stats")
         return out
 
     def set_prematerialize(self, slots: int) -> None:

@@ -83,6 +83,11 @@ class sand_view_stats(ctypes.Structure):
                 ("plan_cpu_ns", u64), ("plan_buffer_wait_ns", u64), ("lock_wait_ns", u64), ("pending_waits", u64)]
 
 
+class sand_object_stats(ctypes.Structure):
+    _fields_ = [("hits", u64), ("fills", u64), ("misses", u64), ("evictions", u64),
+                ("objects", u64), ("bytes_used", u64), ("bytes_budget", u64)]
+
+
 P = ctypes.POINTER
 SIGNATURES = {
     "sand_store_create": (ctypes.c_int, [ctypes.c_int, u64, P(vp)]),
@@ -105,6 +110,8 @@ SIGNATURES = {
     "sand_view_batch_bytes_class": (ctypes.c_int, [vp, u64, u32, u64, u32, P(sand_batch_bytes)]),
     "sand_view_set_timing": (ctypes.c_int, [vp, ctypes.c_int]),
     "sand_view_set_prematerialize": (ctypes.c_int, [vp, u32]),
+    "sand_view_set_object_budget": (ctypes.c_int, [vp, u64]),
+    "sand_view_object_stats": (ctypes.c_int, [vp, P(sand_object_stats)]),
     "sand_view_prematerialize": (ctypes.c_int, [vp, u64, u32, u64]),
     "sand_view_acquire_batch": (ctypes.c_int, [vp, u64, u32, u64, vp, P(vp)]),
     "sand_view_release_batch": (ctypes.c_int, [vp, u64, u32, u64, vp]),

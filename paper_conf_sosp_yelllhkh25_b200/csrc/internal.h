@@ -175,6 +175,10 @@ struct sand_view {
   size_t pre_view_bytes[sand::kMaxViews] = {};
   cudaStream_t pre_stream = nullptr;
   uint64_t pre_made = 0, pre_served = 0;
+  // HBM-budgeted object cache (f2, objcache.cpp): resized frames of short-side views
+  uint64_t obj_budget = 0;
+  struct ObjCache;
+  ObjCache* obj = nullptr;
   uint64_t put_seq_seen = 0;              // store->put_seq the last read_batch stream waited for
   cudaStream_t put_stream_seen = nullptr;
 };
@@ -185,6 +189,19 @@ namespace sand {
 // released) or a new plan.
 std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32_t rank,
                                       std::shared_ptr<EpochPlan> reuse = nullptr);
+bool obj_eligible_group(const sand_view_spec& s, const SpecInfo& info, uint32_t q);
+// launch shape of an arbitrary item list (view.cpp): classifies, orders (mild by clip/group/
+// frame, heavy, stencil) and builds k_plain tasks, as build_plan does for a planned batch
+void shape_items(const sand_view& v, std::vector<WorkItem>& items, const std::vector<GroupParams>& groups,
+                 const std::vector<uint32_t>& dests, const ViewConst* views, uint32_t n_views, std::vector<uint2>* tasks,
+                 BatchShape* shape);
+
+// object cache (objcache.cpp, f2): one batch through the cache; *handled = false when the view
+// has no cache (the caller then launches the plan's kernels)
+int objcache_read(sand_view* v, EpochPlan& plan, uint64_t it, const LaunchParams& base, cudaStream_t stream,
+                  int* launched, bool* handled);
+int objcache_set_budget(sand_view* v, uint64_t bytes);
+void objcache_free(sand_view* v);
 
 // kernels (materialize.cu)
 size_t stencil_smem_bytes(int max_h, int max_w, int max_r);

@@ -9,14 +9,12 @@
 // column pairs per thread; 4 x 112 = 448 for 224-wide outputs at NP = 1, no idle lanes) whose
 // control flow is identical, each frame with its
 // own source rows in shared memory. The band's source rows [y_first, y_last] are walked in
-// CHUNKS of CR rows (chunk boundaries at even rows, so a UV row never straddles two chunks),
-// double-buffered, with one CTA barrier per chunk:
-//   * the NV12 rows of chunk j + 2 are copied HBM -> shared memory by the TMA engine
+// CHUNKS of CR rows (chunk boundaries at even rows, so a UV row never straddles two chunks):
+//   * the NV12 rows of chunks j + 1 and j + 2 are copied HBM -> shared memory by the TMA engine
 //     (cp.async.bulk, one copy per row per frame, completion counted on the staging buffer's
-//     mbarrier) while chunk j is walked (a4);
-//   * chunk j + 1 is converted once into RGBx rows (R#11, the DPX formulation of k_stream.cuh;
-//     a5) while chunk j is walked: each thread owns fixed (frame, 4-pixel group) slots and converts
-//     their UV rows; odd warps walk before converting, so the two phases overlap across warps;
+//     mbarrier; two staging buffers) while chunk j is converted and walked (a4);
+//   * chunk j is converted once into RGBx rows (R#11, the DPX formulation of k_stream.cuh; a5):
+//     each thread owns fixed (frame, 4-pixel group) slots and converts their UV rows;
 //   * the walk is SOURCE-ROW major: each thread owns 2 NP adjacent output columns of its frame,
 //     computes the horizontal lerps of each source row once (R#12, a6; flip mirrors the column
 //     taps, a7) into one of two register sets whose roles alternate with the row's parity
@@ -31,12 +29,8 @@
 namespace sand {
 namespace pl {
 
-#ifndef SAND_PLAIN_SB
-#define SAND_PLAIN_SB 0               // 1: single-buffered chunks (A/B variant)
-#endif
-constexpr int kCR = SAND_PLAIN_SB ? 8 : 6;    // source rows per chunk (even)
+constexpr int kCR = 8;                // source rows per chunk (even)
 constexpr int kRawRows = kCR + kCR / 2 + 1;   // staging rows per chunk: Y rows + their UV rows
-constexpr int kConvBufs = SAND_PLAIN_SB ? 1 : 2;   // conversion buffers per frame
 
 struct Shape {        // host-chosen launch shape of one batch's plain items
   int fpc;            // frames (items of one run) per CTA
@@ -45,10 +39,10 @@ struct Shape {        // host-chosen launch shape of one batch's plain items
   int gw;             // row capacity in pixels (multiple of 16, >= every item's staged span)
 };
 
-// per frame: two converted-row buffers (chunks j and j + 1) then two staging buffers
+// per frame: the converted rows of one chunk, then two staging buffers
 __host__ __device__ inline size_t conv_bytes(const Shape& s) { return (size_t)kCR * s.gw * 4; }
 __host__ __device__ inline size_t raw_bytes(const Shape& s) { return rs::a16((size_t)kRawRows * s.gw); }
-__host__ __device__ inline size_t frame_bytes(const Shape& s) { return kConvBufs * conv_bytes(s) + 2 * raw_bytes(s); }
+__host__ __device__ inline size_t frame_bytes(const Shape& s) { return conv_bytes(s) + 2 * raw_bytes(s); }
 __host__ __device__ inline size_t smem_bytes(const Shape& s) {
   return rs::a16((size_t)s.rb * 8) + 16 + (size_t)s.fpc * frame_bytes(s);
 }
@@ -92,8 +86,7 @@ __global__ void __launch_bounds__(PlainBounds<NP>::kThreads, PlainBounds<NP>::kM
   const uint32_t s_fr = s_bar + 16;                                // frame f at s_fr + f * fbytes
   const uint32_t fbytes = (uint32_t)pl::frame_bytes(sh);
   const uint32_t rowbytes = (uint32_t)sh.gw * 4u;                  // converted row stride
-  const uint32_t convb = (uint32_t)pl::conv_bytes(sh);             // conv buffer b at b * convb
-  const uint32_t raw_off = (uint32_t)pl::kConvBufs * convb;        // staging buffer b at raw_off + b * rawb
+  const uint32_t raw_off = (uint32_t)pl::conv_bytes(sh);           // staging buffer b at raw_off + b * rawb
   const uint32_t rawb = (uint32_t)pl::raw_bytes(sh);
   const uint32_t rawpitch = (uint32_t)sh.gw;                       // staging row stride
 
@@ -213,14 +206,14 @@ __global__ void __launch_bounds__(PlainBounds<NP>::kThreads, PlainBounds<NP>::kM
   // owns slots t, t + nthr, ...); a chunk converts every UV row of every slot
   const int q4 = gwi >> 2;
   const int n_slots = nfr * q4;
-  // chunk j: staged rows -> RGBx rows of conversion buffer j & 1, after waiting for its staging buffer
+  // chunk j: staged rows -> RGBx rows of the conversion buffer, after waiting for its staging buffer
   auto convert = [&](int j) {
     const int ya = chunk_lo(j), yb = chunk_hi(j);
     st::mbar_wait(s_bar + 8u * (uint32_t)(j & 1), (uint32_t)(j >> 1) & 1u);
     const int ny = yb - ya + 1, u0 = ya >> 1, nuv = (yb >> 1) - u0 + 1;
     const uint32_t slot0 = (uint32_t)(ybase + j * kCR);            // absolute row of slot 0
     const uint8_t* rawb0 = smem_raw + (s_fr - s_base) + raw_off + (uint32_t)(j & 1) * rawb;
-    uint8_t* convb0 = smem_raw + (s_fr - s_base) + (uint32_t)(j & (pl::kConvBufs - 1)) * convb;
+    uint8_t* convb0 = smem_raw + (s_fr - s_base);
     for (int sl = tid; sl < n_slots; sl += nthr) {
       const int fr = sl / q4, q = sl - fr * q4;
       const uint8_t* raw = rawb0 + (uint32_t)fr * fbytes + 4u * q;
@@ -248,7 +241,7 @@ __global__ void __launch_bounds__(PlainBounds<NP>::kThreads, PlainBounds<NP>::kM
   // output rows whose top tap is y - 1 are emitted as soon as y's lerps exist
   auto walk = [&](int j) {
     const int ya = chunk_lo(j), yb = chunk_hi(j);
-    uint32_t row = (uint32_t)(j & (pl::kConvBufs - 1)) * convb + (uint32_t)(ya - ybase - j * kCR) * rowbytes;   // row ya
+    uint32_t row = (uint32_t)(ya - ybase - j * kCR) * rowbytes;   // offset of row ya
     int y = ya;
     if ((y - y_first) & 1) {
       hrows(Y, row);
@@ -269,7 +262,6 @@ __global__ void __launch_bounds__(PlainBounds<NP>::kThreads, PlainBounds<NP>::kM
     }
   };
 
-#if SAND_PLAIN_SB
   // single-buffered chunks: convert chunk j, barrier, stage chunk j + 1, walk chunk j
   for (int j = 0; j < nchunks; ++j) {
     __syncthreads();                       // walk of chunk j - 1 done: conversion buffer free
@@ -282,28 +274,6 @@ __global__ void __launch_bounds__(PlainBounds<NP>::kThreads, PlainBounds<NP>::kM
     }
     walk(j);
   }
-#else
-  convert(0);
-  __syncthreads();                         // chunk 0 converted, its staging buffer drained; table visible
-  asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(rt.x), "=r"(rt.y) : "r"(s_tab));
-  for (int j = 0; j < nchunks; ++j) {
-    // staging buffer j & 1 was drained by convert(j) before the last barrier: chunk j + 2 may land
-    if (j + 2 < nchunks && warp == 0) {
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-      stage(j + 2);
-    }
-    // convert chunk j + 1 (buffer (j + 1) & 1, last read by the walk of chunk j - 1 before the
-    // barrier) and walk chunk j; odd warps walk first, so the CTA's warps overlap the two phases
-    for (int ph = 0; ph < 2; ++ph) {
-      if (((ph ^ warp) & 1) == 0) {
-        if (j + 1 < nchunks) convert(j + 1);
-      } else {
-        walk(j);
-      }
-    }
-    __syncthreads();
-  }
-#endif
   // rows at the bottom clamp (y0 == y1 == y_last, lambda 0): emitted from H(y_last) twice
   if ((y_last - y_first) & 1) emit_rows(Y, Y, y_last);
   else emit_rows(X, X, y_last);

@@ -38,6 +38,11 @@ int launch_stream_generic(const LaunchParams& p, const BatchShape& sh, cudaStrea
 // mat_direct.cu — k_direct over heavy items p.items[0, n) (source step > 2)
 int launch_direct(const LaunchParams& p, const BatchShape& sh, cudaStream_t stream);
 
+// mat_crop.cu — crops of cached resized frames (f2): `items` is a device array of n_items
+// CropItem (k_crop.cuh), all of one output dtype
+int launch_crop(const LaunchParams& p, const uint8_t* slab, const void* items, uint32_t n_items, int max_wo,
+                int max_ho, int dtype, cudaStream_t stream);
+
 // mat_stencil.cu — rotation / blur items p.items[0, n): k_stencil2, or k_stencil for planes
 // beyond shared memory
 size_t stencil_smem_bytes(int max_h, int max_w, int max_r);

@@ -32,6 +32,7 @@ int launch_plain(const LaunchParams& p, const BatchShape& sh, int fpc, int nq, c
   if (smem > 200 * 1024) return SAND_OK;                         // pathological widths: generic kernel
   const unsigned threads = (unsigned)((fpc * nq + 31) / 32 * 32);
   if (threads > (unsigned)PlainBounds<kNP>::kThreads) return SAND_OK;   // very wide outputs: generic kernel
+  if (sh.max_wo > 2 * kNP * nq) return SAND_OK;                   // wider than the view's CTA rows
   const uint2* tasks = p.tasks + sh.task_first;
   const bool nd1 = sh.max_dests <= 1;
   switch (sh.dtype) {

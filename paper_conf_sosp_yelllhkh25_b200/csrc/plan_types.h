@@ -50,6 +50,16 @@ struct alignas(16) WorkItem {
   uint32_t pad;
 };
 
+// One crop of a cached resized frame (object reuse, f2; k_crop.cuh, objcache.cpp)
+struct alignas(16) CropItem {
+  uint64_t obj;          // byte offset of the object (plane R) in the object slab
+  uint32_t obj_w, obj_h; // W', H' (plane pitch W', planes W' * H' bytes apart)
+  uint32_t x_off, y_off, flip;
+  uint32_t out_w, out_h;
+  uint32_t dest_begin, n_dest;
+  uint32_t pad;
+};
+
 // destination packing: view (8 bits) << 24 | t (8 bits) << 16 | b (16 bits)
 SAND_HD inline uint32_t pack_dest(uint32_t view, uint32_t t, uint32_t b) {
   return (view << 24) | (t << 16) | b;

@@ -21,11 +21,11 @@
 namespace sand {
 namespace {
 
-constexpr size_t kPlanCache = 4;   // current epoch, kPlanAhead ahead, and the previous one
+constexpr size_t kPlanCache = 5;   // current epoch, kPlanAhead ahead, and the previous one
 constexpr size_t kMaxPooled = 8;   // idle plan buffers kept for reuse
 constexpr size_t kPrealloc = 6;    // spare plan buffers allocated with the first one
 }  // namespace
-constexpr uint64_t kPlanAhead = 2;
+constexpr uint64_t kPlanAhead = 3;
 constexpr uint64_t kInflight = 48;   // batches of one view queued on the GPU at most
 namespace {
 constexpr double kPi = 3.14159265358979323846;
@@ -79,6 +79,19 @@ GroupParams group_params(const sand_view_desc& d, const sand_clip_meta& m, uint3
   }
   return g;
 }
+
+}  // namespace
+
+// object-reuse eligibility (f2, R#27): a group whose leader view is a short-side crop without
+// rotation or blur (its items are crops of one deterministic resized frame)
+bool obj_eligible_group(const sand_view_spec& s, const SpecInfo& info, uint32_t q) {
+  const int lead = info.leader[q];
+  if (lead < 0) return false;
+  const sand_view_desc& d = s.views[lead];
+  return d.geom == SAND_GEOM_SHORTSIDE_CROP && d.rot_p <= 0.0 && d.blur_p <= 0.0;
+}
+
+namespace {
 
 // staged column span of a group (16-aligned pixels the kernels copy per source row): from the
 // first column's i0 to the last column's i1 (taps are monotone; the same set under flip)
@@ -171,6 +184,60 @@ void plain_tasks(const std::vector<WorkItem>& items, size_t first, size_t n, con
 
 }  // namespace
 
+void shape_items(const sand_view& v, std::vector<WorkItem>& items, const std::vector<GroupParams>& groups,
+                 const std::vector<uint32_t>& dests, const ViewConst* views, uint32_t n_views, std::vector<uint2>* tasks,
+                 BatchShape* shape) {
+  BatchShape sh{};
+  sh.direct_identity = 1;
+  sh.src_w_mod4 = 1;
+  sh.even_wo = sh.wo_mod4 = 1;
+  sh.dtype = -2;   // unset
+  for (auto& w : items) {
+    const GroupParams& g = groups[w.gp];
+    const bool mild = g.sc_x <= 2.0f && g.sc_y <= 2.0f;
+    const int cols = span16(g);
+    w.flags = (g.rot_on || g.blur_on) ? 1u : (mild ? 0u : 2u);
+    for (uint32_t d = 0; d < w.n_dest; ++d) {
+      const ViewConst& vc = views[dests[w.dest_begin + d] >> 24];
+      sh.dtype = sh.dtype == -2 ? vc.dtype : (sh.dtype == vc.dtype ? sh.dtype : -1);
+      if (vc.out_w & 1) sh.even_wo = 0;
+      if (vc.out_w & 3) sh.wo_mod4 = 0;
+    }
+    if (w.flags & 1u) {
+      sh.has_stencil = 1;
+      sh.st_max_wo = std::max(sh.st_max_wo, g.out_w);
+      sh.st_max_ho = std::max(sh.st_max_ho, g.out_h);
+      sh.st_cols_bound = std::max(sh.st_cols_bound, cols);
+      sh.st_max_scy = std::max(sh.st_max_scy, g.sc_y);
+    } else {
+      sh.has_direct = 1;
+      sh.max_dests = std::max<int32_t>(sh.max_dests, static_cast<int32_t>(w.n_dest));
+      if (mild) {
+        if (!(g.sc_x == 1.0f && g.sc_y == 1.0f)) sh.direct_identity = 0;
+        if (w.src_w % 4u) sh.src_w_mod4 = 0;
+        sh.max_wo = std::max(sh.max_wo, g.out_w);
+        sh.max_ho = std::max(sh.max_ho, g.out_h);
+        sh.cols_bound = std::max(sh.cols_bound, cols);
+        sh.max_scy = std::max(sh.max_scy, g.sc_y);
+      } else {
+        sh.heavy_max_wo = std::max(sh.heavy_max_wo, g.out_w);
+        sh.heavy_max_ho = std::max(sh.heavy_max_ho, g.out_h);
+      }
+    }
+  }
+  (void)n_views;
+  if (sh.dtype == -2) sh.dtype = -1;
+  auto mid = std::stable_partition(items.begin(), items.end(), [](const WorkItem& w) { return !(w.flags & 1u); });
+  sh.n_direct = static_cast<uint32_t>(mid - items.begin());
+  auto hv = std::stable_partition(items.begin(), mid, [](const WorkItem& w) { return !(w.flags & 2u); });
+  sh.n_mild = static_cast<uint32_t>(hv - items.begin());
+  std::stable_sort(items.begin(), hv, [](const WorkItem& a, const WorkItem& b) {
+    return a.clip_slot != b.clip_slot ? a.clip_slot < b.clip_slot : a.group < b.group;
+  });
+  plain_tasks(items, 0, sh.n_mild, groups, v.pl_fpc, tasks, &sh);
+  *shape = sh;
+}
+
 std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32_t rank,
                                       std::shared_ptr<EpochPlan> plan) {
   const SpecInfo& info = v.info;
@@ -206,6 +273,7 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
   plan->item_begin.push_back(0);
   plan->fetch_begin.push_back(0);
   std::vector<uint64_t> uses_of;   // (frame << 32) | (view << 16) | t
+  std::vector<uint64_t> later;     // (epoch delta << 48) | (group << 32) | frame of later epochs (f2)
   uses_of.reserve(frames_per_clip);
   std::vector<uint32_t> batch_videos(B);
   int32_t common_dtype = s.views[0].out_dtype;
@@ -236,6 +304,21 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
       const uint32_t clip = clips[slot];
       plan_clip(info, epoch, clip, &m);
       const VideoDims& dim = info.dims[clip / s.samples_per_video];
+      // object reuse (f2, R#27): frames this clip selects, per object-eligible group, in the later
+      // epochs of the current k-epoch chunk (their count and the next one travel in WorkItem.pad)
+      const uint32_t kch = std::max<uint32_t>(1, s.pool_epochs);
+      const uint64_t chunk_end = (epoch / kch + 1) * kch;
+      later.clear();
+      if (v.obj_budget > 0)
+        for (uint64_t e2 = epoch + 1; e2 < chunk_end; ++e2) {
+          sand_clip_meta m2;
+          plan_clip(info, e2, clip, &m2);
+          for (uint32_t k = 0; k < s.n_views; ++k)
+            if (obj_eligible_group(s, info, s.views[k].spatial_group))
+              for (uint32_t t = 0; t < s.views[k].clip_len; ++t)
+                later.push_back((static_cast<uint64_t>(e2 - epoch) << 48) |
+                                (static_cast<uint64_t>(s.views[k].spatial_group) << 32) | m2.frames[k][t]);
+        }
       VideoEntry* ent = v.entries[clip / s.samples_per_video];
       for (uint32_t gi = 0; gi < nG; ++gi) {
         const uint32_t q = info.groups[gi];
@@ -303,6 +386,19 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
           w.clip_slot = b;
           w.group = q;
           w.flags = gflags[gi];
+          if (!later.empty() && !(gflags[gi] & 1u) && obj_eligible_group(s, info, q)) {
+            uint32_t uses = 0, next = 0xffffu;   // later epochs selecting frame f for group q
+            uint64_t last_e = 0;
+            for (uint64_t x : later)
+              if (((x >> 32) & 0xffffu) == q && static_cast<uint32_t>(x) == f && (x >> 48) != last_e) {
+                last_e = x >> 48;
+                ++uses;
+                next = std::min<uint32_t>(next, static_cast<uint32_t>(last_e));
+              }
+            w.pad = (uses << 16) | next;
+          } else {
+            w.pad = 0xffffu;                    // no later use known
+          }
           plan->items.push_back(w);
         }
         fetch.push_back({(static_cast<uint64_t>(dim.id) << 32) | f, uses, ent});
@@ -670,7 +766,7 @@ extern "C" int sand_view_create(sand_store* s, const sand_view_spec* spec, sand_
     return sand::cuda_error(e, "cudaStreamCreate(upload)");
   }
   s->live_views++;
-  const int n_workers = 2;   // plan builders: the current epoch's and the next one's
+  const int n_workers = 3;   // plan builders (epochs e + 1 .. e + kPlanAhead)
   for (int i = 0; i < n_workers; ++i) v->workers.emplace_back(sand::worker_loop, v);
   *out = v;
   return SAND_OK;
@@ -987,8 +1083,11 @@ static int read_batch_direct(sand_view* v, uint64_t epoch, uint32_t rank, const 
         }
       }
   }
-  int rc = sand::launch_materialize(lp, bshape, v->stencil_smem, v->pl_fpc, v->pl_nq, stream, v->aux_stream, v->fork_ev,
-                                    v->join_ev, &launched, v->timing ? &cev : nullptr);
+  bool cached = false;
+  int rc = sand::objcache_read(v, *plan, it, lp, stream, &launched, &cached);   // f2 object cache, if configured
+  if (rc == SAND_OK && !cached)
+    rc = sand::launch_materialize(lp, bshape, v->stencil_smem, v->pl_fpc, v->pl_nq, stream, v->aux_stream, v->fork_ev,
+                                  v->join_ev, &launched, v->timing ? &cev : nullptr);
   if (v->timing)
     for (int c = 0; c < 3; ++c) {
       if (cev.used[c] && rc == SAND_OK) {
@@ -1194,6 +1293,7 @@ extern "C" int sand_view_destroy(sand_view* v) {
   for (auto& ev : v->free_events) cudaEventDestroy(ev);
   sand::free_slots(v);
   if (v->pre_stream) cudaStreamDestroy(v->pre_stream);
+  sand::objcache_free(v);
   v->store->live_views--;
   delete v;
   return SAND_OK;

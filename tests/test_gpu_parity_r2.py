@@ -182,7 +182,7 @@ def test_prematerialized_batches_equal_direct_reads():
 
                         class _Dev:               # the library's buffer, wrapped without a copy
                             __cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1",
-                                                        "data": (p_, True), "version": 3}
+                                                        "data": (p_, False), "version": 3}
                         buf = torch.as_tensor(_Dev(), device="cuda")
                         assert torch.equal(buf, b.reshape(-1).view(torch.uint8))
                     view.release_batch(e, 0, it)
@@ -196,5 +196,44 @@ def test_prematerialized_batches_equal_direct_reads():
             view.acquire_batch(2, 0, 3)
     finally:
         ref_view.close()
+        view.close()
+        store.close()
+
+
+@pytest.mark.parametrize("src,budget_objs", [((1280, 720), 10**6), ((1280, 720), 5), ((340, 256), 12)])
+def test_object_cache_bit_identical_and_policy_matches_oracle(src, budget_objs):
+    """f2 (P:L299-359, :396; R#27): with an HBM budget for resized frames, every batch is
+    bit-identical to the uncached path, and the hit / fill / miss / eviction counts after every
+    read equal the oracle's replay of the same policy (oracle/object_cache.py)."""
+    from oracle import object_cache
+    w = configs.slowfast_hd() if src == (1280, 720) else configs.slowfast()
+    w.width, w.height = src
+    w.spec.batch_size = 2
+    w.spec.pool_epochs = 3
+    store, view, ospec, ods, vids = _setup(w, 4)
+    ref = sand.View(store, w.spec, [v[0] for v in vids])
+    try:
+        m0 = oracle.plan_batch(ospec, ods, len(vids), 0, 0, 0)[0]
+        objbytes = 3 * m0.box[0][2] * m0.box[0][3]
+        budget = objbytes * budget_objs + 16 if budget_objs < 10**6 else objbytes * 400
+        view.set_object_budget(budget)
+        reads = [(e, it) for e in range(5) for it in range(view.iterations(e, 0))]
+        expect = object_cache.simulate(ospec, ods, len(vids), budget, reads)
+        for (e, it), ex in zip(reads, expect):
+            a, b = view.alloc_outputs(), ref.alloc_outputs()
+            view.read_batch(e, 0, it, a)
+            ref.read_batch(e, 0, it, b)
+            torch.cuda.synchronize()
+            for x, y in zip(a, b):
+                assert torch.equal(x.view(torch.int16), y.view(torch.int16)), (e, it)
+            st = view.object_stats()
+            got = {"hits": st.hits, "fills": st.fills, "misses": st.misses, "evictions": st.evictions,
+                   "objects": st.objects}
+            assert got == ex, ((e, it), got, ex)
+        assert expect[-1]["hits"] > 0 and expect[-1]["fills"] > 0
+        if budget_objs == 5:
+            assert expect[-1]["evictions"] > 0
+    finally:
+        ref.close()
         view.close()
         store.close()

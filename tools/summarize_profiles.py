@@ -1,11 +1,12 @@
 #!/usr/bin/env python
-"""Turn a scripts/gpu_round.sh run (gpurun_out/) into committed evidence under profiles/.
+"""Turn a scripts/evidence.sh run (gpurun_out/<tag>_*) into committed evidence under profiles/.
 
-    python tools/summarize_profiles.py r01
+    python tools/summarize_profiles.py <tag> [round]      # e.g. r02a r02
 
 Writes profiles/<round>_bench_<config>.json, profiles/<round>_launches_<config>.csv,
-profiles/<round>_ncu_summary.md and profiles/ncu_traffic.json (DRAM bytes per launch of each
-config's dominant kernel, read by bench.py for the roofline "traffic" field).
+profiles/<round>_ncu_summary.md (per-kernel metrics incl. the FMA/ALU pipe utilisation, the ALU
+roofline of the blur/conversion-bound kernels) and profiles/ncu_traffic.json (DRAM bytes per
+launch of each config's dominant kernel, read by bench.py for the roofline "traffic" field).
 """
 import csv
 import glob
@@ -34,6 +35,10 @@ METRICS = [
     ("launch__grid_size", "grid"),
     ("launch__block_size", "block"),
     ("sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active", "tensor pipe %"),
+    ("sm__inst_executed_pipe_fma.avg.pct_of_peak_sustained_active", "FMA pipe inst %"),
+    ("sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active", "FMA pipe cycles %"),
+    ("sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active", "ALU pipe inst %"),
+    ("sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active", "LSU pipe inst %"),
 ]
 
 
@@ -50,16 +55,17 @@ def raw_rows(path):
 
 
 def main():
-    rnd = sys.argv[1] if len(sys.argv) > 1 else "r01"
+    tag = sys.argv[1] if len(sys.argv) > 1 else "r02a"
+    rnd = sys.argv[2] if len(sys.argv) > 2 else tag[:3]
     os.makedirs(PROF, exist_ok=True)
     traffic = {}
     md = [f"# ncu summary, round {rnd}", "",
-          "Captured with `scripts/gpu_round.sh` on one B200 (`ncu --set full --clock-control none`, "
-          "kernels matching `k_(stream|stencil|resample|direct|copy)`, 2 launches after 6 skipped). Per-launch, "
+          "Captured with `scripts/evidence.sh` on one B200 (`ncu --set full --clock-control none`, "
+          "kernels matching `k_(plain|stream|stencil|direct|copy)`, 2 launches after 6 skipped). Per-launch, "
           "cold-cache, serialised: compare shares, not absolutes. Bench numbers come from "
           "`bench.py` (CUDA events, no profiler).", ""]
-    for path in sorted(glob.glob(os.path.join(OUT, "ncu_raw_*.csv"))):
-        cfg = os.path.basename(path)[len("ncu_raw_"):-4]
+    for path in sorted(glob.glob(os.path.join(OUT, f"{tag}_ncu_raw_*.csv"))):
+        cfg = os.path.basename(path)[len(f"{tag}_ncu_raw_"):-4]
         hdr, units, data = raw_rows(path)
         if not data:
             continue
@@ -88,21 +94,21 @@ def main():
         traffic[cfg] = {"kernel": dom[0], "dram_bytes_per_launch": dom[1][1] / dom[1][2],
                         "ncu_duration_per_launch": dom[1][0] / dom[1][2],
                         "source": f"profiles/{rnd}_ncu_summary.md"}
-        det = os.path.join(OUT, f"ncu_details_{cfg}.csv")
+        det = os.path.join(OUT, f"{tag}_ncu_details_{cfg}.csv")
         if os.path.exists(det):
             notes = []
             for r in csv.reader(open(det)):
                 if len(r) > 15 and r[12] in ("IssueSlotUtilization", "CPIStall", "TheoreticalOccupancy") and r[14]:
                     notes.append(f"- {r[4].split('(')[0]} / {r[12]}: {r[14][:300]}")
             md += sorted(set(notes))[:6] + [""]
-    for path in sorted(glob.glob(os.path.join(OUT, "launches_*.csv"))):
-        cfg = os.path.basename(path)[len("launches_"):-4]
+    for path in sorted(glob.glob(os.path.join(OUT, f"{tag}_launches_*.csv"))):
+        cfg = os.path.basename(path)[len(f"{tag}_launches_"):-4]
         rows = [r for r in csv.reader(open(path)) if len(r) > 10]
         if rows:
             with open(os.path.join(PROF, f"{rnd}_launches_{cfg}.csv"), "w", newline="") as f:
                 csv.writer(f).writerows(rows)
-    for path in sorted(glob.glob(os.path.join(OUT, "bench_*.json"))):
-        name = os.path.basename(path)[len("bench_"):-5]
+    for path in sorted(glob.glob(os.path.join(OUT, f"{tag}_bench_*.json"))):
+        name = os.path.basename(path)[len(f"{tag}_bench_"):-5]
         try:
             line = json.loads(open(path).read().strip().splitlines()[-1])
         except (ValueError, IndexError):
@@ -111,8 +117,10 @@ def main():
     open(os.path.join(PROF, f"{rnd}_ncu_summary.md"), "w").write("\n".join(md) + "\n")
     json.dump(traffic, open(os.path.join(PROF, "ncu_traffic.json"), "w"), indent=1)
     for f in ("gpu.txt", "pytest_gpu.log", "smoke.log"):
-        if os.path.exists(os.path.join(OUT, f)):
-            shutil.copy(os.path.join(OUT, f), os.path.join(PROF, f"{rnd}_{f}"))
+        if os.path.exists(os.path.join(OUT, f"{tag}_{f}")):
+            shutil.copy(os.path.join(OUT, f"{tag}_{f}"), os.path.join(PROF, f"{rnd}_{f}"))
+    for path in sorted(glob.glob(os.path.join(OUT, f"{tag}_ncu_sass_*.csv.gz"))):
+        shutil.copy(path, os.path.join(PROF, os.path.basename(path).replace(tag, rnd)))
     print(open(os.path.join(PROF, f"{rnd}_ncu_summary.md")).read())
     print(json.dumps(traffic, indent=1))
 
