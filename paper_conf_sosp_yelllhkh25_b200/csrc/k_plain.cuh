@@ -62,7 +62,7 @@ struct PlainBounds {
   static constexpr int kMinBlocks = 2;
 };
 
-template <int DT, int ND, int NP>
+template <int DT, int ND, int NP, bool FOLD>
 __global__ void __launch_bounds__(PlainBounds<NP>::kThreads, PlainBounds<NP>::kMinBlocks) k_plain(const LaunchParams p, const uint2* __restrict__ tasks, pl::Shape sh) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   using namespace rs;
@@ -180,7 +180,7 @@ __global__ void __launch_bounds__(PlainBounds<NP>::kThreads, PlainBounds<NP>::kM
   const uint32_t* dests = p.dests + wf.dest_begin;
   Dest dl[ND];
 #pragma unroll
-  for (int d = 0; d < ND; ++d) dl[d] = make_dest(p, dests[d < nd ? d : 0], Y0, ox);
+  for (int d = 0; d < ND; ++d) dl[d] = make_dest(p, dests[d < nd ? d : 0], Y0, ox, FOLD);
   Row3 X[NP], Y[NP];
 #pragma unroll
   for (int j = 0; j < NP; ++j)
@@ -195,7 +195,7 @@ __global__ void __launch_bounds__(PlainBounds<NP>::kThreads, PlainBounds<NP>::kM
   // emit every output row whose y0 is `y` from the lerps of rows y (T) and y + 1 (B)
   auto emit_rows = [&](const Row3 (&T)[NP], const Row3 (&B)[NP], int y) {
     while ((int)rt.x == y) {
-      if (active) st::emit_np<DT, ND, NP>(T, B, __uint_as_float(rt.y), dl, p, dests, nd, Y0 + r, ox);
+      if (active) st::emit_np<DT, ND, NP, FOLD>(T, B, __uint_as_float(rt.y), dl, p, dests, nd, Y0 + r, ox);
       ++r;
       rt.x = 0xffffffffu;
       if (r < nr) asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(rt.x), "=r"(rt.y) : "r"(s_tab + 8u * (uint32_t)r));

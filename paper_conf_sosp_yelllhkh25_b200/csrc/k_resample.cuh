@@ -125,7 +125,7 @@ struct Dest {
   float a[3], b[3];
 };
 
-__device__ __forceinline__ Dest make_dest(const LaunchParams& p, uint32_t dest, int oy, int ox) {
+__device__ __forceinline__ Dest make_dest(const LaunchParams& p, uint32_t dest, int oy, int ox, bool fold = false) {
   const uint32_t k = dest >> 24, t = (dest >> 16) & 0xffu, b = dest & 0xffffu;
   const ViewConst& vc = p.views[k];
   Dest d;
@@ -137,7 +137,7 @@ __device__ __forceinline__ Dest make_dest(const LaunchParams& p, uint32_t dest, 
 #pragma unroll
   for (int c = 0; c < 3; ++c) {
     d.a[c] = vc.a[c];
-    d.b[c] = vc.b[c];
+    d.b[c] = fold ? vc.bf[c] : vc.b[c];
   }
   return d;
 }

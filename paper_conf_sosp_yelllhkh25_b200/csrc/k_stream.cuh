@@ -242,7 +242,9 @@ constexpr uint32_t kActFlip = 4;   // y0 = previous y0 + 1: the old bottom set b
 // 2 NP adjacent columns, one 4 NP-byte (bf16) / 8 NP-byte (f32) / 2 NP-byte (u8) store per
 // channel and destination. Requires out_w % (2 NP) == 0 for every view (host-checked), so the
 // stores are aligned.
-template <int DT, int ND, int NP>
+// FOLD: the destinations' b fields hold b' = b - 2^23 a (ViewConst::fold) and the rint bias is
+// 2^23: y = fmaf(2^23 + q, a, b') == fmaf(q, a, b) exactly, one packed add fewer per pair.
+template <int DT, int ND, int NP, bool FOLD = false>
 __device__ __forceinline__ void emit_np(const rs::Row3 (&top)[NP], const rs::Row3 (&bot)[NP], float l,
                                         rs::Dest (&dl)[ND], const LaunchParams& p, const uint32_t* __restrict__ dests,
                                         int nd, int oy, int ox) {
@@ -255,8 +257,14 @@ __device__ __forceinline__ void emit_np(const rs::Row3 (&top)[NP], const rs::Row
 #pragma unroll
     for (int c = 0; c < 3; ++c) {
       const uint64_t dv = f2::fma(top[j].h[c], f2::splat(-1.f), bot[j].h[c]);   // h1 - h0
-      tq[j][c] = rint_biased(f2::fma(ly, dv, top[j].h[c]));                     // rint(fmaf(ly, h1-h0, h0))
-      q[j][c] = DT == SAND_U8 ? tq[j][c] : f2::add(tq[j][c], f2::splat(-kRound));
+      const uint64_t v = f2::fma(ly, dv, top[j].h[c]);                          // fmaf(ly, h1-h0, h0)
+      if constexpr (FOLD) {
+        tq[j][c] = f2::add(v, f2::splat(kBias));                               // 2^23 + rint(v)
+        q[j][c] = tq[j][c];
+      } else {
+        tq[j][c] = rint_biased(v);                                              // 1.5 * 2^23 + rint(v)
+        q[j][c] = DT == SAND_U8 ? tq[j][c] : f2::add(tq[j][c], f2::splat(-kRound));
+      }
     }
   auto store = [&](const Dest& d) {
 #pragma unroll
@@ -297,7 +305,7 @@ __device__ __forceinline__ void emit_np(const rs::Row3 (&top)[NP], const rs::Row
       dl[d].row += dl[d].rstride;
     }
   }
-  for (int d = ND; d < nd; ++d) store(make_dest(p, dests[d], oy, ox));   // rare: more destinations
+  for (int d = ND; d < nd; ++d) store(make_dest(p, dests[d], oy, ox, FOLD));   // rare: more destinations
 }
 
 }  // namespace st

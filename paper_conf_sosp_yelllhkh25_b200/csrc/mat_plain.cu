@@ -13,9 +13,11 @@ int plain_cols_per_thread() { return 2 * kNP; }
 int plain_max_threads() { return PlainBounds<kNP>::kThreads; }
 
 int configure_plain() {
-  for (cudaError_t e : {allow_smem(k_plain<SAND_U8, 1, kNP>), allow_smem(k_plain<SAND_BF16, 1, kNP>),
-                        allow_smem(k_plain<SAND_F32, 1, kNP>), allow_smem(k_plain<SAND_U8, 2, kNP>),
-                        allow_smem(k_plain<SAND_BF16, 2, kNP>), allow_smem(k_plain<SAND_F32, 2, kNP>)})
+  for (cudaError_t e : {allow_smem(k_plain<SAND_U8, 1, kNP, false>), allow_smem(k_plain<SAND_BF16, 1, kNP, false>),
+                        allow_smem(k_plain<SAND_F32, 1, kNP, false>), allow_smem(k_plain<SAND_U8, 2, kNP, false>),
+                        allow_smem(k_plain<SAND_BF16, 2, kNP, false>), allow_smem(k_plain<SAND_F32, 2, kNP, false>),
+                        allow_smem(k_plain<SAND_BF16, 1, kNP, true>), allow_smem(k_plain<SAND_F32, 1, kNP, true>),
+                        allow_smem(k_plain<SAND_BF16, 2, kNP, true>), allow_smem(k_plain<SAND_F32, 2, kNP, true>)})
     if (e != cudaSuccess) return cuda_error(e, "cudaFuncSetAttribute(k_plain)");
   return SAND_OK;
 }
@@ -35,20 +37,33 @@ int launch_plain(const LaunchParams& p, const BatchShape& sh, int fpc, int nq, c
   if (sh.max_wo > 2 * kNP * nq) return SAND_OK;                   // wider than the view's CTA rows
   const uint2* tasks = p.tasks + sh.task_first;
   const bool nd1 = sh.max_dests <= 1;
+#define SAND_PLAIN_LAUNCH(DT, ND, FOLD) k_plain<DT, ND, kNP, FOLD><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s)
+  const bool fold = sh.fold != 0;   // normalisation folds the rint bias (ViewConst::fold)
   switch (sh.dtype) {
     case SAND_U8:
-      if (nd1) k_plain<SAND_U8, 1, kNP><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
-      else k_plain<SAND_U8, 2, kNP><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
+      if (nd1) SAND_PLAIN_LAUNCH(SAND_U8, 1, false);
+      else SAND_PLAIN_LAUNCH(SAND_U8, 2, false);
       break;
     case SAND_BF16:
-      if (nd1) k_plain<SAND_BF16, 1, kNP><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
-      else k_plain<SAND_BF16, 2, kNP><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
+      if (fold) {
+        if (nd1) SAND_PLAIN_LAUNCH(SAND_BF16, 1, true);
+        else SAND_PLAIN_LAUNCH(SAND_BF16, 2, true);
+      } else {
+        if (nd1) SAND_PLAIN_LAUNCH(SAND_BF16, 1, false);
+        else SAND_PLAIN_LAUNCH(SAND_BF16, 2, false);
+      }
       break;
     default:
-      if (nd1) k_plain<SAND_F32, 1, kNP><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
-      else k_plain<SAND_F32, 2, kNP><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);
+      if (fold) {
+        if (nd1) SAND_PLAIN_LAUNCH(SAND_F32, 1, true);
+        else SAND_PLAIN_LAUNCH(SAND_F32, 2, true);
+      } else {
+        if (nd1) SAND_PLAIN_LAUNCH(SAND_F32, 1, false);
+        else SAND_PLAIN_LAUNCH(SAND_F32, 2, false);
+      }
       break;
   }
+#undef SAND_PLAIN_LAUNCH
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_error(e, "k_plain launch");
   *launched = true;

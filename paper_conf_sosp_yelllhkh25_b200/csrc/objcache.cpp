@@ -23,6 +23,7 @@
 #include <algorithm>
 #include <cstring>
 #include <map>
+#include <unordered_map>
 
 #include "internal.h"
 #include "kernels.h"
@@ -40,7 +41,7 @@ struct sand_view::ObjCache {
     uint64_t next_epoch;     // next planned use (UINT64_MAX: none)
     uint64_t last_batch;     // batch sequence number of its last touch (LRU)
   };
-  std::map<std::pair<uint32_t, uint32_t>, Obj> objs;   // (video id, frame)
+  std::unordered_map<uint64_t, Obj> objs;   // key: video id << 32 | frame
   uint64_t seq = 0;
   sand_object_stats stats{};
   // per-batch device arrays (fills, crops, misses), a small ring guarded by events
@@ -112,12 +113,18 @@ namespace {
 // chunk, least recently used first, then (2) by the latest next use (ties: least recently used,
 // then key); during a batch its own objects are kept (protect_batch). Returns objects evicted.
 size_t evict_to_threshold(sand_view::ObjCache* c, uint64_t epoch, uint64_t chunk, bool protect_batch) {
+  const uint64_t keep = c->budget * 3 / (4 * c->obj_bytes);     // objects allowed at 75 %
+  if (c->objs.size() <= keep) return 0;
   struct Cand {
     int needed;
-    uint64_t k1, k2;
-    std::pair<uint32_t, uint32_t> key;
+    uint64_t k1, k2, key;
+    bool operator<(const Cand& b) const {
+      if (needed != b.needed) return needed < b.needed;
+      if (k1 != b.k1) return k1 < b.k1;
+      if (k2 != b.k2) return k2 < b.k2;
+      return key < b.key;
+    }
   };
-  if (static_cast<uint64_t>(c->objs.size()) * c->obj_bytes * 4 <= c->budget * 3) return 0;   // at or below 75 %
   std::vector<Cand> cand;
   cand.reserve(c->objs.size());
   for (const auto& kv : c->objs) {
@@ -127,21 +134,14 @@ size_t evict_to_threshold(sand_view::ObjCache* c, uint64_t epoch, uint64_t chunk
     if (needed) cand.push_back({1, ~o.next_epoch, o.last_batch, kv.first});
     else cand.push_back({0, o.last_batch, 0, kv.first});
   }
-  std::sort(cand.begin(), cand.end(), [](const Cand& a, const Cand& b) {
-    if (a.needed != b.needed) return a.needed < b.needed;
-    if (a.k1 != b.k1) return a.k1 < b.k1;
-    if (a.k2 != b.k2) return a.k2 < b.k2;
-    return a.key < b.key;
-  });
-  size_t n = 0;
-  for (const Cand& x : cand) {
-    if (static_cast<uint64_t>(c->objs.size()) * c->obj_bytes * 4 <= c->budget * 3) break;
-    auto it = c->objs.find(x.key);
+  const size_t n = std::min<size_t>(cand.size(), c->objs.size() - keep);
+  std::partial_sort(cand.begin(), cand.begin() + n, cand.end());   // the n first victims, in order
+  for (size_t i = 0; i < n; ++i) {
+    auto it = c->objs.find(cand[i].key);
     c->free_slots.push_back(it->second.slot);
     c->objs.erase(it);
-    c->stats.evictions++;
-    ++n;
   }
+  c->stats.evictions += n;
   return n;
 }
 
@@ -208,7 +208,7 @@ int objcache_read(sand_view* v, EpochPlan& plan, uint64_t it, const LaunchParams
     }
     const VideoEntry* ent = v->entries[m.clip / s.samples_per_video];
     const uint32_t frame = static_cast<uint32_t>((w.y_off - ent->offset) / ent->frame_stride);
-    const auto key = std::make_pair(ent->id, frame);
+    const uint64_t key = (static_cast<uint64_t>(ent->id) << 32) | frame;
     const uint32_t later = w.pad >> 16, next_delta = w.pad & 0xffffu;
     auto found = c->objs.find(key);
     bool cached = found != c->objs.end();

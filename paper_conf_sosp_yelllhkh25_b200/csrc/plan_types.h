@@ -69,6 +69,11 @@ struct ViewConst {
   float a[3], b[3];      // y = fmaf(q, a_c, b_c)  (R#17)
   int32_t dtype;         // SAND_U8 / SAND_BF16 / SAND_F32
   int32_t T, out_h, out_w;
+  // b'_c = b_c - 2^23 a_c when exactly representable for every channel (fold = 1): then
+  // fmaf(2^23 + q, a_c, b'_c) == fmaf(q, a_c, b_c) exactly (the real values are equal and fmaf
+  // rounds once), so the kernels normalise the biased rint result without un-biasing it
+  float bf[3];
+  int32_t fold;
 };
 
 // Per-batch launch shape of the direct (no rotation/blur) items, from the plan.
@@ -94,6 +99,7 @@ struct BatchShape {
   // k_plain: the batch's task slice, the widest staged span (pixels) and the longest band
   uint32_t task_first, n_tasks;
   int32_t pl_gw, pl_rb;
+  int32_t fold;             // every view's normalisation folds the rint bias (ViewConst::fold)
 };
 
 // k_plain task granularity (view.cpp builds the tasks, k_plain.cuh consumes them)

@@ -188,6 +188,8 @@ void shape_items(const sand_view& v, std::vector<WorkItem>& items, const std::ve
                  const std::vector<uint32_t>& dests, const ViewConst* views, uint32_t n_views, std::vector<uint2>* tasks,
                  BatchShape* shape) {
   BatchShape sh{};
+  sh.fold = 1;
+  for (uint32_t k = 0; k < n_views; ++k) sh.fold &= views[k].fold;
   sh.direct_identity = 1;
   sh.src_w_mod4 = 1;
   sh.even_wo = sh.wo_mod4 = 1;
@@ -225,7 +227,6 @@ void shape_items(const sand_view& v, std::vector<WorkItem>& items, const std::ve
       }
     }
   }
-  (void)n_views;
   if (sh.dtype == -2) sh.dtype = -1;
   auto mid = std::stable_partition(items.begin(), items.end(), [](const WorkItem& w) { return !(w.flags & 1u); });
   sh.n_direct = static_cast<uint32_t>(mid - items.begin());
@@ -285,6 +286,8 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
   }
   for (uint64_t it = 0; it < plan->iterations; ++it) {
     BatchShape shape{};
+    shape.fold = 1;
+    for (uint32_t k = 0; k < s.n_views; ++k) shape.fold &= v.vconst[k].fold;
     shape.direct_identity = 1;
     shape.src_w_mod4 = 1;
     shape.dtype = common_dtype;
@@ -727,9 +730,13 @@ extern "C" int sand_view_create(sand_store* s, const sand_view_spec* spec, sand_
   for (uint32_t k = 0; k < spec->n_views; ++k) {
     const sand_view_desc& vd = spec->views[k];
     sand::ViewConst& c = v->vconst[k];
+    c.fold = 1;
     for (int ch = 0; ch < 3; ++ch) {   // normalisation constants in double, cast once (R#17)
       c.a[ch] = static_cast<float>(1.0 / (255.0 * vd.std[ch]));
       c.b[ch] = static_cast<float>(-vd.mean[ch] / vd.std[ch]);
+      const double bf = static_cast<double>(c.b[ch]) - std::ldexp(static_cast<double>(c.a[ch]), 23);
+      c.bf[ch] = static_cast<float>(bf);
+      if (static_cast<double>(c.bf[ch]) != bf) c.fold = 0;
     }
     c.dtype = vd.out_dtype;
     c.T = static_cast<int32_t>(vd.clip_len);
