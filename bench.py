@@ -107,14 +107,37 @@ def measured_peaks():
 CLASS_KERNELS = {"slowfast": ("k_copy", "k_direct", "k_stencil2")}
 
 
-def ncu_traffic(config: str):
-    """DRAM bytes per launch of the dominant kernel from the committed ncu --set full summary."""
+def ncu_record(config: str):
+    """The committed ncu --set full record of a config's dominant kernel (profiles/ncu_traffic.json)."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(p):
-        d = json.load(open(p))
-        if config in d:
-            return d[config].get("dram_bytes_per_launch")
+        return json.load(open(p)).get(config)
     return None
+
+
+def ncu_traffic(config: str):
+    """DRAM bytes per launch of the dominant kernel from the committed ncu --set full summary."""
+    r = ncu_record(config)
+    return r.get("dram_bytes_per_launch") if r else None
+
+
+def alu_roofline(config, per_class, sm_count, clock_mhz):
+    """Instruction-issue roofline of the dominant kernel: its warp instructions per
+    launch (ncu) over its own event-timed duration, against the issue peak of one warp
+    instruction per SM sub-partition per clock (148 SMs x 4 x clock); with the ALU pipe's share."""
+    r = ncu_record(config)
+    if not r or not r.get("warp_inst_per_launch"):
+        return None
+    name = r["kernel"].replace("void ", "").split("<")[0]
+    ms = next((v["ms_per_launch"] for k, v in per_class.items() if k == name), None)
+    if ms is None:
+        return None
+    peak = sm_count * 4 * clock_mhz * 1e6
+    achieved = r["warp_inst_per_launch"] / (ms / 1e3)
+    return {"bound": "alu", "kernel": name, "achieved": achieved, "peak": peak, "unit": "warp-inst/s",
+            "frac": achieved / peak, "alu_pipe_pct_ncu": r.get("alu_pipe_pct"),
+            "fma_pipe_pct_ncu": r.get("fma_pipe_pct"), "issue_active_pct_ncu": r.get("issue_active_pct"),
+            "source": "warp instructions per launch from " + r.get("source", "profiles/")}
 
 
 # ------------------------------------------------------------------ the oracle (cpu_baseline / reference arm)
@@ -171,7 +194,8 @@ def _oracle_spec(spec):
                              short_side=v.short_side, out_h=v.out_h, out_w=v.out_w, flip_p=v.flip_p,
                              rot_p=v.rot_p, rot_max_deg=v.rot_max_deg, blur_p=v.blur_p, sigma=v.sigma,
                              blur_ksize=v.blur_ksize, blur_truncate=v.blur_truncate, mean=v.mean, std=v.std,
-                             out_dtype=v.out_dtype, subsample_of=v.subsample_of) for v in spec.views]
+                             out_dtype=v.out_dtype, subsample_of=v.subsample_of,
+                             color_matrix=v.color_matrix) for v in spec.views]
     return oracle.make_spec(oracle.SpecDesc(seed=spec.seed, world_size=spec.world_size,
                                             batch_size=spec.batch_size, samples_per_video=spec.samples_per_video,
                                             drop_last=spec.drop_last, shared_window=spec.shared_window, pool_epochs=spec.pool_epochs,
@@ -426,6 +450,8 @@ def run_sand(args):
                      "step": {"achieved": step_achieved, "frac": step_achieved / peak, "kernel_ms_per_step": kernel_ms,
                               "alg_bytes": {"read": alg_read, "write": alg_write}},
                      "peak_source": peak_src, "frac_of_8tbs_spec": achieved / 8000.0},
+        "roofline_alu": alu_roofline(args.config, per_class, torch.cuda.get_device_properties(local).multi_processor_count,
+                                     float(clk.get("sm_max_mhz") or 1965.0)),
         "gpu_launches": int(launches),
         "object_cache": (None if not args.object_budget_gb else
                          {k: int(getattr(view.object_stats(), k)) for k in

@@ -53,6 +53,7 @@ enum {
 };
 enum { SAND_U8 = 0, SAND_BF16 = 1, SAND_F32 = 2 };             /* output dtypes */
 enum { SAND_GEOM_RRC = 0, SAND_GEOM_SHORTSIDE_CROP = 1 };      /* view geometry */
+enum { SAND_BT601 = 0, SAND_BT709 = 1 };                        /* YUV -> RGB matrix (R#11, R#29) */
 
 typedef struct sand_store sand_store; /* opaque; owns the device frame slab */
 typedef struct sand_view sand_view;   /* opaque; a view group over one clip stream */
@@ -163,6 +164,8 @@ typedef struct {
                                T frames are view k's frames at positions floor(t (T_k - 1) / (T - 1))
                                (PySlowFast linspace slow pathway); view k
                                must itself draw from the pool; stride/pool_offset are unused */
+  int32_t color_matrix;     /* SAND_BT601 (R#11, OpenCV's integer form) or SAND_BT709 (R#29); every
+                               view of a spec uses the same matrix (the decoder's colour space) */
 } sand_view_desc;
 
 typedef struct {

@@ -38,7 +38,7 @@ class View(ctypes.Structure):
         ("blur_p", ctypes.c_double), ("sigma_min", ctypes.c_double), ("sigma_max", ctypes.c_double),
         ("blur_ksize", ctypes.c_uint32), ("blur_truncate", ctypes.c_double),
         ("mean", ctypes.c_double * 3), ("std", ctypes.c_double * 3),
-        ("out_dtype", ctypes.c_int32), ("subsample_of", ctypes.c_int32),
+        ("out_dtype", ctypes.c_int32), ("subsample_of", ctypes.c_int32), ("color_matrix", ctypes.c_int32),
     ]
 
 
@@ -108,7 +108,7 @@ def lib():
             "oracle_plan_clip": (None, [P(Spec), P(VideoInfo), u64, u32, P(ClipMeta)]),
             "oracle_iterations": (u64, [P(Spec), u32]),
             "oracle_plan_batch": (ctypes.c_int, [P(Spec), P(VideoInfo), u32, u64, u32, u64, P(ClipMeta)]),
-            "oracle_nv12_to_rgb": (None, [vp, ctypes.c_size_t, vp, ctypes.c_size_t, u32, u32, vp]),
+            "oracle_nv12_to_rgb": (None, [vp, ctypes.c_size_t, vp, ctypes.c_size_t, u32, u32, ctypes.c_int, vp]),
             "oracle_resize": (None, [vp, u32, u32, u32, u32, vp]),
             "oracle_resized_crop": (None, [vp, u32, u32, P(i32), u32, u32, vp]),
             "oracle_shortside_crop": (None, [vp, u32, u32, P(i32), u32, u32, vp]),
@@ -177,12 +177,13 @@ def partition(perm: np.ndarray, world: int, rank: int, drop_last: bool) -> np.nd
     return out[:k].copy()
 
 
-def nv12_to_rgb(y: np.ndarray, uv: np.ndarray) -> np.ndarray:
+def nv12_to_rgb(y: np.ndarray, uv: np.ndarray, matrix: int = 0) -> np.ndarray:
+    """matrix 0: BT.601 (R#11, OpenCV's integer form); 1: BT.709 (R#29)."""
     H, W = y.shape
     y = np.ascontiguousarray(y)
     uv = np.ascontiguousarray(uv)
     out = np.empty((H, W, 3), np.uint8)
-    lib().oracle_nv12_to_rgb(_u8p(y), W, _u8p(uv), W, W, H, _u8p(out))
+    lib().oracle_nv12_to_rgb(_u8p(y), W, _u8p(uv), W, W, H, matrix, _u8p(out))
     return out
 
 
@@ -292,6 +293,7 @@ class ViewDesc:
     std: tuple = (0.229, 0.224, 0.225)
     out_dtype: int = BF16
     subsample_of: int = -1
+    color_matrix: int = 0
 
 
 @dataclass
@@ -331,6 +333,7 @@ def make_spec(sd: SpecDesc) -> Spec:
             o.std[c] = v.std[c]
         o.out_dtype = v.out_dtype
         o.subsample_of = v.subsample_of
+        o.color_matrix = v.color_matrix
     return s
 
 

@@ -54,6 +54,7 @@ typedef struct {
   double mean[3], std[3];
   int32_t out_dtype;               /* OR_U8 / OR_BF16 / OR_F32 */
   int32_t subsample_of;            /* -1: pool view; k: linspace sub-sample of view k (R#26) */
+  int32_t color_matrix;            /* 0: BT.601 (R#11), 1: BT.709 (R#29) */
 } oracle_view;
 
 typedef struct {
@@ -415,20 +416,27 @@ int oracle_plan_batch(const oracle_spec* spec, const oracle_video_info* dataset,
 /* ------------------------------------------------------------------------- */
 static uint8_t sat_u8(int32_t v) { return (uint8_t)(v < 0 ? 0 : (v > 255 ? 255 : v)); }
 
+/* matrix 0: BT.601 limited range, OpenCV's COLOR_YUV2RGB_NV12 integer form (R#11).
+   matrix 1: BT.709 limited range (R#29): the same form with coefficients round(c * 2^20) of the
+   ITU-R BT.709 matrix (Kr = 0.2126, Kb = 0.0722; luma scale 255/219, chroma scale 255/224):
+   cy = 1.16438 -> 1220945, V->R 1.79274 -> 1879825, V->G -0.53291 -> -558796,
+   U->G -0.21325 -> -223607, U->B 2.11240 -> 2215014. */
 void oracle_nv12_to_rgb(const uint8_t* yp, size_t y_pitch, const uint8_t* uvp, size_t uv_pitch,
-                        uint32_t W, uint32_t H, uint8_t* rgb) {
+                        uint32_t W, uint32_t H, int matrix, uint8_t* rgb) {
+  const int32_t cy = matrix ? 1220945 : 1220542, vr = matrix ? 1879825 : 1673527;
+  const int32_t vg = matrix ? -558796 : -852492, ug = matrix ? -223607 : -409993, ub = matrix ? 2215014 : 2116026;
   for (uint32_t y = 0; y < H; ++y) {
     for (uint32_t x = 0; x < W; ++x) {
       int32_t Y = yp[(size_t)y * y_pitch + x];
       int32_t U = uvp[(size_t)(y >> 1) * uv_pitch + 2 * (x >> 1)];
       int32_t V = uvp[(size_t)(y >> 1) * uv_pitch + 2 * (x >> 1) + 1];
       int32_t u = U - 128, v = V - 128;
-      int32_t yy = (Y - 16 > 0 ? Y - 16 : 0) * 1220542;
+      int32_t yy = (Y - 16 > 0 ? Y - 16 : 0) * cy;
       int32_t half = 1 << 19;
       uint8_t* px = rgb + ((size_t)y * W + x) * 3;
-      px[0] = sat_u8((yy + half + 1673527 * v) >> 20);
-      px[1] = sat_u8((yy + half - 852492 * v - 409993 * u) >> 20);
-      px[2] = sat_u8((yy + half + 2116026 * u) >> 20);
+      px[0] = sat_u8((yy + half + vr * v) >> 20);
+      px[1] = sat_u8((yy + half + vg * v + ug * u) >> 20);
+      px[2] = sat_u8((yy + half + ub * u) >> 20);
     }
   }
 }
@@ -632,7 +640,7 @@ void oracle_render_frame(const oracle_spec* spec, const oracle_clip_meta* meta, 
   uint8_t* rgb = (uint8_t*)malloc((size_t)W * H * 3);
   uint8_t* a = (uint8_t*)malloc(n);
   uint8_t* b = (uint8_t*)malloc(n);
-  oracle_nv12_to_rgb(yp, y_pitch, uvp, uv_pitch, W, H, rgb);
+  oracle_nv12_to_rgb(yp, y_pitch, uvp, uv_pitch, W, H, v->color_matrix, rgb);
   if (v->geom == OR_GEOM_RRC)
     oracle_resized_crop(rgb, W, H, meta->box[q], Ho, Wo, a);
   else

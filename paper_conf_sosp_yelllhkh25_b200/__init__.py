@@ -62,6 +62,7 @@ def make_spec(spec: Spec, videos) -> tuple[_abi.sand_view_spec, object]:
             o.std[c] = v.std[c]
         o.out_dtype = v.out_dtype
         o.subsample_of = int(getattr(v, "subsample_of", -1))
+        o.color_matrix = int(getattr(v, "color_matrix", 0))
     return s, arr
 
 

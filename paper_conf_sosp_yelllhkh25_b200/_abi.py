@@ -43,7 +43,7 @@ class sand_view_desc(ctypes.Structure):
         ("flip_p", dbl), ("rot_p", dbl), ("rot_max_deg", dbl),
         ("blur_p", dbl), ("sigma_min", dbl), ("sigma_max", dbl),
         ("blur_ksize", u32), ("blur_truncate", dbl),
-        ("mean", dbl * 3), ("std", dbl * 3), ("out_dtype", i32), ("subsample_of", i32),
+        ("mean", dbl * 3), ("std", dbl * 3), ("out_dtype", i32), ("subsample_of", i32), ("color_matrix", i32),
     ]
 
 

@@ -9,6 +9,7 @@ from __future__ import annotations
 from dataclasses import dataclass, field, replace
 
 U8, BF16, F32 = 0, 1, 2
+BT601, BT709 = 0, 1
 GEOM_RRC, GEOM_SHORTSIDE_CROP = 0, 1
 
 KINETICS_MEAN, KINETICS_STD = (0.45, 0.45, 0.45), (0.225, 0.225, 0.225)
@@ -38,6 +39,7 @@ class ViewSpec:
     std: tuple = IMAGENET_STD
     out_dtype: int = BF16
     subsample_of: int = -1        # >= 0: linspace sub-sample of that view's frames (f4, R#26)
+    color_matrix: int = BT601     # YUV -> RGB matrix: BT601 (R#11) or BT709 (f4, R#29)
 
 
 @dataclass
@@ -100,6 +102,16 @@ def slowfast_linspace() -> Workload:
     return w
 
 
+def k400_two_samples() -> Workload:
+    """Fig. 9's `samples_per_video: 2`: two clips per video per epoch, each with its own
+    temporal and spatial draws (global clip id = video * 2 + sample)."""
+    w = k400()
+    w.name = "k400_two_samples"
+    w.spec.samples_per_video = 2
+    w.description = "Kinetics-400-shaped with two sampled clips per video per epoch (Fig. 9 samples_per_video: 2)"
+    return w
+
+
 def slowfast_hd() -> Workload:
     """SlowFast on 1280x720 sources: short side 256 gives W' = floor(1280 * 256 / 720) = 455, a
     real down-scaling by 2.81 on both axes (SURVEY §8(c) reading 10's variant)."""
@@ -126,7 +138,7 @@ def ray() -> Workload:
 
 
 WORKLOADS = {"tiny": tiny, "k400": k400, "slowfast": slowfast, "twoview": twoview, "ray": ray,
-             "slowfast_hd": slowfast_hd, "slowfast_linspace": slowfast_linspace}
+             "slowfast_hd": slowfast_hd, "slowfast_linspace": slowfast_linspace, "k400_two_samples": k400_two_samples}
 
 
 def get(name: str) -> Workload:

@@ -17,8 +17,8 @@ namespace cp {
 
 // one NV12 pixel (luma Y, chroma terms k) -> three biased floats 2^23 + channel (R#11), the
 // same DPX add-min-relu + IMAD.HI formulation as the other kernels
-__device__ __forceinline__ void px(uint32_t Y, const st::Chroma3& k, uint32_t (&c)[3]) {
-  const int yy = (int)max(Y, 16u) * 1220542 + ((1 << 19) - 16 * 1220542);
+__device__ __forceinline__ void px(uint32_t Y, const st::Chroma3& k, uint32_t (&c)[3], const ColorM& m) {
+  const int yy = (int)max(Y, 16u) * m.cy + ((1 << 19) - 16 * m.cy);
   c[0] = __umulhi((uint32_t)__viaddmin_s32_relu(yy, k.r, 0x0FFFFFFF), 1u << 12) + 0x4B000000u;
   c[1] = __umulhi((uint32_t)__viaddmin_s32_relu(yy, k.g, 0x0FFFFFFF), 1u << 12) + 0x4B000000u;
   c[2] = __umulhi((uint32_t)__viaddmin_s32_relu(yy, k.b, 0x0FFFFFFF), 1u << 12) + 0x4B000000u;
@@ -73,20 +73,20 @@ __global__ void __launch_bounds__(256) k_copy(const LaunchParams p, int RB, int 
     const uint32_t u_hi = (odd || b0) ? __ldg(reinterpret_cast<const uint32_t*>(uvrow + ya + 4)) : 0u;
     const uint64_t uvw = ((uint64_t)u_hi << 32) | u_lo;
     st::Chroma3 k[3];                                     // even sx: 2 samples; odd sx: 3
-    k[0] = st::chroma_at<0>((uint32_t)(uvw >> (8 * b0)));
-    k[1] = st::chroma_at<0>((uint32_t)(uvw >> (8 * b0 + 16)));
-    if (odd) k[2] = st::chroma_at<0>((uint32_t)(uvw >> (8 * b0 + 32)));
+    k[0] = st::chroma_at<0>((uint32_t)(uvw >> (8 * b0)), p.cm);
+    k[1] = st::chroma_at<0>((uint32_t)(uvw >> (8 * b0 + 16)), p.cm);
+    if (odd) k[2] = st::chroma_at<0>((uint32_t)(uvw >> (8 * b0 + 32)), p.cm);
     uint32_t c[4][3];                                     // source pixels sx .. sx+3
     if (!odd) {
-      cp::px(ys & 0xffu, k[0], c[0]);
-      cp::px((ys >> 8) & 0xffu, k[0], c[1]);
-      cp::px((ys >> 16) & 0xffu, k[1], c[2]);
-      cp::px(ys >> 24, k[1], c[3]);
+      cp::px(ys & 0xffu, k[0], c[0], p.cm);
+      cp::px((ys >> 8) & 0xffu, k[0], c[1], p.cm);
+      cp::px((ys >> 16) & 0xffu, k[1], c[2], p.cm);
+      cp::px(ys >> 24, k[1], c[3], p.cm);
     } else {
-      cp::px(ys & 0xffu, k[0], c[0]);
-      cp::px((ys >> 8) & 0xffu, k[1], c[1]);
-      cp::px((ys >> 16) & 0xffu, k[1], c[2]);
-      cp::px(ys >> 24, k[2], c[3]);
+      cp::px(ys & 0xffu, k[0], c[0], p.cm);
+      cp::px((ys >> 8) & 0xffu, k[1], c[1], p.cm);
+      cp::px((ys >> 16) & 0xffu, k[1], c[2], p.cm);
+      cp::px(ys >> 24, k[2], c[3], p.cm);
     }
     // output column ox + j holds source pixel j (or 3 - j under flip)
     if (g.flip) {                                         // output column ox + j <- source pixel 3 - j

@@ -22,9 +22,9 @@ namespace dg {
 struct Px3 {
   uint32_t c[3];
 };
-__device__ __forceinline__ Px3 px3(uint32_t Y, uint32_t uv) {
-  const st::Chroma3 k = st::chroma_at<0>(uv);
-  const int yy = (int)max(Y, 16u) * 1220542 + ((1 << 19) - 16 * 1220542);
+__device__ __forceinline__ Px3 px3(uint32_t Y, uint32_t uv, const ColorM& m) {
+  const st::Chroma3 k = st::chroma_at<0>(uv, m);
+  const int yy = (int)max(Y, 16u) * m.cy + ((1 << 19) - 16 * m.cy);
   Px3 p;
   p.c[0] = __umulhi((uint32_t)__viaddmin_s32_relu(yy, k.r, 0x0FFFFFFF), 1u << 12) + 0x4B000000u;
   p.c[1] = __umulhi((uint32_t)__viaddmin_s32_relu(yy, k.g, 0x0FFFFFFF), 1u << 12) + 0x4B000000u;
@@ -44,7 +44,7 @@ __device__ __forceinline__ uint64_t hlerp_b(uint32_t a0, uint32_t a1, uint32_t b
 template <int NR>
 __device__ __forceinline__ void hrows(rs::Row3* out, const uint8_t* __restrict__ Yp, const uint8_t* __restrict__ UVp,
                                       uint32_t pitch, const int (&ys)[2], int xa0, int xa1, int xb0, int xb1,
-                                      uint64_t lx) {
+                                      uint64_t lx, const ColorM& cm) {
   const int xs[4] = {xa0, xa1, xb0, xb1};
   uint32_t Y[NR][4], UV[NR][4];
 #pragma unroll
@@ -61,7 +61,7 @@ __device__ __forceinline__ void hrows(rs::Row3* out, const uint8_t* __restrict__
   for (int r = 0; r < NR; ++r) {
     Px3 q[4];
 #pragma unroll
-    for (int k = 0; k < 4; ++k) q[k] = px3(Y[r][k], UV[r][k]);
+    for (int k = 0; k < 4; ++k) q[k] = px3(Y[r][k], UV[r][k], cm);
 #pragma unroll
     for (int c = 0; c < 3; ++c) out[r].h[c] = hlerp_b(q[0].c[c], q[1].c[c], q[2].c[c], q[3].c[c], lx);
   }
@@ -154,7 +154,7 @@ __global__ void __launch_bounds__(256, SAND_DIRECT_MINB) k_direct(const LaunchPa
         for (int r = 0; r < 2; ++r) {
           dg::Px3 q[4];
 #pragma unroll
-          for (int k = 0; k < 4; ++k) q[k] = dg::px3(Yc[r][k], UVc[r][k]);
+          for (int k = 0; k < 4; ++k) q[k] = dg::px3(Yc[r][k], UVc[r][k], p.cm);
 #pragma unroll
           for (int c = 0; c < 3; ++c) tb[r].h[c] = dg::hlerp_b(q[0].c[c], q[1].c[c], q[2].c[c], q[3].c[c], lx);
         }
@@ -181,7 +181,7 @@ __global__ void __launch_bounds__(256, SAND_DIRECT_MINB) k_direct(const LaunchPa
       const int ys2[2] = {y0, y1};
       if (y0 != yT && y0 != yB && y1 != yB && y1 != y0) {   // both rows new (the usual case)
         Row3 tb[2];
-        dg::hrows<2>(tb, Yp, UVp, pitch, ys2, xa0, xa1, xb0, xb1, lx);
+        dg::hrows<2>(tb, Yp, UVp, pitch, ys2, xa0, xa1, xb0, xb1, lx, p.cm);
         T = tb[0];
         B = tb[1];
         yT = y0;
@@ -191,7 +191,7 @@ __global__ void __launch_bounds__(256, SAND_DIRECT_MINB) k_direct(const LaunchPa
         if (y0 == yB) {
           T = B;
         } else {
-          dg::hrows<1>(&T, Yp, UVp, pitch, ys2, xa0, xa1, xb0, xb1, lx);
+          dg::hrows<1>(&T, Yp, UVp, pitch, ys2, xa0, xa1, xb0, xb1, lx, p.cm);
         }
         yT = y0;
       }
@@ -200,7 +200,7 @@ __global__ void __launch_bounds__(256, SAND_DIRECT_MINB) k_direct(const LaunchPa
           B = T;
         } else {
           const int ys1[2] = {y1, y1};
-          dg::hrows<1>(&B, Yp, UVp, pitch, ys1, xa0, xa1, xb0, xb1, lx);
+          dg::hrows<1>(&B, Yp, UVp, pitch, ys1, xa0, xa1, xb0, xb1, lx, p.cm);
         }
         yB = y1;
       }

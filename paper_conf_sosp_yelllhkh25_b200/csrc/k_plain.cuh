@@ -78,6 +78,7 @@ __global__ void __launch_bounds__(PlainBounds<NP>::kThreads, PlainBounds<NP>::kM
   const float sc_x = g.sc_x, sc_y = g.sc_y;
   const int off_x = g.off_x, off_y = g.off_y, org_x = g.org_x, org_y = g.org_y;
   const int lim_x = g.lim_x, lim_y = g.lim_y, flip = g.flip;
+  const ColorM cm = p.cm;                                          // YUV -> RGB matrix (R#11 / R#29)
 
   uint32_t s_base = (uint32_t)__cvta_generic_to_shared(smem_raw);
   asm volatile("" : "+r"(s_base));
@@ -221,18 +222,18 @@ __global__ void __launch_bounds__(PlainBounds<NP>::kThreads, PlainBounds<NP>::kM
       for (int u = 0; u < nuv; ++u) {
         const int yt = 2 * (u0 + u);                       // top Y row of this UV row
         const uint32_t uv = *reinterpret_cast<const uint32_t*>(raw + (uint32_t)(ny + u) * rawpitch);
-        const st::Chroma3 c0 = st::chroma_at<0>(uv), c1 = st::chroma_at<16>(uv);
+        const st::Chroma3 c0 = st::chroma_at<0>(uv, cm), c1 = st::chroma_at<16>(uv, cm);
         uint8_t* out = conv + ((uint32_t)yt - slot0) * rowbytes;   // row yt
         if (yt >= ya) {
           const uint32_t yw = *reinterpret_cast<const uint32_t*>(raw + (uint32_t)(yt - ya) * rawpitch);
-          *reinterpret_cast<uint4*>(out) = make_uint4(st::rgbx_dpx(st::byte_of<0>(yw), c0), st::rgbx_dpx(st::byte_of<1>(yw), c0),
-                                                      st::rgbx_dpx(st::byte_of<2>(yw), c1), st::rgbx_dpx(st::byte_of<3>(yw), c1));
+          *reinterpret_cast<uint4*>(out) = make_uint4(st::rgbx_dpx(st::byte_of<0>(yw), c0, cm), st::rgbx_dpx(st::byte_of<1>(yw), c0, cm),
+                                                      st::rgbx_dpx(st::byte_of<2>(yw), c1, cm), st::rgbx_dpx(st::byte_of<3>(yw), c1, cm));
         }
         if (yt + 1 <= yb) {
           const uint32_t yw = *reinterpret_cast<const uint32_t*>(raw + (uint32_t)(yt + 1 - ya) * rawpitch);
           *reinterpret_cast<uint4*>(out + rowbytes) =
-              make_uint4(st::rgbx_dpx(st::byte_of<0>(yw), c0), st::rgbx_dpx(st::byte_of<1>(yw), c0),
-                         st::rgbx_dpx(st::byte_of<2>(yw), c1), st::rgbx_dpx(st::byte_of<3>(yw), c1));
+              make_uint4(st::rgbx_dpx(st::byte_of<0>(yw), c0, cm), st::rgbx_dpx(st::byte_of<1>(yw), c0, cm),
+                         st::rgbx_dpx(st::byte_of<2>(yw), c1, cm), st::rgbx_dpx(st::byte_of<3>(yw), c1, cm));
         }
       }
     }

@@ -30,24 +30,6 @@ __device__ __forceinline__ int tap0(float sc, int off, int o, int org) {
   return org + (int)fmaxf(s, 0.f);
 }
 
-// chroma terms of one (U,V) pair, shared by the pixels of a 2x2 block (R#11)
-struct Chroma {
-  int r, g, b;
-};
-__device__ __forceinline__ Chroma chroma(uint32_t uvpair) {
-  const int u = (int)(uvpair & 0xffu) - 128;
-  const int v = (int)((uvpair >> 8) & 0xffu) - 128;
-  return {1673527 * v, -852492 * v - 409993 * u, 2116026 * u};
-}
-__device__ __forceinline__ int sat8(int x) { return min(max(x, 0), 255); }
-// RGBx word: R | G << 8 | B << 16 | 0x4B << 24. The top byte is the exponent byte of 2^23,
-// so a channel becomes the float 2^23 + value with one byte permute (see biased()).
-__device__ __forceinline__ uint32_t rgbx(int Y, const Chroma& c) {
-  const int yy = max(Y - 16, 0) * 1220542 + (1 << 19);
-  return (uint32_t)sat8((yy + c.r) >> 20) | ((uint32_t)sat8((yy + c.g) >> 20) << 8) |
-         ((uint32_t)sat8((yy + c.b) >> 20) << 16) | 0x4B000000u;
-}
-
 // byte C of an RGBx word as the float 2^23 + byte (exact): result bytes = [w.C, 0, 0, w.3]
 template <int C>
 __device__ __forceinline__ float biased(uint32_t w) {

@@ -606,7 +606,7 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
     band(oy_lo, nr, y_lo, y_hi);
     asm volatile("cp.async.wait_group 0;\n" ::: "memory");
     __syncthreads();                          // raw of this band landed; the previous walk is done with grid/rtab
-    st::convert_rows(s_grid, s_rawb, gw, y_lo, y_hi, y_lo, 1 << 30, 5u, warp, nwarps, lane);   // no wrap
+    st::convert_rows(s_grid, s_rawb, gw, y_lo, y_hi, y_lo, 1 << 30, 5u, warp, nwarps, lane, p.cm);   // no wrap
     for (int r = tid; r < nr; r += nthr) {
       int y0, y1;
       float ly;

@@ -114,23 +114,23 @@ __device__ __forceinline__ void stage_rows_cp(uint32_t raw, const uint8_t* y0, c
   asm volatile("cp.async.commit_group;\n" ::: "memory");
 }
 
-// chroma terms (R#11) of the sample whose U is at bit SHIFT of the UV word
+// chroma terms (R#11 / R#29, matrix m) of the sample whose U is at bit SHIFT of the UV word
 struct Chroma3 {
   int r, g, b;
 };
 template <int SHIFT>
-__device__ __forceinline__ Chroma3 chroma_at(uint32_t uv) {
+__device__ __forceinline__ Chroma3 chroma_at(uint32_t uv, const ColorM& m) {
   const int u = (int)((uv >> SHIFT) & 0xffu) - 128;
   const int v = (int)((uv >> (SHIFT + 8)) & 0xffu) - 128;
-  return {1673527 * v, -852492 * v - 409993 * u, 2116026 * u};
+  return {m.vr * v, m.vg * v + m.ug * u, m.ub * u};
 }
 
 // RGBx word of luma Y with chroma c: sat((yy + term) >> 20) per channel (OpenCV integer
 // BT.601), computed as relu(min(yy + term, 2^28 - 1)) >> 4 (one DPX VIADDMNMX.RELU), whose
 // byte 2 is the channel; PRMT gathers the three bytes and the exponent byte 0x4B tops the word
 // (see rs::biased).
-__device__ __forceinline__ uint32_t rgbx_dpx(uint32_t Y, const Chroma3& c) {
-  const int yy = (int)max(Y, 16u) * 1220542 + ((1 << 19) - 16 * 1220542);
+__device__ __forceinline__ uint32_t rgbx_dpx(uint32_t Y, const Chroma3& c, const ColorM& m) {
+  const int yy = (int)max(Y, 16u) * m.cy + ((1 << 19) - 16 * m.cy);
   // x >> 4 of the clamped sums as IMAD.HI (FMA pipe) to relieve the ALU pipe
   const uint32_t mr = __umulhi((uint32_t)__viaddmin_s32_relu(yy, c.r, 0x0FFFFFFF), 1u << 28);
   const uint32_t mg = __umulhi((uint32_t)__viaddmin_s32_relu(yy, c.g, 0x0FFFFFFF), 1u << 28);
@@ -146,7 +146,8 @@ __device__ __forceinline__ uint32_t byte_of(uint32_t w) {
 
 // convert staged rows [ya, yb] into the ring (slot = (y - y_first) % ring_rows)
 __device__ __forceinline__ void convert_rows(uint32_t ring, uint32_t raw, int gw, int ya, int yb, int y_first,
-                                             int ring_rows, uint32_t ring_magic, int warp, int nwarps, int lane) {
+                                             int ring_rows, uint32_t ring_magic, int warp, int nwarps, int lane,
+                                             const ColorM& cm) {
   const int ny = yb - ya + 1;
   if (ny <= 0) return;
   const int u0 = ya >> 1, nuv = (yb >> 1) - u0 + 1;
@@ -163,16 +164,16 @@ __device__ __forceinline__ void convert_rows(uint32_t ring, uint32_t raw, int gw
     const uint32_t uvrow = rawUV + (uint32_t)(u * gw);
     for (int q = lane; q < q4; q += 32) {
       const uint32_t uv = lds32(uvrow + 4 * q);
-      const Chroma3 c0 = chroma_at<0>(uv), c1 = chroma_at<16>(uv);
+      const Chroma3 c0 = chroma_at<0>(uv, cm), c1 = chroma_at<16>(uv, cm);
       if (top) {
         const uint32_t yw = lds32(yrow_t + 4 * q);
-        sts128(out_t + 16 * q, make_uint4(rgbx_dpx(byte_of<0>(yw), c0), rgbx_dpx(byte_of<1>(yw), c0),
-                                          rgbx_dpx(byte_of<2>(yw), c1), rgbx_dpx(byte_of<3>(yw), c1)));
+        sts128(out_t + 16 * q, make_uint4(rgbx_dpx(byte_of<0>(yw), c0, cm), rgbx_dpx(byte_of<1>(yw), c0, cm),
+                                          rgbx_dpx(byte_of<2>(yw), c1, cm), rgbx_dpx(byte_of<3>(yw), c1, cm)));
       }
       if (bot) {
         const uint32_t yw = lds32(yrow_b + 4 * q);
-        sts128(out_b + 16 * q, make_uint4(rgbx_dpx(byte_of<0>(yw), c0), rgbx_dpx(byte_of<1>(yw), c0),
-                                          rgbx_dpx(byte_of<2>(yw), c1), rgbx_dpx(byte_of<3>(yw), c1)));
+        sts128(out_b + 16 * q, make_uint4(rgbx_dpx(byte_of<0>(yw), c0, cm), rgbx_dpx(byte_of<1>(yw), c0, cm),
+                                          rgbx_dpx(byte_of<2>(yw), c1, cm), rgbx_dpx(byte_of<3>(yw), c1, cm)));
       }
     }
   }
@@ -181,7 +182,7 @@ __device__ __forceinline__ void convert_rows(uint32_t ring, uint32_t raw, int gw
 // convert_rows with the (UV row, 4-pixel group) units flattened over all threads of the CTA,
 // so a row width that is not a multiple of 32 groups leaves no lane idle
 __device__ __forceinline__ void convert_rows_flat(uint32_t ring, uint32_t raw, int gw, int ya, int yb, int y_first,
-                                                  int ring_rows, uint32_t ring_magic, int tid, int nthr) {
+                                                  int ring_rows, uint32_t ring_magic, int tid, int nthr, const ColorM& cm) {
   const int ny = yb - ya + 1;
   if (ny <= 0) return;
   const int u0 = ya >> 1, nuv = (yb >> 1) - u0 + 1;
@@ -198,18 +199,18 @@ __device__ __forceinline__ void convert_rows_flat(uint32_t ring, uint32_t raw, i
     const int sb = st + 1 == ring_rows ? 0 : st + 1;
     const uint32_t yrow_t = raw + (uint32_t)((yt - ya) * gw + 4 * q);
     const uint32_t uv = lds32(rawUV + (uint32_t)(u * gw + 4 * q));
-    const Chroma3 c0 = chroma_at<0>(uv), c1 = chroma_at<16>(uv);
+    const Chroma3 c0 = chroma_at<0>(uv, cm), c1 = chroma_at<16>(uv, cm);
     if (yt >= ya) {
       const uint32_t yw = lds32(yrow_t);
       sts128(ring + (uint32_t)st * rowbytes + 16u * q,
-             make_uint4(rgbx_dpx(byte_of<0>(yw), c0), rgbx_dpx(byte_of<1>(yw), c0), rgbx_dpx(byte_of<2>(yw), c1),
-                        rgbx_dpx(byte_of<3>(yw), c1)));
+             make_uint4(rgbx_dpx(byte_of<0>(yw), c0, cm), rgbx_dpx(byte_of<1>(yw), c0, cm), rgbx_dpx(byte_of<2>(yw), c1, cm),
+                        rgbx_dpx(byte_of<3>(yw), c1, cm)));
     }
     if (yt + 1 <= yb) {
       const uint32_t yw = lds32(yrow_t + (uint32_t)gw);
       sts128(ring + (uint32_t)sb * rowbytes + 16u * q,
-             make_uint4(rgbx_dpx(byte_of<0>(yw), c0), rgbx_dpx(byte_of<1>(yw), c0), rgbx_dpx(byte_of<2>(yw), c1),
-                        rgbx_dpx(byte_of<3>(yw), c1)));
+             make_uint4(rgbx_dpx(byte_of<0>(yw), c0, cm), rgbx_dpx(byte_of<1>(yw), c0, cm), rgbx_dpx(byte_of<2>(yw), c1, cm),
+                        rgbx_dpx(byte_of<3>(yw), c1, cm)));
     }
     q += dq;
     u += du;
@@ -450,8 +451,8 @@ __global__ void __launch_bounds__(NP == 1 ? 256 : 128, NP == 1 ? 3 : SAND_NP2_MI
     }
     __syncthreads();                                 // walk(k-1) finished: its ring rows are free
     if (staged) {
-      if (sh.opts & 1) st::convert_rows(s_ring, s_raw, gw, ya, yb, y_first, sh.ring, sh.ring_magic, warp, nthr >> 5, lane);
-      else st::convert_rows_flat(s_ring, s_raw, gw, ya, yb, y_first, sh.ring, sh.ring_magic, tid, nthr);
+      if (sh.opts & 1) st::convert_rows(s_ring, s_raw, gw, ya, yb, y_first, sh.ring, sh.ring_magic, warp, nthr >> 5, lane, p.cm);
+      else st::convert_rows_flat(s_ring, s_raw, gw, ya, yb, y_first, sh.ring, sh.ring_magic, tid, nthr, p.cm);
     }
     staged = false;
     __syncthreads();                                 // ring holds every row of sub-band k; raw drained

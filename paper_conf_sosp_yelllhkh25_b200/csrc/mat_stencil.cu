@@ -20,13 +20,13 @@ constexpr int kStripRows = 32;     // output rows per blur strip
 __device__ __forceinline__ int clamp_u8(int v) { return min(max(v, 0), 255); }
 
 __device__ __forceinline__ int nv12_chan(const uint8_t* __restrict__ Yp, const uint8_t* __restrict__ UVp,
-                                         uint32_t pitch, int x, int y, int c) {
+                                         uint32_t pitch, int x, int y, int c, const ColorM& m) {
   const int Yv = __ldg(Yp + (size_t)y * pitch + x);
   const uint8_t* uvr = UVp + (size_t)(y >> 1) * pitch + (x & ~1);
   const int u = (int)__ldg(uvr) - 128;
   const int v = (int)__ldg(uvr + 1) - 128;
-  const int yy = max(Yv - 16, 0) * 1220542 + (1 << 19);
-  const int t = c == 0 ? 1673527 * v : (c == 1 ? -852492 * v - 409993 * u : 2116026 * u);
+  const int yy = max(Yv - 16, 0) * m.cy + (1 << 19);
+  const int t = c == 0 ? m.vr * v : (c == 1 ? m.vg * v + m.ug * u : m.ub * u);
   return clamp_u8((yy + t) >> 20);
 }
 
@@ -89,10 +89,10 @@ __global__ void __launch_bounds__(512) k_stencil(const LaunchParams p) {
       float lx, ly;
       src_tap(g.sc_x, g.off_x, oxm, g.lim_x, g.org_x, x0, x1, lx);
       src_tap(g.sc_y, g.off_y, oy, g.lim_y, g.org_y, y0, y1, ly);
-      const float h0 = lerp_rn(lx, (float)nv12_chan(Yp, UVp, w.pitch, x0, y0, c),
-                               (float)nv12_chan(Yp, UVp, w.pitch, x1, y0, c));
-      const float h1 = lerp_rn(lx, (float)nv12_chan(Yp, UVp, w.pitch, x0, y1, c),
-                               (float)nv12_chan(Yp, UVp, w.pitch, x1, y1, c));
+      const float h0 = lerp_rn(lx, (float)nv12_chan(Yp, UVp, w.pitch, x0, y0, c, p.cm),
+                               (float)nv12_chan(Yp, UVp, w.pitch, x1, y0, c, p.cm));
+      const float h1 = lerp_rn(lx, (float)nv12_chan(Yp, UVp, w.pitch, x0, y1, c, p.cm),
+                               (float)nv12_chan(Yp, UVp, w.pitch, x1, y1, c, p.cm));
       q2[pix] = (uint8_t)quant(lerp_rn(ly, h0, h1));
     }
     __syncthreads();

@@ -120,6 +120,17 @@ SAND_HD inline void tap_ref(float sc, int off, int o, int lim, int org, int* i0,
   *i1 = org + (i + 1 < lim - 1 ? i + 1 : lim - 1);
 }
 
+// YUV -> RGB coefficients in 2^20 fixed point (R#11 BT.601 / R#29 BT.709): yy = max(Y, 16) cy +
+// (2^19 - 16 cy); R = sat((yy + vr v) >> 20), G = sat((yy + vg v + ug u) >> 20),
+// B = sat((yy + ub u) >> 20), u = U - 128, v = V - 128
+struct ColorM {
+  int32_t cy, vr, vg, ug, ub;
+};
+SAND_HD inline ColorM color_matrix(int32_t m) {
+  return m == 1 ? ColorM{1220945, 1879825, -558796, -223607, 2215014}    // BT.709 from Kr, Kb (R#29)
+                : ColorM{1220542, 1673527, -852492, -409993, 2116026};  // BT.601, OpenCV (R#11)
+}
+
 struct LaunchParams {
   const uint8_t* slab;
   const WorkItem* items;   // this batch's items
@@ -131,6 +142,7 @@ struct LaunchParams {
   uint32_t n_views;
   uint32_t batch;          // B
   const uint2* tasks;      // k_plain tasks of this batch (view.cpp)
+  ColorM cm;               // the spec's YUV -> RGB matrix (kernel-parameter constants)
 };
 
 }  // namespace sand

@@ -79,6 +79,8 @@ int validate_spec(const sand_view_spec& s, std::string* why) {
         (static_cast<uint32_t>(v.subsample_of) >= s.n_views || v.subsample_of == static_cast<int32_t>(k) ||
          s.views[v.subsample_of].subsample_of >= 0))
       return bad("subsample_of must name another view that draws from the pool");
+    if (v.color_matrix != SAND_BT601 && v.color_matrix != SAND_BT709) return bad("unknown color_matrix");
+    if (v.color_matrix != s.views[0].color_matrix) return bad("every view must use the same color_matrix");
   }
   uint32_t g = 0;
   for (uint32_t k = 0; k < s.n_views; ++k)

@@ -1064,6 +1064,7 @@ static int read_batch_direct(sand_view* v, uint64_t epoch, uint32_t rank, const 
   lp.n_views = s.n_views;
   lp.batch = s.batch_size;
   lp.tasks = plan->d_tasks;
+  lp.cm = sand::color_matrix(s.views[0].color_matrix);
   for (uint32_t k = 0; k < s.n_views; ++k) {
     lp.out[k] = out->data[k];
     lp.views[k] = v->vconst[k];

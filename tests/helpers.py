@@ -22,7 +22,8 @@ def to_oracle(spec) -> oracle.Spec:
                              short_side=v.short_side, out_h=v.out_h, out_w=v.out_w, flip_p=v.flip_p,
                              rot_p=v.rot_p, rot_max_deg=v.rot_max_deg, blur_p=v.blur_p, sigma=v.sigma,
                              blur_ksize=v.blur_ksize, blur_truncate=v.blur_truncate, mean=v.mean, std=v.std,
-                             out_dtype=v.out_dtype, subsample_of=v.subsample_of) for v in spec.views]
+                             out_dtype=v.out_dtype, subsample_of=v.subsample_of,
+                             color_matrix=v.color_matrix) for v in spec.views]
     return oracle.make_spec(oracle.SpecDesc(seed=spec.seed, world_size=spec.world_size,
                                             batch_size=spec.batch_size, samples_per_video=spec.samples_per_video,
                                             drop_last=spec.drop_last, shared_window=spec.shared_window, pool_epochs=spec.pool_epochs,

@@ -237,3 +237,23 @@ def test_object_cache_bit_identical_and_policy_matches_oracle(src, budget_objs):
         ref.close()
         view.close()
         store.close()
+
+
+@pytest.mark.parametrize("name", ["k400", "slowfast", "slowfast_hd", "twoview", "ray"])
+def test_bt709_whole_batches(name):
+    """f4 (R#29): BT.709 sources through every kernel class (k_plain, k_copy, k_direct,
+    k_stencil2, mixed Ray trials), whole batches bit-identical to the oracle."""
+    w = configs.get(name)
+    for v in w.spec.views:
+        v.color_matrix = configs.BT709
+    w.spec.batch_size = {"twoview": 4, "ray": 2}.get(name, 4)
+    if name in ("slowfast", "slowfast_hd"):
+        w.spec.batch_size = 2
+    _run(w, 8, epochs=(0,), its=(0,))
+
+
+def test_two_samples_per_video_whole_batches():
+    """Fig. 9's samples_per_video: 2: two clips per video per epoch, whole batches."""
+    w = configs.k400_two_samples()
+    w.spec.batch_size = 4
+    _run(w, 6, epochs=(0, 1))

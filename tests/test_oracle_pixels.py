@@ -222,3 +222,51 @@ def test_normalize_vs_torchvision_and_bf16():
     L = oracle.lib()
     vals = np.array([L.oracle_normalize(i, float(a[0]), float(b[0])) for i in range(256)], np.float32)
     assert np.abs(vals - (np.arange(256) / 255.0 - mean[0]) / std[0]).max() <= 1e-6
+
+
+def _all_triples():
+    Wc, Hc = 4096, 1024
+    idx = np.arange(Wc * Hc, dtype=np.int64).reshape(Hc, Wc)
+    uvpair = idx % 65536
+    block = idx // 65536
+    U = (uvpair // 256).astype(np.uint8)
+    V = (uvpair % 256).astype(np.uint8)
+    Y = np.empty((2 * Hc, 2 * Wc), np.uint8)
+    base = (block * 4).astype(np.uint8)
+    Y[0::2, 0::2] = base
+    Y[0::2, 1::2] = base + 1
+    Y[1::2, 0::2] = base + 2
+    Y[1::2, 1::2] = base + 3
+    uv = np.empty((Hc, 2 * Wc), np.uint8)
+    uv[:, 0::2] = U
+    uv[:, 1::2] = V
+    Uf = np.repeat(np.repeat(U, 2, axis=0), 2, axis=1).astype(np.float64)
+    Vf = np.repeat(np.repeat(V, 2, axis=0), 2, axis=1).astype(np.float64)
+    return Y, uv, Y.astype(np.float64), Uf, Vf
+
+
+def test_bt709_exhaustive_vs_itu_matrix():
+    """f4 (R#29): the BT.709 integer form against the ITU-R BT.709 matrix computed in float64
+    from Kr = 0.2126, Kb = 0.0722 with the limited-range scales 255/219 and 255/224 (the
+    standard's definition, not the oracle's constants): within 1 LSB for every (Y, U, V) with
+    Y >= 16, identical in > 99.8 % of them; below 16 luma clamps like OpenCV's BT.601 form."""
+    Y, uv, Yf, Uf, Vf = _all_triples()
+    ours = oracle.nv12_to_rgb(Y, uv, 1).astype(np.int32)
+    Kr, Kb = 0.2126, 0.0722
+    Kg = 1 - Kr - Kb
+    sy, sc = 255.0 / 219.0, 255.0 / 224.0
+    yl = sy * (np.maximum(Yf, 16) - 16)
+    u, v = Uf - 128, Vf - 128
+    ref = np.stack([yl + 2 * (1 - Kr) * sc * v,
+                    yl - 2 * Kb * (1 - Kb) / Kg * sc * u - 2 * Kr * (1 - Kr) / Kg * sc * v,
+                    yl + 2 * (1 - Kb) * sc * u], axis=-1)
+    ref = np.clip(np.floor(ref + 0.5), 0, 255).astype(np.int32)
+    d = np.abs(ours - ref)
+    assert d.max() <= 1
+    assert (d == 0).mean() > 0.998
+    # BT.709 differs from BT.601 (not a relabelled 601): most saturated colours change
+    assert (ours != oracle.nv12_to_rgb(Y, uv, 0)).any(axis=-1).mean() > 0.5
+    # Y < 16 behaves as Y = 16 (the clamp of the integer form)
+    lo = Y < 16
+    Y16 = np.where(lo, 16, Y).astype(np.uint8)
+    assert np.array_equal(ours[lo], oracle.nv12_to_rgb(Y16, uv, 1).astype(np.int32)[lo])

@@ -94,6 +94,18 @@ def main():
         traffic[cfg] = {"kernel": dom[0], "dram_bytes_per_launch": dom[1][1] / dom[1][2],
                         "ncu_duration_per_launch": dom[1][0] / dom[1][2],
                         "source": f"profiles/{rnd}_ncu_summary.md"}
+        # instruction counts and pipe utilisation of the dominant kernel (the ALU roofline)
+        for d in data:
+            if d[hdr.index("Kernel Name")].split("(")[0] != dom[0]:
+                continue
+            def val(m):
+                return float(d[hdr.index(m)].replace(",", "")) if m in hdr and d[hdr.index(m)] else None
+            traffic[cfg].update({
+                "warp_inst_per_launch": val("smsp__inst_executed.sum"),
+                "alu_pipe_pct": val("sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active"),
+                "fma_pipe_pct": val("sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active"),
+                "issue_active_pct": val("smsp__issue_active.avg.pct_of_peak_sustained_active")})
+            break
         det = os.path.join(OUT, f"{tag}_ncu_details_{cfg}.csv")
         if os.path.exists(det):
             notes = []
