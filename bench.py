@@ -195,7 +195,8 @@ def _oracle_spec(spec):
                              rot_p=v.rot_p, rot_max_deg=v.rot_max_deg, blur_p=v.blur_p, sigma=v.sigma,
                              blur_ksize=v.blur_ksize, blur_truncate=v.blur_truncate, mean=v.mean, std=v.std,
                              out_dtype=v.out_dtype, subsample_of=v.subsample_of,
-                             color_matrix=v.color_matrix) for v in spec.views]
+                             color_matrix=v.color_matrix, jitter_p=v.jitter_p, brightness=v.brightness,
+                             contrast=v.contrast, saturation=v.saturation) for v in spec.views]
     return oracle.make_spec(oracle.SpecDesc(seed=spec.seed, world_size=spec.world_size,
                                             batch_size=spec.batch_size, samples_per_video=spec.samples_per_video,
                                             drop_last=spec.drop_last, shared_window=spec.shared_window, pool_epochs=spec.pool_epochs,
@@ -455,7 +456,8 @@ def run_sand(args):
         "gpu_launches": int(launches),
         "object_cache": (None if not args.object_budget_gb else
                          {k: int(getattr(view.object_stats(), k)) for k in
-                          ("hits", "fills", "misses", "evictions", "objects", "bytes_used", "bytes_budget")}),
+                          ("hits", "fills", "misses", "evictions", "objects", "bytes_used", "bytes_budget",
+                           "decide_ns", "stage_ns", "launch_ns")}),
         "host": host,
         "clocks": clk,
         "reuse": {"fetches": totals[0], "uses": totals[1], "batches": totals[2], "per_rank": per_rank},

@@ -166,6 +166,8 @@ typedef struct {
                                must itself draw from the pool; stride/pool_offset are unused */
   int32_t color_matrix;     /* SAND_BT601 (R#11, OpenCV's integer form) or SAND_BT709 (R#29); every
                                view of a spec uses the same matrix (the decoder's colour space) */
+  double jitter_p;          /* colour jitter gate (R#30): brightness, contrast and saturation */
+  double brightness, contrast, saturation;   /* magnitudes m: factor ~ U[max(0, 1 - m), 1 + m]  */
 } sand_view_desc;
 
 typedef struct {
@@ -248,6 +250,7 @@ int sand_view_set_object_budget(sand_view* v, uint64_t bytes);
 typedef struct {
   uint64_t hits, fills, misses, evictions;   /* eligible items served by each path; objects evicted */
   uint64_t objects, bytes_used, bytes_budget;
+  uint64_t decide_ns, stage_ns, launch_ns;   /* host time in read_batch: decisions, staging, launches */
 } sand_object_stats;
 int sand_view_object_stats(const sand_view* v, sand_object_stats* out);
 
@@ -265,6 +268,8 @@ typedef struct {
   uint32_t flip[SAND_MAX_GROUPS], rot_on[SAND_MAX_GROUPS], blur_on[SAND_MAX_GROUPS],
       blur_r[SAND_MAX_GROUPS];
   double theta[SAND_MAX_GROUPS], sigma[SAND_MAX_GROUPS];
+  uint32_t jitter_on[SAND_MAX_GROUPS], jitter_order[SAND_MAX_GROUPS];   /* R#30: order 0..5 of (B, C, S) */
+  double jitter_f[SAND_MAX_GROUPS][3];                                  /* brightness, contrast, saturation */
 } sand_clip_meta;
 int sand_view_get_meta(sand_view* v, uint64_t epoch, uint32_t rank, uint64_t iteration,
                        sand_clip_meta* out);

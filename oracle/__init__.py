@@ -39,6 +39,8 @@ class View(ctypes.Structure):
         ("blur_ksize", ctypes.c_uint32), ("blur_truncate", ctypes.c_double),
         ("mean", ctypes.c_double * 3), ("std", ctypes.c_double * 3),
         ("out_dtype", ctypes.c_int32), ("subsample_of", ctypes.c_int32), ("color_matrix", ctypes.c_int32),
+        ("jitter_p", ctypes.c_double), ("brightness", ctypes.c_double), ("contrast", ctypes.c_double),
+        ("saturation", ctypes.c_double),
     ]
 
 
@@ -65,6 +67,8 @@ class ClipMeta(ctypes.Structure):
         ("flip", ctypes.c_uint32 * MAX_GROUPS), ("rot_on", ctypes.c_uint32 * MAX_GROUPS),
         ("blur_on", ctypes.c_uint32 * MAX_GROUPS), ("blur_r", ctypes.c_uint32 * MAX_GROUPS),
         ("theta", ctypes.c_double * MAX_GROUPS), ("sigma", ctypes.c_double * MAX_GROUPS),
+        ("jitter_on", ctypes.c_uint32 * MAX_GROUPS), ("jitter_order", ctypes.c_uint32 * MAX_GROUPS),
+        ("jitter_f", (ctypes.c_double * 3) * MAX_GROUPS),
     ]
 
 
@@ -114,6 +118,7 @@ def lib():
             "oracle_shortside_crop": (None, [vp, u32, u32, P(i32), u32, u32, vp]),
             "oracle_flip": (None, [vp, u32, u32, vp]),
             "oracle_rotate": (None, [vp, u32, u32, dbl, vp]),
+            "oracle_color_jitter": (None, [vp, u32, u32, ctypes.POINTER(ctypes.c_double), u32]),
             "oracle_blur_weights": (None, [dbl, u32, P(ctypes.c_float)]),
             "oracle_blur": (None, [vp, u32, u32, dbl, u32, vp]),
             "oracle_norm_coeffs": (None, [P(dbl), P(dbl), P(ctypes.c_float), P(ctypes.c_float)]),
@@ -229,6 +234,15 @@ def rotate(img: np.ndarray, theta_deg: float) -> np.ndarray:
     return out
 
 
+def color_jitter(img: np.ndarray, factors, order: int) -> np.ndarray:
+    """img: HWC uint8; factors (brightness, contrast, saturation); order 0..5 (R#30)."""
+    out = np.ascontiguousarray(img, np.uint8).copy()
+    H, W, _ = out.shape
+    f = (ctypes.c_double * 3)(*factors)
+    lib().oracle_color_jitter(_u8p(out), H, W, f, order)
+    return out
+
+
 def blur_weights(sigma: float, r: int) -> np.ndarray:
     w = (ctypes.c_float * 64)()
     lib().oracle_blur_weights(sigma, r, w)
@@ -294,6 +308,10 @@ class ViewDesc:
     out_dtype: int = BF16
     subsample_of: int = -1
     color_matrix: int = 0
+    jitter_p: float = 0.0
+    brightness: float = 0.0
+    contrast: float = 0.0
+    saturation: float = 0.0
 
 
 @dataclass
@@ -334,6 +352,7 @@ def make_spec(sd: SpecDesc) -> Spec:
         o.out_dtype = v.out_dtype
         o.subsample_of = v.subsample_of
         o.color_matrix = v.color_matrix
+        o.jitter_p, o.brightness, o.contrast, o.saturation = v.jitter_p, v.brightness, v.contrast, v.saturation
     return s
 
 

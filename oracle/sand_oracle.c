@@ -55,6 +55,7 @@ typedef struct {
   int32_t out_dtype;               /* OR_U8 / OR_BF16 / OR_F32 */
   int32_t subsample_of;            /* -1: pool view; k: linspace sub-sample of view k (R#26) */
   int32_t color_matrix;            /* 0: BT.601 (R#11), 1: BT.709 (R#29) */
+  double jitter_p, brightness, contrast, saturation;   /* colour jitter (R#30) */
 } oracle_view;
 
 typedef struct {
@@ -75,6 +76,8 @@ typedef struct {
   int32_t box[OR_MAX_GROUPS][4];   /* RRC: x0,y0,w,h ; SHORTSIDE: x_off,y_off,W',H' */
   uint32_t flip[OR_MAX_GROUPS], rot_on[OR_MAX_GROUPS], blur_on[OR_MAX_GROUPS], blur_r[OR_MAX_GROUPS];
   double theta[OR_MAX_GROUPS], sigma[OR_MAX_GROUPS];
+  uint32_t jitter_on[OR_MAX_GROUPS], jitter_order[OR_MAX_GROUPS];
+  double jitter_f[OR_MAX_GROUPS][3];   /* brightness, contrast, saturation factors */
 } oracle_clip_meta;
 
 /* ------------------------------------------------------------------------- */
@@ -373,6 +376,18 @@ void oracle_spatial(const oracle_spec* spec, uint64_t epoch, uint32_t clip, uint
       double rr = floor(v->blur_truncate * meta->sigma[q] + 0.5);
       meta->blur_r[q] = rr < (double)rmax ? (uint32_t)rr : rmax;
     }
+    /* colour jitter (R#30): gate, factors U[max(0, 1 - m), 1 + m] (torchvision
+       ColorJitter's ranges), then the order of the three ops: one of the 6 permutations of
+       (brightness, contrast, saturation) in lexicographic order */
+    draw(seed, OR_AUG, q, 2, 0, clip, epoch, x);
+    meta->jitter_on[q] = (uint32_t)oracle_bern(x[0], v->jitter_p);
+    double mags[3] = {v->brightness, v->contrast, v->saturation};
+    for (int i = 0; i < 3; ++i) {
+      double lo = mags[i] < 1.0 ? 1.0 - mags[i] : 0.0, hi = 1.0 + mags[i];
+      meta->jitter_f[q][i] = lo + (hi - lo) * oracle_u01(x[1 + i]);
+    }
+    draw(seed, OR_AUG, q, 3, 0, clip, epoch, x);
+    meta->jitter_order[q] = oracle_bounded(x[0], 6);
   }
 }
 
@@ -626,6 +641,52 @@ uint16_t oracle_bf16_rne(float f) {               /* round to nearest even (fini
 }
 
 /* ------------------------------------------------------------------------- */
+/* Colour jitter ("colour jitter"; R#30), on an HWC uint8 image in place, */
+/* after flip and before rotation (op order R#14 + R#30). torchvision's         */
+/* adjust_brightness / adjust_contrast / adjust_saturation on uint8 tensors,     */
+/* written out with every float32 operation rounded on its own:                 */
+/*   brightness f: o = trunc(clamp(x * f, 0, 255))                               */
+/*   gray(r,g,b) = floor((r * 0.2989f + g * 0.587f) + b * 0.114f)                */
+/*   saturation f: o = trunc(clamp(x * f + gray * (float)(1 - f), 0, 255))       */
+/*   contrast f:   m = (float)sum(gray) / (float)(H W) (an exact integer sum),   */
+/*                 o = trunc(clamp(x * f + m * (float)(1 - f), 0, 255))          */
+/* order k = 0..5 is the k-th permutation of (brightness, contrast, saturation)  */
+/* in lexicographic order.                                                       */
+/* ------------------------------------------------------------------------- */
+static float jit_gray(uint8_t r, uint8_t g, uint8_t b) {
+  float t = (float)r * 0.2989f;
+  t = t + (float)g * 0.587f;
+  t = t + (float)b * 0.114f;
+  return floorf(t);
+}
+static uint8_t jit_u8(float v) {
+  if (v < 0.f) v = 0.f;
+  if (v > 255.f) v = 255.f;
+  return (uint8_t)v;            /* truncation toward zero, like torch's float -> uint8 */
+}
+void oracle_color_jitter(uint8_t* img, uint32_t H, uint32_t W, const double f[3], uint32_t order) {
+  static const int perm[6][3] = {{0, 1, 2}, {0, 2, 1}, {1, 0, 2}, {1, 2, 0}, {2, 0, 1}, {2, 1, 0}};
+  size_t n = (size_t)H * W;
+  for (int s = 0; s < 3; ++s) {
+    int op = perm[order % 6][s];
+    float fx = (float)f[op], fa = (float)(1.0 - f[op]);
+    if (op == 0) {
+      for (size_t i = 0; i < 3 * n; ++i) img[i] = jit_u8((float)img[i] * fx);
+    } else if (op == 1) {
+      uint64_t sum = 0;
+      for (size_t i = 0; i < n; ++i) sum += (uint64_t)jit_gray(img[3 * i], img[3 * i + 1], img[3 * i + 2]);
+      float mean = (float)sum / (float)n;
+      for (size_t i = 0; i < 3 * n; ++i) img[i] = jit_u8((float)img[i] * fx + mean * fa);
+    } else {
+      for (size_t i = 0; i < n; ++i) {
+        float gr = jit_gray(img[3 * i], img[3 * i + 1], img[3 * i + 2]);
+        for (int c = 0; c < 3; ++c) img[3 * i + c] = jit_u8((float)img[3 * i + c] * fx + gr * fa);
+      }
+    }
+  }
+}
+
+/* ------------------------------------------------------------------------- */
 /* Render one output frame (view k, time t) of one planned clip:              */
 /* NV12 -> RGB (Q1) -> crop/resize (Q2) -> flip -> rotate (Q3) -> blur (Q4)   */
 /* -> normalise -> out[c][y][x] in the view's dtype (op order R#14).          */
@@ -646,6 +707,7 @@ void oracle_render_frame(const oracle_spec* spec, const oracle_clip_meta* meta, 
   else
     oracle_shortside_crop(rgb, W, H, meta->box[q], Ho, Wo, a);
   if (meta->flip[q]) { oracle_flip(a, Ho, Wo, b); memcpy(a, b, n); }
+  if (meta->jitter_on[q]) oracle_color_jitter(a, Ho, Wo, meta->jitter_f[q], meta->jitter_order[q]);
   if (meta->rot_on[q]) { oracle_rotate(a, Ho, Wo, meta->theta[q], b); memcpy(a, b, n); }
   if (meta->blur_on[q]) { oracle_blur(a, Ho, Wo, meta->sigma[q], meta->blur_r[q], b); memcpy(a, b, n); }
   float ca[3], cb[3];

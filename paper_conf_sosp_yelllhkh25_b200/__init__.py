@@ -63,6 +63,10 @@ def make_spec(spec: Spec, videos) -> tuple[_abi.sand_view_spec, object]:
         o.out_dtype = v.out_dtype
         o.subsample_of = int(getattr(v, "subsample_of", -1))
         o.color_matrix = int(getattr(v, "color_matrix", 0))
+        o.jitter_p = float(getattr(v, "jitter_p", 0.0))
+        o.brightness = float(getattr(v, "brightness", 0.0))
+        o.contrast = float(getattr(v, "contrast", 0.0))
+        o.saturation = float(getattr(v, "saturation", 0.0))
     return s, arr
 
 

@@ -44,6 +44,7 @@ class sand_view_desc(ctypes.Structure):
         ("blur_p", dbl), ("sigma_min", dbl), ("sigma_max", dbl),
         ("blur_ksize", u32), ("blur_truncate", dbl),
         ("mean", dbl * 3), ("std", dbl * 3), ("out_dtype", i32), ("subsample_of", i32), ("color_matrix", i32),
+        ("jitter_p", dbl), ("brightness", dbl), ("contrast", dbl), ("saturation", dbl),
     ]
 
 
@@ -70,6 +71,7 @@ class sand_clip_meta(ctypes.Structure):
         ("box", (i32 * 4) * MAX_GROUPS),
         ("flip", u32 * MAX_GROUPS), ("rot_on", u32 * MAX_GROUPS), ("blur_on", u32 * MAX_GROUPS),
         ("blur_r", u32 * MAX_GROUPS), ("theta", dbl * MAX_GROUPS), ("sigma", dbl * MAX_GROUPS),
+        ("jitter_on", u32 * MAX_GROUPS), ("jitter_order", u32 * MAX_GROUPS), ("jitter_f", (dbl * 3) * MAX_GROUPS),
     ]
 
 
@@ -85,7 +87,8 @@ class sand_view_stats(ctypes.Structure):
 
 class sand_object_stats(ctypes.Structure):
     _fields_ = [("hits", u64), ("fills", u64), ("misses", u64), ("evictions", u64),
-                ("objects", u64), ("bytes_used", u64), ("bytes_budget", u64)]
+                ("objects", u64), ("bytes_used", u64), ("bytes_budget", u64),
+                ("decide_ns", u64), ("stage_ns", u64), ("launch_ns", u64)]
 
 
 P = ctypes.POINTER

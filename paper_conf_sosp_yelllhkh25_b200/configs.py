@@ -40,6 +40,10 @@ class ViewSpec:
     out_dtype: int = BF16
     subsample_of: int = -1        # >= 0: linspace sub-sample of that view's frames (f4, R#26)
     color_matrix: int = BT601     # YUV -> RGB matrix: BT601 (R#11) or BT709 (f4, R#29)
+    jitter_p: float = 0.0         # colour jitter gate (f4, R#30) and torchvision ColorJitter magnitudes
+    brightness: float = 0.0
+    contrast: float = 0.0
+    saturation: float = 0.0
 
 
 @dataclass

@@ -544,6 +544,56 @@ __device__ __forceinline__ void blur_plane(const LaunchParams& p, const GroupPar
   }
 }
 
+// Colour jitter (R#30) on the three Q2 planes in place, after flip, before rotation:
+// the ops of the drawn order one after the other, each a full pass (barrier between), every fp32
+// operation rounded on its own as in the oracle; contrast's mean is an exact integer sum of the
+// floored greys (block reduction) divided once. s_acc: 4 free bytes of shared memory.
+__device__ __forceinline__ float jit_gray(float r, float g, float b) {
+  return floorf(__fadd_rn(__fadd_rn(__fmul_rn(r, 0.2989f), __fmul_rn(g, 0.587f)), __fmul_rn(b, 0.114f)));
+}
+__device__ __forceinline__ uint32_t jit_u8(float v) {   // clamp to [0, 255], truncate (torch float -> uint8)
+  return __float2uint_rz(fminf(fmaxf(v, 0.f), 255.f));
+}
+__device__ void jitter_planes(const GroupParams& g, uint32_t q2, uint32_t plane, int n, uint32_t s_acc, int tid,
+                              int nthr) {
+  const int ord = g.jit_order;             // op of step s at bits 4 s (view.cpp)
+  for (int step = 0; step < 3; ++step) {
+    const int op = (ord >> (4 * step)) & 0xf;
+    const float fx = g.jit_f[op], fa = g.jit_a[op];
+    float mean = 0.f;
+    if (op == 1) {                         // contrast: mean grey of the current image
+      if (tid == 0) sts32(s_acc, 0u);
+      __syncthreads();
+      uint32_t sum = 0;
+      for (int i = tid; i < n; i += nthr)
+        sum += (uint32_t)jit_gray(u8f(ldsu8(q2 + i)), u8f(ldsu8(q2 + plane + i)), u8f(ldsu8(q2 + 2 * plane + i)));
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, o);
+      if ((tid & 31) == 0) asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(s_acc), "r"(sum) : "memory");
+      __syncthreads();
+      mean = __fdiv_rn((float)st::lds32(s_acc), (float)n);
+    }
+    for (int i = tid; i < n; i += nthr) {
+      const float r = u8f(ldsu8(q2 + i)), gg = u8f(ldsu8(q2 + plane + i)), b = u8f(ldsu8(q2 + 2 * plane + i));
+      float o0, o1, o2;
+      if (op == 0) {                       // brightness
+        o0 = __fmul_rn(r, fx);
+        o1 = __fmul_rn(gg, fx);
+        o2 = __fmul_rn(b, fx);
+      } else {                             // contrast (blend with the mean) or saturation (with the grey)
+        const float other = __fmul_rn(op == 1 ? mean : jit_gray(r, gg, b), fa);
+        o0 = __fadd_rn(__fmul_rn(r, fx), other);
+        o1 = __fadd_rn(__fmul_rn(gg, fx), other);
+        o2 = __fadd_rn(__fmul_rn(b, fx), other);
+      }
+      stsu8(q2 + i, jit_u8(o0));
+      stsu8(q2 + plane + i, jit_u8(o1));
+      stsu8(q2 + 2 * plane + i, jit_u8(o2));
+    }
+    __syncthreads();
+  }
+}
+
 }  // namespace sc
 
 template <int DT, bool VEC>
@@ -677,6 +727,9 @@ __global__ void __launch_bounds__(512, 1) k_stencil2(const LaunchParams p, sc::S
     }
   }
   __syncthreads();
+
+  // ------------------------------------------------------------- phase 1b: colour jitter (R#30)
+  if (g.jit_on) jitter_planes(g, q2, (uint32_t)sh.plane, Wo * Ho, ureg, tid, nthr);
 
   // ------------------------------------------------------------- phase 2: per channel
   const int r = g.blur_on ? g.blur_r : 0;

@@ -209,6 +209,8 @@ int launch_stencil(const LaunchParams& ps, const BatchShape& shape, size_t stenc
     return SAND_OK;
   }
   if (stencil_smem > 227 * 1024) return set_error(SAND_EINVAL, "stencil planes exceed shared memory");
+  if (shape.has_jitter)   // the per-channel fallback has no 3-plane stage for the jitter (R#30)
+    return set_error(SAND_EINVAL, "colour jitter needs crops with a source step <= 2 (k_stencil2)");
   k_stencil<<<ps.n_items, 512, stencil_smem, stream>>>(ps);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_error(e, "k_stencil launch");

@@ -21,6 +21,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cstring>
 #include <map>
 #include <unordered_map>
@@ -62,6 +63,10 @@ namespace sand {
 
 namespace {
 size_t a256(size_t x) { return (x + 255) / 256 * 256; }
+uint64_t now_ns() {
+  return static_cast<uint64_t>(
+      std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now().time_since_epoch()).count());
+}
 }  // namespace
 
 void objcache_free(sand_view* v) {
@@ -162,6 +167,7 @@ int objcache_read(sand_view* v, EpochPlan& plan, uint64_t it, const LaunchParams
   auto* c = v->obj;
   if (!c) return SAND_OK;
   *handled = true;
+  const uint64_t t0 = now_ns();
   const sand_view_spec& s = v->info.spec;
   const uint32_t B = s.batch_size;
   const uint32_t kch = std::max<uint32_t>(1, s.pool_epochs);
@@ -291,6 +297,7 @@ int objcache_read(sand_view* v, EpochPlan& plan, uint64_t it, const LaunchParams
   if (!fills.empty()) shape_items(*v, fills, fill_groups, fill_dests, views, vview + 1, &fill_tasks, &fill_shape);
   if (!misses.empty()) shape_items(*v, misses, plan.groups, plan.dests, base.views, s.n_views, &miss_tasks, &miss_shape);
 
+  const uint64_t t1 = now_ns();
   // stage the per-batch arrays (one H2D copy on the caller's stream)
   std::vector<uint8_t> hbuf;
   const size_t o_fg = put(hbuf, fill_groups), o_fi = put(hbuf, fills), o_fd = put(hbuf, fill_dests),
@@ -313,6 +320,7 @@ int objcache_read(sand_view* v, EpochPlan& plan, uint64_t it, const LaunchParams
   if (e == cudaSuccess && !hbuf.empty()) e = cudaMemcpyAsync(st.d, st.h, hbuf.size(), cudaMemcpyHostToDevice, stream);
   if (e != cudaSuccess) return cuda_error(e, "object cache staging copy");
   auto* d = static_cast<uint8_t*>(st.d);
+  const uint64_t t2 = now_ns();
 
   int n = 0, rc = SAND_OK;
   if (!fills.empty()) {                 // resized frames into their slots (a uint8 virtual view)
@@ -351,6 +359,10 @@ int objcache_read(sand_view* v, EpochPlan& plan, uint64_t it, const LaunchParams
   st.used = true;
   c->batch_recorded = true;
   *launched = n;
+  const uint64_t t3 = now_ns();
+  c->stats.decide_ns += t1 - t0;
+  c->stats.stage_ns += t2 - t1;
+  c->stats.launch_ns += t3 - t2;
   return SAND_OK;
 }
 

@@ -35,6 +35,10 @@ struct alignas(16) GroupParams {
   float sc_x, sc_y, rot_c, rot_s;
   int32_t flip, rot_on, blur_on, blur_r;
   float blur_w[24];
+  // colour jitter (R#30): gate, order 0..5, per op (brightness, contrast, saturation) the factor
+  // f as float and (float)(1 - f) (computed in double)
+  int32_t jit_on, jit_order, pad0, pad1;
+  float jit_f[4], jit_a[4];
 };
 
 struct alignas(16) WorkItem {
@@ -100,6 +104,7 @@ struct BatchShape {
   uint32_t task_first, n_tasks;
   int32_t pl_gw, pl_rb;
   int32_t fold;             // every view's normalisation folds the rint bias (ViewConst::fold)
+  int32_t has_jitter;       // a stencil item applies colour jitter (k_stencil2 only, R#30)
 };
 
 // k_plain task granularity (view.cpp builds the tasks, k_plain.cuh consumes them)

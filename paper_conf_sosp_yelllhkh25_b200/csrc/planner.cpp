@@ -40,7 +40,9 @@ static bool same_spatial(const sand_view_desc& a, const sand_view_desc& b) {
          a.ratio_min == b.ratio_min && a.ratio_max == b.ratio_max && a.short_side == b.short_side &&
          a.out_h == b.out_h && a.out_w == b.out_w && a.flip_p == b.flip_p && a.rot_p == b.rot_p &&
          a.rot_max_deg == b.rot_max_deg && a.blur_p == b.blur_p && a.sigma_min == b.sigma_min &&
-         a.sigma_max == b.sigma_max && a.blur_ksize == b.blur_ksize && a.blur_truncate == b.blur_truncate;
+         a.sigma_max == b.sigma_max && a.blur_ksize == b.blur_ksize && a.blur_truncate == b.blur_truncate &&
+         a.jitter_p == b.jitter_p && a.brightness == b.brightness && a.contrast == b.contrast &&
+         a.saturation == b.saturation;
 }
 
 int validate_spec(const sand_view_spec& s, std::string* why) {
@@ -80,6 +82,11 @@ int validate_spec(const sand_view_spec& s, std::string* why) {
          s.views[v.subsample_of].subsample_of >= 0))
       return bad("subsample_of must name another view that draws from the pool");
     if (v.color_matrix != SAND_BT601 && v.color_matrix != SAND_BT709) return bad("unknown color_matrix");
+    if (!(v.jitter_p >= 0.0 && v.jitter_p <= 1.0) || !(v.brightness >= 0.0) || !(v.contrast >= 0.0) ||
+        !(v.saturation >= 0.0))
+      return bad("colour jitter: probability in [0, 1], magnitudes >= 0");
+    if (v.jitter_p > 0.0 && static_cast<uint64_t>(v.out_h) * v.out_w > 65536)
+      return bad("colour-jitter views are limited to out_h*out_w <= 65536");
     if (v.color_matrix != s.views[0].color_matrix) return bad("every view must use the same color_matrix");
   }
   uint32_t g = 0;
@@ -288,6 +295,15 @@ void plan_clip(const SpecInfo& info, uint64_t epoch, uint32_t clip, sand_clip_me
     } else {
       m->blur_r[q] = cap;
     }
+    // colour jitter (R#30): gate and the three factors, then the order of the three ops
+    const auto xj = d.get(Purpose::kAug, q, 2, 0, clip);
+    m->jitter_on[q] = draw_coin(xj[0], v.jitter_p);
+    const double mags[3] = {v.brightness, v.contrast, v.saturation};
+    for (int i = 0; i < 3; ++i) {
+      const double lo = mags[i] < 1.0 ? 1.0 - mags[i] : 0.0, hi = 1.0 + mags[i];
+      m->jitter_f[q][i] = lo + (hi - lo) * draw_unit(xj[1 + i]);
+    }
+    m->jitter_order[q] = draw_below(d.get(Purpose::kAug, q, 3, 0, clip)[0], 6);
   }
 }
 

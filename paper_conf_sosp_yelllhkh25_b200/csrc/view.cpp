@@ -77,6 +77,15 @@ GroupParams group_params(const sand_view_desc& d, const sand_clip_meta& m, uint3
     }
     for (int i = 0; i <= 2 * r; ++i) g.blur_w[i] = static_cast<float>(e[i] / total);
   }
+  g.jit_on = static_cast<int32_t>(m.jitter_on[q]);
+  // order k (the k-th permutation of (brightness 0, contrast 1, saturation 2) in lexicographic
+  // order) as the op of step s at bits 4 s
+  static const int32_t kOrder[6] = {0x210, 0x120, 0x201, 0x021, 0x102, 0x012};
+  g.jit_order = kOrder[m.jitter_order[q] % 6];
+  for (int i = 0; i < 3; ++i) {   // factors and blend weights in double, cast once (R#30)
+    g.jit_f[i] = static_cast<float>(m.jitter_f[q][i]);
+    g.jit_a[i] = static_cast<float>(1.0 - m.jitter_f[q][i]);
+  }
   return g;
 }
 
@@ -198,7 +207,7 @@ void shape_items(const sand_view& v, std::vector<WorkItem>& items, const std::ve
     const GroupParams& g = groups[w.gp];
     const bool mild = g.sc_x <= 2.0f && g.sc_y <= 2.0f;
     const int cols = span16(g);
-    w.flags = (g.rot_on || g.blur_on) ? 1u : (mild ? 0u : 2u);
+    w.flags = (g.rot_on || g.blur_on || g.jit_on) ? 1u : (mild ? 0u : 2u);
     for (uint32_t d = 0; d < w.n_dest; ++d) {
       const ViewConst& vc = views[dests[w.dest_begin + d] >> 24];
       sh.dtype = sh.dtype == -2 ? vc.dtype : (sh.dtype == vc.dtype ? sh.dtype : -1);
@@ -207,6 +216,7 @@ void shape_items(const sand_view& v, std::vector<WorkItem>& items, const std::ve
     }
     if (w.flags & 1u) {
       sh.has_stencil = 1;
+      if (g.jit_on) sh.has_jitter = 1;
       sh.st_max_wo = std::max(sh.st_max_wo, g.out_w);
       sh.st_max_ho = std::max(sh.st_max_ho, g.out_h);
       sh.st_cols_bound = std::max(sh.st_cols_bound, cols);
@@ -335,9 +345,10 @@ std::shared_ptr<EpochPlan> build_plan(const sand_view& v, uint64_t epoch, uint32
         // wide crop overrun the staging kernels' shared memory)
         const int cols = span16(g);
         const bool mild = g.sc_x <= 2.0f && g.sc_y <= 2.0f;
-        gflags[gi] = (g.rot_on || g.blur_on) ? 1u : (mild ? 0u : 2u);
+        gflags[gi] = (g.rot_on || g.blur_on || g.jit_on) ? 1u : (mild ? 0u : 2u);
         if (gflags[gi] & 1u) {
           shape.has_stencil = 1;
+          if (g.jit_on) shape.has_jitter = 1;
           shape.st_max_wo = std::max(shape.st_max_wo, g.out_w);
           shape.st_max_ho = std::max(shape.st_max_ho, g.out_h);
           shape.st_cols_bound = std::max(shape.st_cols_bound, cols);
@@ -742,7 +753,7 @@ extern "C" int sand_view_create(sand_store* s, const sand_view_spec* spec, sand_
     c.T = static_cast<int32_t>(vd.clip_len);
     c.out_h = static_cast<int32_t>(vd.out_h);
     c.out_w = static_cast<int32_t>(vd.out_w);
-    if (vd.rot_p > 0.0 || vd.blur_p > 0.0) {
+    if (vd.rot_p > 0.0 || vd.blur_p > 0.0 || vd.jitter_p > 0.0) {
       stencil = true;
       max_h = std::max(max_h, static_cast<int>(vd.out_h));
       max_w = std::max(max_w, static_cast<int>(vd.out_w));

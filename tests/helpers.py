@@ -23,7 +23,8 @@ def to_oracle(spec) -> oracle.Spec:
                              rot_p=v.rot_p, rot_max_deg=v.rot_max_deg, blur_p=v.blur_p, sigma=v.sigma,
                              blur_ksize=v.blur_ksize, blur_truncate=v.blur_truncate, mean=v.mean, std=v.std,
                              out_dtype=v.out_dtype, subsample_of=v.subsample_of,
-                             color_matrix=v.color_matrix) for v in spec.views]
+                             color_matrix=v.color_matrix, jitter_p=v.jitter_p, brightness=v.brightness,
+                             contrast=v.contrast, saturation=v.saturation) for v in spec.views]
     return oracle.make_spec(oracle.SpecDesc(seed=spec.seed, world_size=spec.world_size,
                                             batch_size=spec.batch_size, samples_per_video=spec.samples_per_video,
                                             drop_last=spec.drop_last, shared_window=spec.shared_window, pool_epochs=spec.pool_epochs,
@@ -44,6 +45,8 @@ def meta_fields(spec, m):
         "flip": [m.flip[q] for q in groups], "rot_on": [m.rot_on[q] for q in groups],
         "blur_on": [m.blur_on[q] for q in groups], "blur_r": [m.blur_r[q] for q in groups],
         "theta": [m.theta[q] for q in groups], "sigma": [m.sigma[q] for q in groups],
+        "jitter_on": [m.jitter_on[q] for q in groups], "jitter_order": [m.jitter_order[q] for q in groups],
+        "jitter_f": [list(m.jitter_f[q]) for q in groups],
     }
 
 

@@ -257,3 +257,20 @@ def test_two_samples_per_video_whole_batches():
     w = configs.k400_two_samples()
     w.spec.batch_size = 4
     _run(w, 6, epochs=(0, 1))
+
+
+@pytest.mark.parametrize("dtype", [configs.BF16, configs.U8, configs.F32])
+def test_color_jitter_whole_batches(dtype):
+    """f4 (R#30): colour jitter (p 0.8; brightness, contrast, saturation 0.4; random order)
+    with and without rotation and blur, through k_stencil2's three-plane stage; whole batches
+    bit-identical to the oracle."""
+    w = configs.twoview()
+    for v in w.spec.views:
+        v.jitter_p, v.brightness, v.contrast, v.saturation = 0.8, 0.4, 0.4, 0.4
+        v.out_dtype = dtype
+    w.spec.batch_size = 4
+    spec, vids = w.spec, videos_of(w, 8)
+    metas = oracle.plan_batch(to_oracle(spec), oracle.make_dataset(vids), 8, 0, 0, 0)
+    combos = {(bool(m.jitter_on[q]), bool(m.rot_on[q]), bool(m.blur_on[q])) for m in metas for q in (0, 1)}
+    assert (True, False, False) in combos or len(combos) > 3
+    _run(w, 8, epochs=(0, 1), its=(0,))

@@ -270,3 +270,40 @@ def test_bt709_exhaustive_vs_itu_matrix():
     lo = Y < 16
     Y16 = np.where(lo, 16, Y).astype(np.uint8)
     assert np.array_equal(ours[lo], oracle.nv12_to_rgb(Y16, uv, 1).astype(np.int32)[lo])
+
+
+def test_color_jitter_vs_torchvision():
+    """f4 (R#30): the oracle's colour jitter against torchvision's adjust_brightness /
+    adjust_contrast / adjust_saturation on uint8 tensors (the ops ColorJitter applies), one op at
+    a time (within 1 LSB, identical for > 99 % of values) and composed in each of the 6 orders
+    (within 1 LSB per stage); factor 1 is the identity."""
+    import torch
+    from torchvision.transforms.v2 import functional as TF
+    rng = np.random.default_rng(11)
+    ops = [TF.adjust_brightness, TF.adjust_contrast, TF.adjust_saturation]
+    perms = [(0, 1, 2), (0, 2, 1), (1, 0, 2), (1, 2, 0), (2, 0, 1), (2, 1, 0)]
+    diffs, composed = [], []
+    for trial in range(24):
+        img = rng.integers(0, 256, size=(40, 56, 3), dtype=np.uint8)
+        if trial % 3 == 0:                               # natural-image-like smooth content
+            img = np.clip(np.cumsum(rng.integers(-3, 4, size=(40, 56, 3)), axis=1) + 128, 0, 255).astype(np.uint8)
+        f = rng.uniform(0.6, 1.4, size=3)
+        order = trial % 6
+        ours = oracle.color_jitter(img, f, order)
+        t = torch.from_numpy(img).permute(2, 0, 1).contiguous()
+        for op in perms[order]:
+            t = ops[op](t, float(f[op]))
+        ref = t.permute(1, 2, 0).numpy()
+        composed.append(np.abs(ours.astype(int) - ref.astype(int)))
+        for op in range(3):                              # each op alone (the others at factor 1)
+            g = np.ones(3)
+            g[op] = f[op]
+            one = oracle.color_jitter(img, g, 0)
+            r1 = ops[op](torch.from_numpy(img).permute(2, 0, 1).contiguous(), float(f[op])).permute(1, 2, 0).numpy()
+            diffs.append(np.abs(one.astype(int) - r1.astype(int)))
+        assert np.array_equal(oracle.color_jitter(img, [1.0, 1.0, 1.0], order), img)
+    d = np.concatenate([x.ravel() for x in diffs])
+    assert d.max() <= 1 and (d == 0).mean() > 0.99
+    # composed: a 1 LSB tie flip in one stage may grow by the next factor (<= 1.4): <= 1 per stage
+    dc = np.concatenate([x.ravel() for x in composed])
+    assert dc.max() <= 3 and (dc == 0).mean() > 0.99

@@ -139,3 +139,16 @@ def test_host_plan_rrc_central_fallback_matches_oracle():
         vids = [(1000 + i, 30, 340, 256) for i in range(4)]
         for got in _plan_equal(spec, vids, (0, 1, 5), range(4)):
             assert list(got.box[0]) == box
+
+
+def test_host_plan_color_jitter_draws_match_oracle():
+    """f4 (R#30): colour-jitter gates, factors and op orders plan bit-exactly like the oracle."""
+    w = configs.twoview()
+    for v in w.spec.views:
+        v.jitter_p, v.brightness, v.contrast, v.saturation = 0.8, 0.4, 0.4, 0.4
+    vids = videos_of(w, 16)
+    got = list(_plan_equal(w.spec, vids, (0, 3), range(16)))
+    on = [m.jitter_on[q] for m in got for q in (0, 1)]
+    assert 0 < sum(on) < len(on)
+    assert all(0.6 <= m.jitter_f[q][i] <= 1.4 for m in got for q in (0, 1) for i in range(3))
+    assert {m.jitter_order[q] for m in got for q in (0, 1)} == set(range(6))
