@@ -108,7 +108,8 @@ static void draw(uint64_t seed, uint32_t purpose, uint32_t group, uint32_t sub, 
                  uint32_t c2, uint64_t epoch, uint32_t out[4]) {
   uint32_t ctr[4] = {c0, (purpose << 24) | ((group & 0xffu) << 16) | (sub & 0xffffu), c2,
                      (uint32_t)epoch};
-  uint32_t key[2] = {(uint32_t)seed, (uint32_t)(seed >> 32)};
+  /* R#1: the epoch's high word is XORed into the key's high word (epochs >= 2^32 stay distinct) */
+  uint32_t key[2] = {(uint32_t)seed, (uint32_t)(seed >> 32) ^ (uint32_t)(epoch >> 32)};
   oracle_philox4x32_10(ctr, key, out);
 }
 

@@ -27,10 +27,13 @@ class Philox4x32 {
 
 enum class Purpose : uint32_t { kPerm = 1, kTemporal = 2, kCrop = 3, kAug = 4, kWindow = 5 };
 
-// The draws of one epoch: counter (index, purpose<<24|group<<16|sub, unit, epoch).
+// The draws of one epoch: counter (index, purpose<<24|group<<16|sub, unit, epoch lo); the epoch's
+// high 32 bits are XORed into the key's high word (R#1), so epochs e and e + 2^32 draw
+// independent streams while every epoch below 2^32 keeps the plain (seed lo, seed hi) key.
 class EpochDraws {
  public:
-  EpochDraws(uint64_t seed, uint64_t epoch) : gen_(seed), epoch_lo_(static_cast<uint32_t>(epoch)) {}
+  EpochDraws(uint64_t seed, uint64_t epoch)
+      : gen_(seed ^ (epoch & 0xffffffff00000000ull)), epoch_lo_(static_cast<uint32_t>(epoch)) {}
   std::array<uint32_t, 4> get(Purpose p, uint32_t group, uint32_t sub, uint32_t index, uint32_t unit) const {
     const uint32_t tag = (static_cast<uint32_t>(p) << 24) | ((group & 0xffu) << 16) | (sub & 0xffffu);
     return gen_({index, tag, unit, epoch_lo_});

@@ -134,3 +134,14 @@ def test_partition_exactly_once_per_epoch(n, world):
     perm = oracle.permutation(n, seed=11, epoch=0)
     allc = np.concatenate([oracle.partition(perm, world, r, False) for r in range(world)])
     assert sorted(allc.tolist()) == list(range(n))
+
+
+def test_permutation_epoch_high_bits_enter_the_key():
+    # R#1: the counter holds the epoch's low word; its high word is XORed into the
+    # key's high word, so epochs e and e + 2^32 are independent streams and the stream of
+    # (seed, e + 2^32) is the one of (seed ^ 2^32, e)
+    a = oracle.permutation(1024, 7, 3)
+    b = oracle.permutation(1024, 7, 3 + 2**32)
+    c = oracle.permutation(1024, 7 ^ (1 << 32), 3)
+    assert (a != b).any()
+    assert (b == c).all()
