@@ -18,7 +18,7 @@ namespace cp {
 // one NV12 pixel (luma Y, chroma terms k) -> three biased floats 2^23 + channel (R#11), the
 // same DPX add-min-relu + IMAD.HI formulation as the other kernels
 __device__ __forceinline__ void px(uint32_t Y, const st::Chroma3& k, uint32_t (&c)[3], const ColorM& m) {
-  const int yy = (int)max(Y, 16u) * m.cy + ((1 << 19) - 16 * m.cy);
+  const int yy = (int)max(Y, 16u) * m.cy + m.yk;
   c[0] = __umulhi((uint32_t)__viaddmin_s32_relu(yy, k.r, 0x0FFFFFFF), 1u << 12) + 0x4B000000u;
   c[1] = __umulhi((uint32_t)__viaddmin_s32_relu(yy, k.g, 0x0FFFFFFF), 1u << 12) + 0x4B000000u;
   c[2] = __umulhi((uint32_t)__viaddmin_s32_relu(yy, k.b, 0x0FFFFFFF), 1u << 12) + 0x4B000000u;

@@ -24,7 +24,7 @@ struct Px3 {
 };
 __device__ __forceinline__ Px3 px3(uint32_t Y, uint32_t uv, const ColorM& m) {
   const st::Chroma3 k = st::chroma_at<0>(uv, m);
-  const int yy = (int)max(Y, 16u) * m.cy + ((1 << 19) - 16 * m.cy);
+  const int yy = (int)max(Y, 16u) * m.cy + m.yk;
   Px3 p;
   p.c[0] = __umulhi((uint32_t)__viaddmin_s32_relu(yy, k.r, 0x0FFFFFFF), 1u << 12) + 0x4B000000u;
   p.c[1] = __umulhi((uint32_t)__viaddmin_s32_relu(yy, k.g, 0x0FFFFFFF), 1u << 12) + 0x4B000000u;

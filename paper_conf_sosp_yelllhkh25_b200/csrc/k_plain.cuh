@@ -29,7 +29,13 @@
 namespace sand {
 namespace pl {
 
-constexpr int kCR = 8;                // source rows per chunk (even)
+#ifndef SAND_PL_CR
+#define SAND_PL_CR 8
+#endif
+#ifndef SAND_PL_MINB
+#define SAND_PL_MINB 2
+#endif
+constexpr int kCR = SAND_PL_CR;       // source rows per chunk (even)
 constexpr int kRawRows = kCR + kCR / 2 + 1;   // staging rows per chunk: Y rows + their UV rows
 
 struct Shape {        // host-chosen launch shape of one batch's plain items
@@ -59,7 +65,7 @@ __device__ __forceinline__ int small_div(int r, float inv_n) { return (int)(((fl
 template <int NP>
 struct PlainBounds {
   static constexpr int kThreads = NP == 1 ? 448 : 224;
-  static constexpr int kMinBlocks = 2;
+  static constexpr int kMinBlocks = SAND_PL_MINB;
 };
 
 template <int DT, int ND, int NP, bool FOLD>
@@ -215,6 +221,32 @@ __global__ void __launch_bounds__(PlainBounds<NP>::kThreads, PlainBounds<NP>::kM
     const uint32_t slot0 = (uint32_t)(ybase + j * kCR);            // absolute row of slot 0
     const uint8_t* rawb0 = smem_raw + (s_fr - s_base) + raw_off + (uint32_t)(j & 1) * rawb;
     uint8_t* convb0 = smem_raw + (s_fr - s_base);
+#if SAND_PL_FLAT
+    // units = (frame, UV row, 4-pixel group), flattened over the CTA (balanced)
+    const int upf = nuv * q4;
+    const float inv_upf = 1.0f / (float)upf, inv_q4 = 1.0f / (float)q4;
+    for (int i = tid; i < nfr * upf; i += nthr) {
+      const int fr = pl::small_div(i, inv_upf), rem = i - fr * upf;
+      const int u = pl::small_div(rem, inv_q4), q = rem - u * q4;
+      const uint8_t* raw = rawb0 + (uint32_t)fr * fbytes + 4u * q;
+      uint8_t* conv = convb0 + (uint32_t)fr * fbytes + 16u * q;
+      const int yt = 2 * (u0 + u);
+      const uint32_t uv = *reinterpret_cast<const uint32_t*>(raw + (uint32_t)(ny + u) * rawpitch);
+      const st::Chroma3 c0 = st::chroma_at<0>(uv, cm), c1 = st::chroma_at<16>(uv, cm);
+      uint8_t* out = conv + ((uint32_t)yt - slot0) * rowbytes;
+      if (yt >= ya) {
+        const uint32_t yw = *reinterpret_cast<const uint32_t*>(raw + (uint32_t)(yt - ya) * rawpitch);
+        *reinterpret_cast<uint4*>(out) = make_uint4(st::rgbx_dpx(st::byte_of<0>(yw), c0, cm), st::rgbx_dpx(st::byte_of<1>(yw), c0, cm),
+                                                    st::rgbx_dpx(st::byte_of<2>(yw), c1, cm), st::rgbx_dpx(st::byte_of<3>(yw), c1, cm));
+      }
+      if (yt + 1 <= yb) {
+        const uint32_t yw = *reinterpret_cast<const uint32_t*>(raw + (uint32_t)(yt + 1 - ya) * rawpitch);
+        *reinterpret_cast<uint4*>(out + rowbytes) =
+            make_uint4(st::rgbx_dpx(st::byte_of<0>(yw), c0, cm), st::rgbx_dpx(st::byte_of<1>(yw), c0, cm),
+                       st::rgbx_dpx(st::byte_of<2>(yw), c1, cm), st::rgbx_dpx(st::byte_of<3>(yw), c1, cm));
+      }
+    }
+#else
     for (int sl = tid; sl < n_slots; sl += nthr) {
       const int fr = sl / q4, q = sl - fr * q4;
       const uint8_t* raw = rawb0 + (uint32_t)fr * fbytes + 4u * q;
@@ -237,6 +269,7 @@ __global__ void __launch_bounds__(PlainBounds<NP>::kThreads, PlainBounds<NP>::kM
         }
       }
     }
+#endif
   };
   // walk of chunk j: source row y's lerps go to X when (y - y_first) is even, else to Y; the
   // output rows whose top tap is y - 1 are emitted as soon as y's lerps exist

@@ -80,6 +80,17 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
       "r"(parity)
       : "memory");
 }
+// the same wait with a suspend-time hint: a warp whose data has not landed sleeps in the
+// barrier instead of re-issuing try_wait (no issue slots taken from the SM's other warps)
+__device__ __forceinline__ void mbar_wait_sleep(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n"
+      "SAND_WAITS_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n"
+      " @!p bra SAND_WAITS_%=;\n}\n" ::"r"(bar),
+      "r"(parity), "r"(1000000u)
+      : "memory");
+}
 __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
                "l"(src), "r"(bytes), "r"(bar)
@@ -130,7 +141,7 @@ __device__ __forceinline__ Chroma3 chroma_at(uint32_t uv, const ColorM& m) {
 // byte 2 is the channel; PRMT gathers the three bytes and the exponent byte 0x4B tops the word
 // (see rs::biased).
 __device__ __forceinline__ uint32_t rgbx_dpx(uint32_t Y, const Chroma3& c, const ColorM& m) {
-  const int yy = (int)max(Y, 16u) * m.cy + ((1 << 19) - 16 * m.cy);
+  const int yy = (int)max(Y, 16u) * m.cy + m.yk;
   // x >> 4 of the clamped sums as IMAD.HI (FMA pipe) to relieve the ALU pipe
   const uint32_t mr = __umulhi((uint32_t)__viaddmin_s32_relu(yy, c.r, 0x0FFFFFFF), 1u << 28);
   const uint32_t mg = __umulhi((uint32_t)__viaddmin_s32_relu(yy, c.g, 0x0FFFFFFF), 1u << 28);

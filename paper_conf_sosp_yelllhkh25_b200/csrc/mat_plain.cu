@@ -1,6 +1,7 @@
 // mat_plain.cu — launcher of the multi-frame plain kernel (k_plain.cuh).
 #include "kernels_common.cuh"
 #include "k_plain.cuh"
+#include "k_plainw.cuh"
 
 namespace sand {
 
@@ -8,11 +9,80 @@ namespace sand {
 #define SAND_PLAIN_NP 2       // column pairs per thread (k_plain.cuh)
 #endif
 constexpr int kNP = SAND_PLAIN_NP;
+#ifndef SAND_PLAINW
+#define SAND_PLAINW 1         // warp-granular k_plainw for widths <= 256 (k_plain otherwise)
+#endif
 
 int plain_cols_per_thread() { return 2 * kNP; }
-int plain_max_threads() { return PlainBounds<kNP>::kThreads; }
+#ifndef SAND_PW_FPC_THREADS
+#define SAND_PW_FPC_THREADS 112   // k_plainw: two frames (four warps) per task at 224 columns
+#endif
+int plain_max_threads() { return SAND_PLAINW ? SAND_PW_FPC_THREADS : PlainBounds<kNP>::kThreads; }
+
+
+#define SAND_PLAINW_KERNELS(X, NPJ)                                                                   \
+  X(SAND_U8, 1, NPJ, false) X(SAND_U8, 2, NPJ, false) X(SAND_BF16, 1, NPJ, false) X(SAND_BF16, 2, NPJ, false) \
+  X(SAND_F32, 1, NPJ, false) X(SAND_F32, 2, NPJ, false) X(SAND_BF16, 1, NPJ, true) X(SAND_BF16, 2, NPJ, true) \
+  X(SAND_F32, 1, NPJ, true) X(SAND_F32, 2, NPJ, true)
+
+static int configure_plainw() {
+#define SAND_PW_ALLOW(DT, ND, NPJ, FOLD)                                                   \
+  if (cudaError_t e = allow_smem(k_plainw<DT, ND, NPJ, FOLD>); e != cudaSuccess) \
+    return cuda_error(e, "cudaFuncSetAttribute(k_plainw)");
+  SAND_PLAINW_KERNELS(SAND_PW_ALLOW, 1)
+  SAND_PLAINW_KERNELS(SAND_PW_ALLOW, 2)
+#undef SAND_PW_ALLOW
+  return SAND_OK;
+}
+
+// k_plainw: one warp per frame of a task (k_plainw.cuh); *launched = false when the batch does
+// not fit it (mixed dtypes, widths not a multiple of 4 or > 256, spans beyond kGWMax)
+static int launch_plainw(const LaunchParams& p, const BatchShape& sh, int fpc, cudaStream_t stream, bool* launched) {
+  *launched = false;
+  if (!SAND_PLAINW || sh.n_tasks == 0 || sh.dtype < 0 || !sh.wo_mod4 || sh.max_wo > 256 || sh.pl_gw > pw::kGWMax ||
+      sh.pl_rb > 32 || fpc < 1 || fpc > pw::kMaxFrames)
+    return SAND_OK;
+  pw::Shape s;
+  s.fpc = fpc;
+  s.gw = sh.pl_gw;
+  const size_t smem = pw::smem_bytes(s);
+  if (smem > 200 * 1024) return SAND_OK;
+  const uint2* tasks = p.tasks + sh.task_first;
+  const bool nd1 = sh.max_dests <= 1, fold = sh.fold != 0 && sh.dtype != SAND_U8;
+  const bool narrow = sh.max_wo <= 128;
+  const unsigned threads = 64u * (unsigned)fpc;
+#define SAND_PW_GO(NPJ)                                                                                     \
+  do {                                                                                                       \
+    switch (sh.dtype) {                                                                                      \
+      case SAND_U8:                                                                                          \
+        if (nd1) k_plainw<SAND_U8, 1, NPJ, false><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);       \
+        else k_plainw<SAND_U8, 2, NPJ, false><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);           \
+        break;                                                                                               \
+      case SAND_BF16:                                                                                        \
+        if (fold && nd1) k_plainw<SAND_BF16, 1, NPJ, true><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);  \
+        else if (fold) k_plainw<SAND_BF16, 2, NPJ, true><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);    \
+        else if (nd1) k_plainw<SAND_BF16, 1, NPJ, false><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);    \
+        else k_plainw<SAND_BF16, 2, NPJ, false><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);             \
+        break;                                                                                               \
+      default:                                                                                               \
+        if (fold && nd1) k_plainw<SAND_F32, 1, NPJ, true><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);   \
+        else if (fold) k_plainw<SAND_F32, 2, NPJ, true><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);     \
+        else if (nd1) k_plainw<SAND_F32, 1, NPJ, false><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);     \
+        else k_plainw<SAND_F32, 2, NPJ, false><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);              \
+        break;                                                                                               \
+    }                                                                                                        \
+  } while (0)
+  if (narrow) SAND_PW_GO(1);
+  else SAND_PW_GO(2);
+#undef SAND_PW_GO
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_error(e, "k_plainw launch");
+  *launched = true;
+  return SAND_OK;
+}
 
 int configure_plain() {
+  if (int rc = configure_plainw(); rc != SAND_OK) return rc;
   for (cudaError_t e : {allow_smem(k_plain<SAND_U8, 1, kNP, false>), allow_smem(k_plain<SAND_BF16, 1, kNP, false>),
                         allow_smem(k_plain<SAND_F32, 1, kNP, false>), allow_smem(k_plain<SAND_U8, 2, kNP, false>),
                         allow_smem(k_plain<SAND_BF16, 2, kNP, false>), allow_smem(k_plain<SAND_F32, 2, kNP, false>),
@@ -24,6 +94,7 @@ int configure_plain() {
 
 int launch_plain(const LaunchParams& p, const BatchShape& sh, int fpc, int nq, cudaStream_t stream, bool* launched) {
   *launched = false;
+  if (int rc = launch_plainw(p, sh, fpc, stream, launched); rc != SAND_OK || *launched) return rc;
   if (sh.n_tasks == 0 || sh.dtype < 0 || (kNP == 2 ? !sh.wo_mod4 : !sh.even_wo)) return SAND_OK;
   pl::Shape s;
   s.fpc = fpc;
