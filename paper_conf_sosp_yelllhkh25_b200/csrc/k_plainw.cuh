@@ -2,8 +2,8 @@
 // Kinetics RRC, two-view plain groups, short-side crops with real scaling; SURVEY §8(a) a4-a7,
 // a10, a11).
 //
-// A task is (up to kMaxFrames frames of ONE (clip slot, group), band of <= 32 output rows), as
-// for k_plain. Each frame of the task is served by a FRAME GROUP of two warps that synchronise
+// A task is (up to 8 frames of ONE (clip slot, group), band of <= 32 output rows), as for k_plain;
+// a CTA serves kFrames of its frames. Each frame is served by a FRAME GROUP of two warps that synchronise
 // only with each other (named barrier 1 + frame, 64 threads), never with the rest of the CTA:
 //   * the group stages its frame's source rows in QUADS (four Y rows from an even row and their
 //     two UV rows), one TMA bulk copy (`cp.async.bulk`) per row into a ring of kStages quads,
@@ -24,7 +24,7 @@
 #pragma once
 
 #ifndef SAND_PW_MINB
-#define SAND_PW_MINB 2
+#define SAND_PW_MINB 5
 #endif
 
 namespace sand {
@@ -34,14 +34,17 @@ namespace pw {
 #define SAND_PW_STAGES 3
 #endif
 constexpr int kStages = SAND_PW_STAGES;   // NV12 row quads in flight per frame
-constexpr int kGWMax = 512;               // widest staged span (pixels); wider batches take k_plain
+#ifndef SAND_PW_GWMAX
+#define SAND_PW_GWMAX 384
+#endif
+constexpr int kGWMax = SAND_PW_GWMAX;     // widest staged span (pixels); wider batches take k_plain
 constexpr int kRow = 4 * kGWMax;          // byte stride of the converted RGBx rows
-constexpr int kMaxFrames = 4;             // frames per CTA (two warps each)
+constexpr int kFrames = 2;                // frames per CTA (two warps each: 128 threads)
 constexpr uint32_t kTabBytes = 272;       // output-row table: 33 (y0, lambda) entries, sentinel last
 constexpr uint32_t kBarBytes = (8u * kStages + 15u) & ~15u;   // the stages' mbarriers
 
 struct Shape {
-  int fpc;   // frames per CTA (2 fpc warps)
+  int nsub;  // CTAs per task: CTA s of a task serves its frames [kFrames s, kFrames (s + 1))
   int gw;    // staged row capacity in pixels (multiple of 16, >= every item's span, <= kGWMax)
 };
 
@@ -51,31 +54,29 @@ __host__ __device__ inline uint32_t stage_bytes(int gw) { return 6u * (uint32_t)
 __host__ __device__ inline uint32_t frame_bytes(int gw) {
   return 8u * kRow + kStages * stage_bytes(gw) + kBarBytes + kTabBytes;   // a multiple of 16
 }
-__host__ __device__ inline size_t smem_bytes(const Shape& s) { return (size_t)s.fpc * frame_bytes(s.gw); }
+__host__ __device__ inline size_t smem_bytes(const Shape& s) { return (size_t)kFrames * frame_bytes(s.gw); }
 
 // named barrier 1 + f of frame group f (immediate ids: a register id would reserve all 16)
 __device__ __forceinline__ void group_sync(int f) {
-  switch (f) {
-    case 0: asm volatile("bar.sync 1, 64;" ::: "memory"); break;
-    case 1: asm volatile("bar.sync 2, 64;" ::: "memory"); break;
-    case 2: asm volatile("bar.sync 3, 64;" ::: "memory"); break;
-    default: asm volatile("bar.sync 4, 64;" ::: "memory"); break;
-  }
+  if (f == 0) asm volatile("bar.sync 1, 64;" ::: "memory");
+  else asm volatile("bar.sync 2, 64;" ::: "memory");
 }
 
 }  // namespace pw
 
 template <int DT, int ND, int NPJ, bool FOLD>
-__global__ void __launch_bounds__(256, SAND_PW_MINB) k_plainw(const LaunchParams p, const uint2* __restrict__ tasks,
+__global__ void __launch_bounds__(128, SAND_PW_MINB) k_plainw(const LaunchParams p, const uint2* __restrict__ tasks,
                                                                pw::Shape sh) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   using namespace rs;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int fr = warp >> 1, half = warp & 1, gt = threadIdx.x & 63;   // frame, half, thread in group
-  const uint2 tk = tasks[blockIdx.x];
+  const int task = (int)blockIdx.x / sh.nsub, sub = (int)blockIdx.x - task * sh.nsub;
+  const uint2 tk = tasks[task];
   const int nfr = (int)(tk.y & 0xffu), nr = (int)((tk.y >> 8) & 0xfffu), Y0 = (int)(tk.y >> 20);
-  if (fr >= nfr) return;                                           // only group barriers follow
-  const WorkItem w = p.items[tk.x + fr];
+  const int fi = pw::kFrames * sub + fr;                           // frame of the task
+  if (fi >= nfr) return;                                           // only group barriers follow
+  const WorkItem w = p.items[tk.x + fi];
   const GroupParams& g = p.groups[w.gp];
   const int Wo = g.out_w;
   const float sc_x = g.sc_x, sc_y = g.sc_y;
@@ -152,8 +153,9 @@ __global__ void __launch_bounds__(256, SAND_PW_MINB) k_plainw(const LaunchParams
     for (int k = 0; k < min(nquads, pw::kStages); ++k) stage(k);
   }
 
-  // column taps of the lane's pairs: shared addresses of tap i0 in RGBx row 0 of buffer 0 (tap
-  // i1 is the next word; at the right clamp i1 == i0 lambda is 0 instead, fmaf(0, d, p0) == p0)
+  // column taps of the lane's pairs: shared addresses of tap i0 in RGBx row 0 of the current
+  // quad's buffer (rebased per quad; tap i1 is the next word; at the right clamp i1 == i0 lambda
+  // is 0 instead, fmaf(0, d, p0) == p0)
   uint32_t ca[NPJ], cb[NPJ];
   uint64_t lx[NPJ];
 #pragma unroll
@@ -174,7 +176,7 @@ __global__ void __launch_bounds__(256, SAND_PW_MINB) k_plainw(const LaunchParams
   bool act[NPJ];
 #pragma unroll
   for (int j = 0; j < NPJ; ++j) act[j] = 2 * lane + 64 * j < Wh;
-  const int nd = (int)w.n_dest;
+  const int nd = (int)w.n_dest;                                   // <= ND (host-checked)
   const uint32_t* dests = p.dests + w.dest_begin;
   // destinations kept in registers: one row pointer per channel plane, advanced per row
   struct DestC {
@@ -212,7 +214,7 @@ __global__ void __launch_bounds__(256, SAND_PW_MINB) k_plainw(const LaunchParams
   };
 
   // one output row from the lerps of its top (T) and bottom (B) source rows
-  auto emit = [&](const Row3 (&T)[NPJ], const Row3 (&B)[NPJ], float l, int oy) {
+  auto emit = [&](const Row3 (&T)[NPJ], const Row3 (&B)[NPJ], float l) {
     const uint64_t ly = f2::splat(l);
     // channel c of pair j: quantised pair (2^23 or 1.5 * 2^23 + rint(v)), stored to plane o
     auto put = [&](uint8_t* o, float a_c, float b_c, int j, uint64_t q) {
@@ -230,32 +232,22 @@ __global__ void __launch_bounds__(256, SAND_PW_MINB) k_plainw(const LaunchParams
         }
       }
     };
-    uint64_t q[NPJ][3];
 #pragma unroll
     for (int j = 0; j < NPJ; ++j)
 #pragma unroll
       for (int c = 0; c < 3; ++c) {
         const uint64_t dv = f2::fma(T[j].h[c], f2::splat(-1.f), B[j].h[c]);   // h1 - h0
         const uint64_t v = f2::fma(ly, dv, T[j].h[c]);                        // fmaf(ly, h1 - h0, h0)
-        q[j][c] = FOLD ? f2::add(v, f2::splat(kBias))                          // 2^23 + rint(v)
-                       : rint_biased(v);                                       // 1.5 * 2^23 + rint(v)
+        const uint64_t q = FOLD ? f2::add(v, f2::splat(kBias))                 // 2^23 + rint(v)
+                                : rint_biased(v);                              // 1.5 * 2^23 + rint(v)
 #pragma unroll
         for (int d = 0; d < ND; ++d)
-          if (d == 0 || d < nd) put(dl[d].o[c], dl[d].a[c], dl[d].b[c], j, q[j][c]);
+          if (d == 0 || d < nd) put(dl[d].o[c], dl[d].a[c], dl[d].b[c], j, q);
       }
 #pragma unroll
     for (int d = 0; d < ND; ++d)
 #pragma unroll
       for (int c = 0; c < 3; ++c) dl[d].o[c] += dl[d].rstride;
-    if (nd > ND) {                                  // rare: more destinations than registers
-      for (int d = ND; d < nd; ++d) {
-        const Dest e = make_dest(p, dests[d], oy, c0 + 2 * lane, FOLD);
-#pragma unroll
-        for (int j = 0; j < NPJ; ++j)
-#pragma unroll
-          for (int c = 0; c < 3; ++c) put(e.row + (size_t)c * e.cstride, e.a[c], e.b[c], j, q[j][c]);
-      }
-    }
   };
 
   pw::group_sync(fr);                           // row table, mbarrier init visible
@@ -265,7 +257,7 @@ __global__ void __launch_bounds__(256, SAND_PW_MINB) k_plainw(const LaunchParams
   // every output row whose y0 is `y`, from the lerps of rows y (T) and y + 1 (B)
   auto emit_rows = [&](const Row3 (&T)[NPJ], const Row3 (&B)[NPJ], int y) {
     while ((int)cy0 == y) {
-      emit(T, B, __uint_as_float(cl), Y0 + r);
+      emit(T, B, __uint_as_float(cl));
       ++r;
       asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(cy0), "=r"(cl) : "r"(s_tab + 8u * r));
     }
@@ -279,7 +271,8 @@ __global__ void __launch_bounds__(256, SAND_PW_MINB) k_plainw(const LaunchParams
     st::mbar_wait_sleep(s_bar + 8u * (uint32_t)(k % pw::kStages), (uint32_t)(k / pw::kStages) & 1u);
     // conversion: units (UV row u, 4-pixel group q) over the group's 64 lanes; a unit converts
     // the two Y rows sharing UV row u (rows outside the band hold stale bytes: converted, unread)
-    for (int i = gt; i < 2 * q4; i += 64) {
+    const int units = yq + 2 <= y_last ? 2 * q4 : q4;  // UV row 1 of the last quad may be unused
+    for (int i = gt; i < units; i += 64) {
       const int u = i >= q4 ? 1 : 0, q = i - u * q4;
       const uint32_t uv = st::lds32(stg + (uint32_t)(4 + u) * gw + 4u * q);
       const st::Chroma3 k0 = st::chroma_at<0>(uv, cm), k1 = st::chroma_at<16>(uv, cm);
@@ -298,22 +291,27 @@ __global__ void __launch_bounds__(256, SAND_PW_MINB) k_plainw(const LaunchParams
       if (lane < 6) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       stage(k + pw::kStages);
     }
-    const uint32_t rb = buf - s_rgb;                // buffer offset of the tap addresses
     if (yq >= y_first) {
-      hrows(X, rb);
+      hrows(X, 0u);
       emit_rows(Yr, X, yq - 1);
     }
     if (yq + 1 <= y_last) {
-      hrows(Yr, rb + (uint32_t)pw::kRow);
+      hrows(Yr, (uint32_t)pw::kRow);
       emit_rows(X, Yr, yq);
     }
     if (yq + 2 <= y_last) {
-      hrows(X, rb + 2u * pw::kRow);
+      hrows(X, 2u * pw::kRow);
       emit_rows(Yr, X, yq + 1);
     }
     if (yq + 3 <= y_last) {
-      hrows(Yr, rb + 3u * pw::kRow);
+      hrows(Yr, 3u * pw::kRow);
       emit_rows(X, Yr, yq + 2);
+    }
+    const uint32_t flipb = (k & 1) ? 0u - 4u * pw::kRow : 4u * pw::kRow;   // next quad's buffer
+#pragma unroll
+    for (int j = 0; j < NPJ; ++j) {
+      ca[j] += flipb;
+      cb[j] += flipb;
     }
   }
   // rows at the bottom clamp (y0 == y1 == y_last, lambda 0): emitted from H(y_last) twice

@@ -36,39 +36,41 @@ static int configure_plainw() {
 }
 
 // k_plainw: one warp per frame of a task (k_plainw.cuh); *launched = false when the batch does
-// not fit it (mixed dtypes, widths not a multiple of 4 or > 256, spans beyond kGWMax)
+// not fit it (mixed dtypes, widths not a multiple of 4 or > 256, spans beyond kGWMax, items with
+// more than two destinations)
 static int launch_plainw(const LaunchParams& p, const BatchShape& sh, int fpc, cudaStream_t stream, bool* launched) {
   *launched = false;
   if (!SAND_PLAINW || sh.n_tasks == 0 || sh.dtype < 0 || !sh.wo_mod4 || sh.max_wo > 256 || sh.pl_gw > pw::kGWMax ||
-      sh.pl_rb > 32 || fpc < 1 || fpc > pw::kMaxFrames)
+      sh.pl_rb > 32 || fpc < 1 || sh.max_dests > 2)
     return SAND_OK;
   pw::Shape s;
-  s.fpc = fpc;
+  s.nsub = (fpc + pw::kFrames - 1) / pw::kFrames;
   s.gw = sh.pl_gw;
   const size_t smem = pw::smem_bytes(s);
   if (smem > 200 * 1024) return SAND_OK;
   const uint2* tasks = p.tasks + sh.task_first;
   const bool nd1 = sh.max_dests <= 1, fold = sh.fold != 0 && sh.dtype != SAND_U8;
   const bool narrow = sh.max_wo <= 128;
-  const unsigned threads = 64u * (unsigned)fpc;
+  const unsigned threads = 64u * pw::kFrames;
+  const unsigned grid = sh.n_tasks * (unsigned)s.nsub;
 #define SAND_PW_GO(NPJ)                                                                                     \
   do {                                                                                                       \
     switch (sh.dtype) {                                                                                      \
       case SAND_U8:                                                                                          \
-        if (nd1) k_plainw<SAND_U8, 1, NPJ, false><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);       \
-        else k_plainw<SAND_U8, 2, NPJ, false><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);           \
+        if (nd1) k_plainw<SAND_U8, 1, NPJ, false><<<grid, threads, smem, stream>>>(p, tasks, s);       \
+        else k_plainw<SAND_U8, 2, NPJ, false><<<grid, threads, smem, stream>>>(p, tasks, s);           \
         break;                                                                                               \
       case SAND_BF16:                                                                                        \
-        if (fold && nd1) k_plainw<SAND_BF16, 1, NPJ, true><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);  \
-        else if (fold) k_plainw<SAND_BF16, 2, NPJ, true><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);    \
-        else if (nd1) k_plainw<SAND_BF16, 1, NPJ, false><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);    \
-        else k_plainw<SAND_BF16, 2, NPJ, false><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);             \
+        if (fold && nd1) k_plainw<SAND_BF16, 1, NPJ, true><<<grid, threads, smem, stream>>>(p, tasks, s);  \
+        else if (fold) k_plainw<SAND_BF16, 2, NPJ, true><<<grid, threads, smem, stream>>>(p, tasks, s);    \
+        else if (nd1) k_plainw<SAND_BF16, 1, NPJ, false><<<grid, threads, smem, stream>>>(p, tasks, s);    \
+        else k_plainw<SAND_BF16, 2, NPJ, false><<<grid, threads, smem, stream>>>(p, tasks, s);             \
         break;                                                                                               \
       default:                                                                                               \
-        if (fold && nd1) k_plainw<SAND_F32, 1, NPJ, true><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);   \
-        else if (fold) k_plainw<SAND_F32, 2, NPJ, true><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);     \
-        else if (nd1) k_plainw<SAND_F32, 1, NPJ, false><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);     \
-        else k_plainw<SAND_F32, 2, NPJ, false><<<sh.n_tasks, threads, smem, stream>>>(p, tasks, s);              \
+        if (fold && nd1) k_plainw<SAND_F32, 1, NPJ, true><<<grid, threads, smem, stream>>>(p, tasks, s);   \
+        else if (fold) k_plainw<SAND_F32, 2, NPJ, true><<<grid, threads, smem, stream>>>(p, tasks, s);     \
+        else if (nd1) k_plainw<SAND_F32, 1, NPJ, false><<<grid, threads, smem, stream>>>(p, tasks, s);     \
+        else k_plainw<SAND_F32, 2, NPJ, false><<<grid, threads, smem, stream>>>(p, tasks, s);              \
         break;                                                                                               \
     }                                                                                                        \
   } while (0)
