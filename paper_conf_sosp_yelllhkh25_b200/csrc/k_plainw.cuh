@@ -173,9 +173,10 @@ __global__ void __launch_bounds__(128, SAND_PW_MINB) k_plainw(const LaunchParams
     cb[j] = s_rgb + 4u * (uint32_t)(b0 - x16);
     lx[j] = f2::pack(__float_as_uint(la), __float_as_uint(lb));
   }
+  // pair j of the lane is a real column pair (NPJ = 2 is used for Wh > 64: pair 0 always is)
   bool act[NPJ];
 #pragma unroll
-  for (int j = 0; j < NPJ; ++j) act[j] = 2 * lane + 64 * j < Wh;
+  for (int j = 0; j < NPJ; ++j) act[j] = (NPJ == 2 && j == 0) || 2 * lane + 64 * j < Wh;
   const int nd = (int)w.n_dest;                                   // <= ND (host-checked)
   const uint32_t* dests = p.dests + w.dest_begin;
   // destinations kept in registers: one row pointer per channel plane, advanced per row
@@ -287,7 +288,7 @@ __global__ void __launch_bounds__(128, SAND_PW_MINB) k_plainw(const LaunchParams
     // one group barrier per quad: quad k converted (buffer k & 1), its stage drained, and the
     // walk of quad k - 1 (buffer (k + 1) & 1, rewritten by quad k + 1) finished in both warps
     pw::group_sync(fr);
-    if (half == 0 && k + pw::kStages < nquads) {
+    if (half == (k & 1) && k + pw::kStages < nquads) {   // the two warps take turns
       if (lane < 6) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       stage(k + pw::kStages);
     }
