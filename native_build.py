@@ -89,9 +89,13 @@ def build_product(force=False, variant=None, defines=()):
         os.makedirs(bdir, exist_ok=True)
         objs = []
         inc = ["-I", os.path.join(ROOT, "include"), "-I", CSRC]
-        for s in PRODUCT_CPP:
-            objs.append(os.path.join(PKG, "build", s + ".o"))
         jobs = []
+        for s in PRODUCT_CPP:   # host units too: the defines may change shared headers
+            obj = os.path.join(bdir, s + ".o")
+            objs.append(obj)
+            jobs.append(["g++", "-O2", "-std=c++17", "-fPIC", "-ffp-contract=off", "-fno-fast-math", "-Wall",
+                         "-I", os.path.join(CUDA_HOME, "include"), *["-D" + d for d in defines], *inc, "-c",
+                         os.path.join(CSRC, s), "-o", obj])
         for s in PRODUCT_CU:
             obj = os.path.join(bdir, s + ".o")
             objs.append(obj)

@@ -2,7 +2,7 @@
 // Kinetics RRC, two-view plain groups, short-side crops with real scaling; SURVEY §8(a) a4-a7,
 // a10, a11).
 //
-// A task is (up to 8 frames of ONE (clip slot, group), band of <= 32 output rows), as for k_plain;
+// A task is (up to 8 frames of ONE (clip slot, group), band of <= kMaxRB output rows), as for k_plain;
 // a CTA serves kFrames of its frames. Each frame is served by a FRAME GROUP of two warps that synchronise
 // only with each other (named barrier 1 + frame, 64 threads), never with the rest of the CTA:
 //   * the group stages its frame's source rows in QUADS (four Y rows from an even row and their
@@ -40,7 +40,8 @@ constexpr int kStages = SAND_PW_STAGES;   // NV12 row quads in flight per frame
 constexpr int kGWMax = SAND_PW_GWMAX;     // widest staged span (pixels); wider batches take k_plain
 constexpr int kRow = 4 * kGWMax;          // byte stride of the converted RGBx rows
 constexpr int kFrames = 2;                // frames per CTA (two warps each: 128 threads)
-constexpr uint32_t kTabBytes = 272;       // output-row table: 33 (y0, lambda) entries, sentinel last
+constexpr int kMaxRB = 64;                // output rows per band (task) at most
+constexpr uint32_t kTabBytes = (8u * (kMaxRB + 1) + 15u) & ~15u;   // output-row table + sentinel
 constexpr uint32_t kBarBytes = (8u * kStages + 15u) & ~15u;   // the stages' mbarriers
 
 struct Shape {
@@ -92,7 +93,7 @@ __global__ void __launch_bounds__(128, SAND_PW_MINB) k_plainw(const LaunchParams
   const uint32_t s_rgb = s_f;                                      // buffer b, row i at + (4b + i) kRow
   const uint32_t s_stage = s_f + 8u * pw::kRow;                    // stage s at + s stb: Y0..Y3, UV0, UV1
   const uint32_t s_bar = s_stage + pw::kStages * stb;              // mbarrier of stage s at + 8 s
-  const uint32_t s_tab = s_bar + pw::kBarBytes;                   // row table (33 x 8 B)
+  const uint32_t s_tab = s_bar + pw::kBarBytes;                   // row table (nr + 1 entries of 8 B)
 
   // staged column span [x16, x16 + gwi) of the whole frame row (monotone taps)
   const int x_lo = tap0(sc_x, off_x, 0, org_x);
@@ -104,22 +105,24 @@ __global__ void __launch_bounds__(128, SAND_PW_MINB) k_plainw(const LaunchParams
   if (gwi > sh.gw) __trap();                                       // host bound violated (never)
 
   // output-row table (warp 0 of the group): entry r = row Y0 + r's (y0, lambda); lambda 0 at the
-  // bottom clamp (y1 == y0), where the row is emitted from (H(y0), H(y0)): fmaf(0, h - h, h) == h
-  int ry0 = 0x7fffffff, ry1 = 0;
-  float rl = 0.f;
-  if (lane < nr) {
-    tap(sc_y, off_y, Y0 + lane, lim_y, org_y, ry0, ry1, rl);
-    if (ry1 == ry0) rl = 0.f;
-  }
+  // bottom clamp (y1 == y0), where the row is emitted from (H(y0), H(y0)): fmaf(0, h - h, h) == h;
+  // entry nr is a sentinel
   if (half == 0) {
-    if (lane < nr)
-      asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(s_tab + 8u * lane), "r"(ry0), "r"(__float_as_uint(rl))
-                   : "memory");
-    if (lane == (nr & 31))   // the sentinel after the last row (lane 0 when nr == 32)
-      asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(s_tab + 8u * nr), "r"(0x7fffffff), "r"(0u) : "memory");
+    for (int r = lane; r <= nr; r += 32) {
+      uint32_t e0 = 0x7fffffffu, e1 = 0u;
+      if (r < nr) {
+        int a, b;
+        float l;
+        tap(sc_y, off_y, Y0 + r, lim_y, org_y, a, b, l);
+        e0 = (uint32_t)a;
+        e1 = __float_as_uint(b == a ? 0.f : l);
+      }
+      asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(s_tab + 8u * r), "r"(e0), "r"(e1) : "memory");
+    }
   }
-  const int y_first = __shfl_sync(0xffffffffu, ry0, 0);
-  const int y_last = __shfl_sync(0xffffffffu, ry1, nr - 1);
+  const int y_first = tap0(sc_y, off_y, Y0, org_y);
+  int y_last;
+  tap(sc_y, off_y, Y0 + nr - 1, lim_y, org_y, dmy, y_last, fl);
   const int ybase = y_first & ~1;
   const int nquads = ((y_last - ybase) >> 2) + 1;
 

@@ -41,7 +41,7 @@ static int configure_plainw() {
 static int launch_plainw(const LaunchParams& p, const BatchShape& sh, int fpc, cudaStream_t stream, bool* launched) {
   *launched = false;
   if (!SAND_PLAINW || sh.n_tasks == 0 || sh.dtype < 0 || !sh.wo_mod4 || sh.max_wo > 256 || sh.pl_gw > pw::kGWMax ||
-      sh.pl_rb > 32 || fpc < 1 || sh.max_dests > 2)
+      sh.pl_rb > pw::kMaxRB || fpc < 1 || sh.max_dests > 2)
     return SAND_OK;
   pw::Shape s;
   s.nsub = (fpc + pw::kFrames - 1) / pw::kFrames;

@@ -108,7 +108,10 @@ struct BatchShape {
 };
 
 // k_plain task granularity (view.cpp builds the tasks, k_plain.cuh consumes them)
-constexpr int kPlainRB = 32;       // output rows per band
+#ifndef SAND_PLAIN_RB
+#define SAND_PLAIN_RB 64
+#endif
+constexpr int kPlainRB = SAND_PLAIN_RB;   // output rows per band
 constexpr int kPlainRBTail = 8;    // band of the tasks that make up the last part of the work
 constexpr double kPlainTailFrac = 0.25;
 
