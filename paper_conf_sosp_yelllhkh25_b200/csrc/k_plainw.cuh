@@ -267,7 +267,8 @@ __global__ void __launch_bounds__(128, SAND_PW_MINB) k_plainw(const LaunchParams
     }
   };
 
-  const int q4 = gwi >> 2;                          // 4-pixel groups per row
+  // 4-pixel groups of a row that any tap reads: [qlo, qlo + nq) (taps i0 in [x_lo, x_hi], i1 = i0 + 1)
+  const int qlo = (x_lo - x16) >> 2, nq = ((x_hi + 1 - x16) >> 2) - qlo + 1;
   for (int k = 0; k < nquads; ++k) {
     const int yq = ybase + 4 * k;
     const uint32_t stg = s_stage + (uint32_t)(k % pw::kStages) * stb;
@@ -275,9 +276,9 @@ __global__ void __launch_bounds__(128, SAND_PW_MINB) k_plainw(const LaunchParams
     st::mbar_wait_sleep(s_bar + 8u * (uint32_t)(k % pw::kStages), (uint32_t)(k / pw::kStages) & 1u);
     // conversion: units (UV row u, 4-pixel group q) over the group's 64 lanes; a unit converts
     // the two Y rows sharing UV row u (rows outside the band hold stale bytes: converted, unread)
-    const int units = yq + 2 <= y_last ? 2 * q4 : q4;  // UV row 1 of the last quad may be unused
+    const int units = yq + 2 <= y_last ? 2 * nq : nq;  // UV row 1 of the last quad may be unused
     for (int i = gt; i < units; i += 64) {
-      const int u = i >= q4 ? 1 : 0, q = i - u * q4;
+      const int u = i >= nq ? 1 : 0, q = qlo + i - u * nq;
       const uint32_t uv = st::lds32(stg + (uint32_t)(4 + u) * gw + 4u * q);
       const st::Chroma3 k0 = st::chroma_at<0>(uv, cm), k1 = st::chroma_at<16>(uv, cm);
       const uint32_t yt = st::lds32(stg + (uint32_t)(2 * u) * gw + 4u * q);

@@ -112,8 +112,14 @@ struct BatchShape {
 #define SAND_PLAIN_RB 64
 #endif
 constexpr int kPlainRB = SAND_PLAIN_RB;   // output rows per band
-constexpr int kPlainRBTail = 8;    // band of the tasks that make up the last part of the work
-constexpr double kPlainTailFrac = 0.25;
+#ifndef SAND_PLAIN_RB_TAIL
+#define SAND_PLAIN_RB_TAIL 16
+#endif
+#ifndef SAND_PLAIN_TAIL_FRAC
+#define SAND_PLAIN_TAIL_FRAC 0.25
+#endif
+constexpr int kPlainRBTail = SAND_PLAIN_RB_TAIL;   // band of the tasks that make up the last part of the work
+constexpr double kPlainTailFrac = SAND_PLAIN_TAIL_FRAC;
 
 // k_plain task word: frames | band rows << 8 | first output row << 20
 SAND_HD inline uint32_t pl_task_y(uint32_t nfr, uint32_t nr, uint32_t y0) { return nfr | (nr << 8) | (y0 << 20); }
