@@ -104,7 +104,10 @@ def measured_peaks():
 
 # kernel of each item class (SAND_N_CLASSES: mild plain, heavy plain, rotation/blur); the roofline's
 # subject is the class with the most kernel time, its bytes / its own event-timed duration
+# kernel of each item class (plain mild, heavy, stencil) per config: the mild class runs k_plainw
+# (k_plain only for views wider than 256 / spans beyond 384 px), identity-scale batches k_copy
 CLASS_KERNELS = {"slowfast": ("k_copy", "k_direct", "k_stencil2")}
+DEFAULT_CLASS_KERNELS = ("k_plainw", "k_direct", "k_stencil2")
 
 
 def ncu_record(config: str):
@@ -400,7 +403,7 @@ def run_sand(args):
     # per-kernel roofline: each item class is its own kernel; time each class with
     # CUDA events recorded by the library around its launch, on the stream it runs on, over a
     # separate pass of the same batches (so the timed loop above carries no timing events)
-    cls_names = CLASS_KERNELS.get(args.config, ("k_plain", "k_direct", "k_stencil2"))
+    cls_names = CLASS_KERNELS.get(args.config, DEFAULT_CLASS_KERNELS)
     view.set_timing(True)
     n_cls_steps = min(args.steps, 200)
     s_cls = first_timed
