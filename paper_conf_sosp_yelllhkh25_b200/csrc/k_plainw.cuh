@@ -72,6 +72,9 @@ __global__ void __launch_bounds__(128, SAND_PW_MINB) k_plainw(const LaunchParams
   using namespace rs;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int fr = warp >> 1, half = warp & 1, gt = threadIdx.x & 63;   // frame, half, thread in group
+  // the next batch's kernel may launch once every CTA of this one is resident: its prologue then
+  // overlaps this grid's tail (it waits for this grid before touching frames or outputs)
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   const int task = (int)blockIdx.x / sh.nsub, sub = (int)blockIdx.x - task * sh.nsub;
   const uint2 tk = tasks[task];
   const int nfr = (int)(tk.y & 0xffu), nr = (int)((tk.y >> 8) & 0xfffu), Y0 = (int)(tk.y >> 20);
@@ -152,8 +155,6 @@ __global__ void __launch_bounds__(128, SAND_PW_MINB) k_plainw(const LaunchParams
       for (int s = 0; s < pw::kStages; ++s) st::mbar_init(s_bar + 8u * s, 1);
       asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    __syncwarp();
-    for (int k = 0; k < min(nquads, pw::kStages); ++k) stage(k);
   }
 
   // column taps of the lane's pairs: shared addresses of tap i0 in RGBx row 0 of the current
@@ -199,6 +200,15 @@ __global__ void __launch_bounds__(128, SAND_PW_MINB) k_plainw(const LaunchParams
       dl[d].b[c] = e.b[c];
     }
     dl[d].rstride = e.rstride;
+  }
+
+  // Programmatic dependent launch (mat_plain.cu): everything above reads only this batch's plan
+  // (uploaded and ordered before the launch); frames and outputs are touched only after the
+  // previous kernel on the stream has completed (a no-op when the launch is not programmatic)
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  if (half == 0) {
+    __syncwarp();
+    for (int k = 0; k < min(nquads, pw::kStages); ++k) stage(k);
   }
 
   Row3 X[NPJ], Yr[NPJ];                                            // lerps of even / odd source rows

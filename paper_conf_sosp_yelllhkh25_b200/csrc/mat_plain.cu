@@ -35,6 +35,28 @@ static int configure_plainw() {
   return SAND_OK;
 }
 
+#ifndef SAND_PW_PDL
+#define SAND_PW_PDL 1
+#endif
+// launch with programmatic stream serialisation: consecutive batches' kernels on one stream overlap
+// the next grid's prologue with this grid's tail (k_plainw waits on the previous grid before it
+// touches frames or outputs)
+template <typename K>
+static void launch_pdl(K kernel, unsigned grid, unsigned threads, size_t smem, cudaStream_t stream,
+                       const LaunchParams& p, const uint2* tasks, const pw::Shape& s) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(threads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = SAND_PW_PDL;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  (void)cudaLaunchKernelEx(&cfg, kernel, p, tasks, s);   // errors surface via cudaGetLastError
+}
+
 // k_plainw: one warp per frame of a task (k_plainw.cuh); *launched = false when the batch does
 // not fit it (mixed dtypes, widths not a multiple of 4 or > 256, spans beyond kGWMax, items with
 // more than two destinations)
@@ -57,20 +79,20 @@ static int launch_plainw(const LaunchParams& p, const BatchShape& sh, int fpc, c
   do {                                                                                                       \
     switch (sh.dtype) {                                                                                      \
       case SAND_U8:                                                                                          \
-        if (nd1) k_plainw<SAND_U8, 1, NPJ, false><<<grid, threads, smem, stream>>>(p, tasks, s);       \
-        else k_plainw<SAND_U8, 2, NPJ, false><<<grid, threads, smem, stream>>>(p, tasks, s);           \
+        if (nd1) launch_pdl(k_plainw<SAND_U8, 1, NPJ, false>, grid, threads, smem, stream, p, tasks, s);       \
+        else launch_pdl(k_plainw<SAND_U8, 2, NPJ, false>, grid, threads, smem, stream, p, tasks, s);           \
         break;                                                                                               \
       case SAND_BF16:                                                                                        \
-        if (fold && nd1) k_plainw<SAND_BF16, 1, NPJ, true><<<grid, threads, smem, stream>>>(p, tasks, s);  \
-        else if (fold) k_plainw<SAND_BF16, 2, NPJ, true><<<grid, threads, smem, stream>>>(p, tasks, s);    \
-        else if (nd1) k_plainw<SAND_BF16, 1, NPJ, false><<<grid, threads, smem, stream>>>(p, tasks, s);    \
-        else k_plainw<SAND_BF16, 2, NPJ, false><<<grid, threads, smem, stream>>>(p, tasks, s);             \
+        if (fold && nd1) launch_pdl(k_plainw<SAND_BF16, 1, NPJ, true>, grid, threads, smem, stream, p, tasks, s);  \
+        else if (fold) launch_pdl(k_plainw<SAND_BF16, 2, NPJ, true>, grid, threads, smem, stream, p, tasks, s);    \
+        else if (nd1) launch_pdl(k_plainw<SAND_BF16, 1, NPJ, false>, grid, threads, smem, stream, p, tasks, s);    \
+        else launch_pdl(k_plainw<SAND_BF16, 2, NPJ, false>, grid, threads, smem, stream, p, tasks, s);             \
         break;                                                                                               \
       default:                                                                                               \
-        if (fold && nd1) k_plainw<SAND_F32, 1, NPJ, true><<<grid, threads, smem, stream>>>(p, tasks, s);   \
-        else if (fold) k_plainw<SAND_F32, 2, NPJ, true><<<grid, threads, smem, stream>>>(p, tasks, s);     \
-        else if (nd1) k_plainw<SAND_F32, 1, NPJ, false><<<grid, threads, smem, stream>>>(p, tasks, s);     \
-        else k_plainw<SAND_F32, 2, NPJ, false><<<grid, threads, smem, stream>>>(p, tasks, s);              \
+        if (fold && nd1) launch_pdl(k_plainw<SAND_F32, 1, NPJ, true>, grid, threads, smem, stream, p, tasks, s);   \
+        else if (fold) launch_pdl(k_plainw<SAND_F32, 2, NPJ, true>, grid, threads, smem, stream, p, tasks, s);     \
+        else if (nd1) launch_pdl(k_plainw<SAND_F32, 1, NPJ, false>, grid, threads, smem, stream, p, tasks, s);     \
+        else launch_pdl(k_plainw<SAND_F32, 2, NPJ, false>, grid, threads, smem, stream, p, tasks, s);              \
         break;                                                                                               \
     }                                                                                                        \
   } while (0)
