@@ -365,7 +365,11 @@ def run_sand(args):
     start.record(stream)
     for i in range(args.steps):
         e, it = step_id(s)
+        if args.step_events:
+            kstart[i].record(stream)
         view.read_batch(e, rank, it, outs_a if s % 2 == 0 else outs_b, stream.cuda_stream)
+        if args.step_events:
+            kend[i].record(stream)
         s += 1
     end.record(stream)
     torch.cuda.synchronize()
@@ -648,6 +652,8 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=16)
     ap.add_argument("--pool-epochs", type=int, default=0, help="k-epoch shared frame pool (f1, R#25)")
     ap.add_argument("--object-budget-gb", type=float, default=0.0, help="HBM object cache (f2, R#27)")
+    ap.add_argument("--step-events", action="store_true",
+                    help="diagnostics: record per-step CUDA events inside the timed loop")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend (gloo: test mode, ranks may share one GPU)")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)

@@ -46,8 +46,12 @@ def main():
         r, n = a.split(":")
         lo, hi = r.split("-")
         ranges.append((int(lo), int(hi), n))
-    txt = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
-                         capture_output=True, text=True).stdout
+    if rep.endswith(".csv.gz"):      # a saved `--page source --print-source sass --csv` export
+        import gzip
+        txt = gzip.open(rep, "rt").read()
+    else:
+        txt = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
+                             capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(txt)))
     hdr, blk, cur = None, None, None
     for r in rows:
