@@ -128,19 +128,21 @@ __global__ void __launch_bounds__(256, SAND_DIRECT_MINB) k_direct(const LaunchPa
     {
       uint32_t Yc[2][4], UVc[2][4];
       float lyc;
+      // unsigned 32-bit column offsets (no sign extension in the 64-bit address arithmetic)
+      const uint32_t xs[4] = {(uint32_t)xa0, (uint32_t)xa1, (uint32_t)xb0, (uint32_t)xb1};
+      const uint32_t xuv[4] = {xs[0] & ~1u, xs[1] & ~1u, xs[2] & ~1u, xs[3] & ~1u};
       auto load_row = [&](int oy, uint32_t (&Yv)[2][4], uint32_t (&UVv)[2][4], float& ly) {
         int y0, y1;
         tap(g.sc_y, g.off_y, oy, g.lim_y, g.org_y, y0, y1, ly);
-        const int xs[4] = {xa0, xa1, xb0, xb1};
-        const int ys[2] = {y0, y1};
+        const uint32_t ys[2] = {(uint32_t)y0, (uint32_t)y1};
 #pragma unroll
         for (int r = 0; r < 2; ++r) {
-          const uint8_t* yr = Yp + (size_t)ys[r] * pitch;
-          const uint8_t* uvr = UVp + (size_t)(ys[r] >> 1) * pitch;
+          const uint8_t* yr = Yp + (size_t)(ys[r] * pitch);          // frame offsets fit 32 bits
+          const uint8_t* uvr = UVp + (size_t)((ys[r] >> 1) * pitch);
 #pragma unroll
           for (int k = 0; k < 4; ++k) {
             Yv[r][k] = __ldg(yr + xs[k]);
-            UVv[r][k] = __ldg(reinterpret_cast<const uint16_t*>(uvr + (xs[k] & ~1)));
+            UVv[r][k] = __ldg(reinterpret_cast<const uint16_t*>(uvr + xuv[k]));
           }
         }
       };

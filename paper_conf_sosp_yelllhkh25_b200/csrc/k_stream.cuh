@@ -131,9 +131,11 @@ struct Chroma3 {
 };
 template <int SHIFT>
 __device__ __forceinline__ Chroma3 chroma_at(uint32_t uv, const ColorM& m) {
-  const int u = (int)((uv >> SHIFT) & 0xffu) - 128;
-  const int v = (int)((uv >> (SHIFT + 8)) & 0xffu) - 128;
-  return {m.vr * v, m.vg * v + m.ug * u, m.ub * u};
+  // raw bytes U, V (one PRMT each); the -128 offsets are folded into the IMAD addends:
+  // vr (V - 128) = vr V + kr etc. (exact integer arithmetic)
+  const int u = (int)__byte_perm(uv, 0u, 0x4440 | (SHIFT / 8));
+  const int v = (int)__byte_perm(uv, 0u, 0x4440 | (SHIFT / 8 + 1));
+  return {m.vr * v + m.kr, m.vg * v + (m.ug * u + m.kg), m.ub * u + m.kb};
 }
 
 // RGBx word of luma Y with chroma c: sat((yy + term) >> 20) per channel (OpenCV integer

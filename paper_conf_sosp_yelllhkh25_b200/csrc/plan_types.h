@@ -139,11 +139,15 @@ SAND_HD inline void tap_ref(float sc, int off, int o, int lim, int org, int* i0,
 // B = sat((yy + ub u) >> 20), u = U - 128, v = V - 128
 struct ColorM {
   int32_t cy, vr, vg, ug, ub;
-  int32_t yk;   // 2^19 - 16 cy: yy = max(Y, 16) cy + yk in one IMAD
+  int32_t yk;           // 2^19 - 16 cy: yy = max(Y, 16) cy + yk in one IMAD
+  int32_t kr, kg, kb;   // -128 x (vr, vg + ug, ub): the chroma terms from the raw U, V bytes
 };
+SAND_HD inline ColorM color_matrix_of(int32_t cy, int32_t vr, int32_t vg, int32_t ug, int32_t ub) {
+  return ColorM{cy, vr, vg, ug, ub, (1 << 19) - 16 * cy, -128 * vr, -128 * (vg + ug), -128 * ub};
+}
 SAND_HD inline ColorM color_matrix(int32_t m) {
-  return m == 1 ? ColorM{1220945, 1879825, -558796, -223607, 2215014, (1 << 19) - 16 * 1220945}   // BT.709 (R#29)
-                : ColorM{1220542, 1673527, -852492, -409993, 2116026, (1 << 19) - 16 * 1220542};  // BT.601 (R#11)
+  return m == 1 ? color_matrix_of(1220945, 1879825, -558796, -223607, 2215014)    // BT.709 from Kr, Kb (R#29)
+                : color_matrix_of(1220542, 1673527, -852492, -409993, 2116026);  // BT.601, OpenCV (R#11)
 }
 
 struct LaunchParams {
