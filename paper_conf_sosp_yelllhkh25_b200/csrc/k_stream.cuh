@@ -145,18 +145,10 @@ __device__ __forceinline__ Chroma3 chroma_at(uint32_t uv, const ColorM& m) {
 __device__ __forceinline__ uint32_t rgbx_dpx(uint32_t Y, const Chroma3& c, const ColorM& m) {
   const int yy = (int)max(Y, 16u) * m.cy + m.yk;
   // x >> 4 of the clamped sums as IMAD.HI (FMA pipe) to relieve the ALU pipe
-#if SAND_RGBX_IMAD
-  // channel bytes as x >> 20 (IMAD.HI) packed by IMADs: FMA-pipe work instead of ALU PRMTs
-  const uint32_t R = __umulhi((uint32_t)__viaddmin_s32_relu(yy, c.r, 0x0FFFFFFF), 1u << 12);
-  const uint32_t G = __umulhi((uint32_t)__viaddmin_s32_relu(yy, c.g, 0x0FFFFFFF), 1u << 12);
-  const uint32_t B = __umulhi((uint32_t)__viaddmin_s32_relu(yy, c.b, 0x0FFFFFFF), 1u << 12);
-  return B * 65536u + (G * 256u + (R + 0x4B000000u));
-#else
   const uint32_t mr = __umulhi((uint32_t)__viaddmin_s32_relu(yy, c.r, 0x0FFFFFFF), 1u << 28);
   const uint32_t mg = __umulhi((uint32_t)__viaddmin_s32_relu(yy, c.g, 0x0FFFFFFF), 1u << 28);
   const uint32_t mb = __umulhi((uint32_t)__viaddmin_s32_relu(yy, c.b, 0x0FFFFFFF), 1u << 28) + 0x4B000000u;
   return __byte_perm(__byte_perm(mr, mg, 0x0062), mb, 0x7610);
-#endif
 }
 
 // byte I of w, zero-extended (one PRMT)
