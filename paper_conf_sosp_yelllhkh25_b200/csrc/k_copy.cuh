@@ -31,7 +31,9 @@ __device__ __forceinline__ void px(uint32_t Y, const st::Chroma3& k, uint32_t (&
 #endif
 constexpr int kCopyUnroll = SAND_COPY_UNROLL;   // rows in flight per thread (load latency)
 
-template <int DT>
+// FOLD: the destinations' b fields hold b' = b - 2^23 a (ViewConst::fold): the biased pixel
+// 2^23 + q is normalised directly, fmaf(2^23 + q, a, b') == fmaf(q, a, b) exactly
+template <int DT, bool FOLD>
 __global__ void __launch_bounds__(256) k_copy(const LaunchParams p, int RB, int nbands) {
   using namespace rs;
   const int item_idx = blockIdx.x / nbands;
@@ -56,8 +58,8 @@ __global__ void __launch_bounds__(256) k_copy(const LaunchParams p, int RB, int 
   const int nd = (int)w.n_dest;
   const uint32_t* dests = p.dests + w.dest_begin;
   // the first two destinations in registers, advanced per row (a third and later: rare)
-  Dest dl0 = make_dest(p, dests[0], y_begin + r0, ox), dl1 = dl0;
-  if (nd > 1) dl1 = make_dest(p, dests[1], y_begin + r0, ox);
+  Dest dl0 = make_dest(p, dests[0], y_begin + r0, ox, FOLD), dl1 = dl0;
+  if (nd > 1) dl1 = make_dest(p, dests[1], y_begin + r0, ox, FOLD);
 #pragma unroll (kCopyUnroll)
   for (int oy = y_begin + r0; oy < y_end; oy += rpi) {
     const int sy = sy0 + oy;
@@ -101,7 +103,7 @@ __global__ void __launch_bounds__(256) k_copy(const LaunchParams p, int RB, int 
       }
     }
     for (int d = 0; d < nd; ++d) {
-      const Dest e = d == 0 ? dl0 : (d == 1 ? dl1 : make_dest(p, dests[d], oy, ox));
+      const Dest e = d == 0 ? dl0 : (d == 1 ? dl1 : make_dest(p, dests[d], oy, ox, FOLD));
 #pragma unroll
       for (int ch = 0; ch < 3; ++ch) {
         const uint32_t t0 = c[0][ch], t1 = c[1][ch], t2 = c[2][ch], t3 = c[3][ch];
@@ -111,8 +113,8 @@ __global__ void __launch_bounds__(256) k_copy(const LaunchParams p, int RB, int 
               __byte_perm(__byte_perm(t0, t1, 0x0040), __byte_perm(t2, t3, 0x0040), 0x5410);
         } else {
           const uint64_t a2 = f2::splat(e.a[ch]), b2 = f2::splat(e.b[ch]);
-          const uint64_t q01 = f2::add(f2::pack(t0, t1), f2::splat(-kBias));   // exact q
-          const uint64_t q23 = f2::add(f2::pack(t2, t3), f2::splat(-kBias));
+          const uint64_t q01 = FOLD ? f2::pack(t0, t1) : f2::add(f2::pack(t0, t1), f2::splat(-kBias));   // (2^23 +) q
+          const uint64_t q23 = FOLD ? f2::pack(t2, t3) : f2::add(f2::pack(t2, t3), f2::splat(-kBias));
           const uint64_t y01 = f2::fma(q01, a2, b2), y23 = f2::fma(q23, a2, b2);   // fmaf(q, a_c, b_c)
           if constexpr (DT == SAND_BF16) {
             const __nv_bfloat162 v0 = __floats2bfloat162_rn(f2::lof(y01), f2::hif(y01));

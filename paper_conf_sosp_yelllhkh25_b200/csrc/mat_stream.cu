@@ -28,10 +28,17 @@ int launch_copy(const LaunchParams& p, const BatchShape& sh, cudaStream_t stream
   constexpr int RB = 32;
   const int nbands = (sh.max_ho + RB - 1) / RB;
   const unsigned blocks = (unsigned)((uint64_t)p.n_items * nbands);
+  const bool fold = sh.fold != 0;   // normalisation folds the rint bias (ViewConst::fold)
   switch (sh.dtype) {
-    case SAND_U8: k_copy<SAND_U8><<<blocks, threads, 0, stream>>>(p, RB, nbands); break;
-    case SAND_BF16: k_copy<SAND_BF16><<<blocks, threads, 0, stream>>>(p, RB, nbands); break;
-    default: k_copy<SAND_F32><<<blocks, threads, 0, stream>>>(p, RB, nbands); break;
+    case SAND_U8: k_copy<SAND_U8, false><<<blocks, threads, 0, stream>>>(p, RB, nbands); break;
+    case SAND_BF16:
+      if (fold) k_copy<SAND_BF16, true><<<blocks, threads, 0, stream>>>(p, RB, nbands);
+      else k_copy<SAND_BF16, false><<<blocks, threads, 0, stream>>>(p, RB, nbands);
+      break;
+    default:
+      if (fold) k_copy<SAND_F32, true><<<blocks, threads, 0, stream>>>(p, RB, nbands);
+      else k_copy<SAND_F32, false><<<blocks, threads, 0, stream>>>(p, RB, nbands);
+      break;
   }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_error(e, "k_copy launch");
