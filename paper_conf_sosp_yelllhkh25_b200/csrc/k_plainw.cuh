@@ -37,7 +37,8 @@ constexpr int kStages = SAND_PW_STAGES;   // NV12 row quads in flight per frame
 #ifndef SAND_PW_GWMAX
 #define SAND_PW_GWMAX 384
 #endif
-constexpr int kGWMax = SAND_PW_GWMAX;     // widest staged span (pixels); wider batches take k_plain
+constexpr int kGWMax = SAND_PW_GWMAX;     // widest staged span (pixels); wider tasks take k_plain
+static_assert(kGWMax == kPlainwMaxSpan, "the host partitions tasks at kPlainwMaxSpan");
 constexpr int kRow = 4 * kGWMax;          // byte stride of the converted RGBx rows
 constexpr int kFrames = 2;                // frames per CTA (two warps each: 128 threads)
 constexpr int kMaxRB = 64;                // output rows per band (task) at most

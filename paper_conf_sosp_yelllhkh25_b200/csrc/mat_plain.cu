@@ -62,19 +62,19 @@ static void launch_pdl(K kernel, unsigned grid, unsigned threads, size_t smem, c
 // more than two destinations)
 static int launch_plainw(const LaunchParams& p, const BatchShape& sh, int fpc, cudaStream_t stream, bool* launched) {
   *launched = false;
-  if (!SAND_PLAINW || sh.n_tasks == 0 || sh.dtype < 0 || !sh.wo_mod4 || sh.max_wo > 256 || sh.pl_gw > pw::kGWMax ||
+  if (!SAND_PLAINW || sh.n_tasks_w == 0 || sh.dtype < 0 || !sh.wo_mod4 || sh.max_wo > 256 || sh.pl_gw_w > pw::kGWMax ||
       sh.pl_rb > pw::kMaxRB || fpc < 1 || sh.max_dests > 2)
     return SAND_OK;
   pw::Shape s;
   s.nsub = (fpc + pw::kFrames - 1) / pw::kFrames;
-  s.gw = sh.pl_gw;
+  s.gw = sh.pl_gw_w;
   const size_t smem = pw::smem_bytes(s);
   if (smem > 200 * 1024) return SAND_OK;
   const uint2* tasks = p.tasks + sh.task_first;
   const bool nd1 = sh.max_dests <= 1, fold = sh.fold != 0 && sh.dtype != SAND_U8;
   const bool narrow = sh.max_wo <= 128;
   const unsigned threads = 64u * pw::kFrames;
-  const unsigned grid = sh.n_tasks * (unsigned)s.nsub;
+  const unsigned grid = sh.n_tasks_w * (unsigned)s.nsub;   // the k_plainw-eligible tasks (first)
 #define SAND_PW_GO(NPJ)                                                                                     \
   do {                                                                                                       \
     switch (sh.dtype) {                                                                                      \
@@ -116,9 +116,27 @@ int configure_plain() {
   return SAND_OK;
 }
 
-int launch_plain(const LaunchParams& p, const BatchShape& sh, int fpc, int nq, cudaStream_t stream, bool* launched) {
+static int launch_plain_tasks(const LaunchParams& p, const BatchShape& sh, int fpc, int nq, cudaStream_t stream,
+                              bool* launched);
+
+int launch_plain(const LaunchParams& p, const BatchShape& sh_in, int fpc, int nq, cudaStream_t stream, bool* launched) {
   *launched = false;
-  if (int rc = launch_plainw(p, sh, fpc, stream, launched); rc != SAND_OK || *launched) return rc;
+  BatchShape sh = sh_in;
+  if (int rc = launch_plainw(p, sh, fpc, stream, launched); rc != SAND_OK) return rc;
+  if (*launched) {                      // k_plainw took the eligible tasks; k_plain the wider rest
+    if (sh.n_tasks_w == sh.n_tasks) return SAND_OK;
+    sh.task_first += sh.n_tasks_w;
+    sh.n_tasks -= sh.n_tasks_w;
+    *launched = false;   // if k_plain declines them too, the generic kernel redoes the whole class
+    return launch_plain_tasks(p, sh, fpc, nq, stream, launched);
+  }
+  return launch_plain_tasks(p, sh, fpc, nq, stream, launched);
+}
+
+// k_plain over the tasks [task_first, task_first + n_tasks) of the batch
+static int launch_plain_tasks(const LaunchParams& p, const BatchShape& sh, int fpc, int nq, cudaStream_t stream,
+                              bool* launched) {
+  *launched = false;
   if (sh.n_tasks == 0 || sh.dtype < 0 || (kNP == 2 ? !sh.wo_mod4 : !sh.even_wo)) return SAND_OK;
   pl::Shape s;
   s.fpc = fpc;

@@ -103,6 +103,10 @@ struct BatchShape {
   // k_plain: the batch's task slice, the widest staged span (pixels) and the longest band
   uint32_t task_first, n_tasks;
   int32_t pl_gw, pl_rb;
+  // the tasks are ordered k_plainw-eligible first (staged span <= kPlainwMaxSpan): the first
+  // n_tasks_w of them with widest span pl_gw_w; the rest (wider spans) go to k_plain
+  uint32_t n_tasks_w;
+  int32_t pl_gw_w;
   int32_t fold;             // every view's normalisation folds the rint bias (ViewConst::fold)
   int32_t has_jitter;       // a stencil item applies colour jitter (k_stencil2 only, R#30)
 };
@@ -120,6 +124,8 @@ constexpr int kPlainRB = SAND_PLAIN_RB;   // output rows per band
 #endif
 constexpr int kPlainRBTail = SAND_PLAIN_RB_TAIL;   // band of the tasks that make up the last part of the work
 constexpr double kPlainTailFrac = SAND_PLAIN_TAIL_FRAC;
+
+constexpr int kPlainwMaxSpan = 384;   // widest staged span k_plainw takes (k_plainw.cuh kGWMax)
 
 // k_plain task word: frames | band rows << 8 | first output row << 20
 SAND_HD inline uint32_t pl_task_y(uint32_t nfr, uint32_t nr, uint32_t y0) { return nfr | (nr << 8) | (y0 << 20); }

@@ -180,15 +180,26 @@ void plain_tasks(const std::vector<WorkItem>& items, size_t first, size_t n, con
   std::reverse(big.begin(), big.end());
   std::stable_sort(tail.begin(), tail.end(), [](const T& a, const T& b) { return a.cost > b.cost; });
   shape->task_first = (uint32_t)out->size();
-  shape->pl_gw = shape->pl_rb = 0;
-  for (const auto* v : {&big, &tail})
-    for (const T& t : *v) {
-      const GroupParams& g = groups[items[first + t.item].gp];
-      shape->pl_gw = std::max(shape->pl_gw, span16(g));
-      shape->pl_rb = std::max(shape->pl_rb, (int)t.nr);
-      out->push_back(make_uint2(t.item, pl_task_y(t.nfr, t.nr, t.y0)));
-    }
+  shape->pl_gw = shape->pl_rb = shape->pl_gw_w = 0;
+  // per task (not per batch maximum): tasks whose span k_plainw can stage first, then the rest
+  for (int wide = 0; wide < 2; ++wide)
+    for (const auto* v : {&big, &tail})
+      for (const T& t : *v) {
+        const GroupParams& g = groups[items[first + t.item].gp];
+        const int span = span16(g);
+        if ((span > kPlainwMaxSpan) != (wide == 1)) continue;
+        shape->pl_gw = std::max(shape->pl_gw, span);
+        if (!wide) shape->pl_gw_w = std::max(shape->pl_gw_w, span);
+        shape->pl_rb = std::max(shape->pl_rb, (int)t.nr);
+        out->push_back(make_uint2(t.item, pl_task_y(t.nfr, t.nr, t.y0)));
+      }
   shape->n_tasks = (uint32_t)out->size() - shape->task_first;
+  shape->n_tasks_w = 0;
+  for (uint32_t i = shape->task_first; i < (uint32_t)out->size(); ++i) {
+    const WorkItem& w = items[first + (*out)[i].x];
+    if (span16(groups[w.gp]) > kPlainwMaxSpan) break;
+    shape->n_tasks_w++;
+  }
 }
 
 }  // namespace
