@@ -134,8 +134,9 @@ __global__ void __launch_bounds__(128, SAND_PW_MINB) k_plainw(const LaunchParams
   const uint8_t* uvsrc = ysrc + (size_t)w.pitch * w.src_h;         // column x16 of UV row 0
   const uint32_t pitch = w.pitch;
   // quad k (Y rows ybase + 4k .. + 3 inside [y_first, y_last] and their UV rows) -> stage
-  // k % kStages; warp 0 of the group, lanes 0..5 one row copy each (the mbarrier's tx-count
-  // may go transiently negative before lane 0's expect)
+  // k % kStages by one warp of the group (the first kStages quads: warp 0; then the warps take
+  // turns), lanes 0..5 one row copy each (the mbarrier's tx-count may go transiently negative
+  // before lane 0's expect)
   auto stage = [&](int k) {
     const int yq = ybase + 4 * k;
     const int ya = max(yq, y_first), yb = min(yq + 3, y_last);
